@@ -1,0 +1,375 @@
+/*
+ * proact_device.cuh -- device side of libproact (sm_100a).
+ *
+ * What a producer kernel uses instead of the paper's compiler pass (Sec. IV-A,
+ * L172-L176, Listing 1 user_kernel_decoupled L198-L219):
+ *
+ *   __global__ void k(proact::launch_ctx lc, Params p) {
+ *       if (proact::agent_dispatch(lc)) return;            // agent CTAs run the transfer loop
+ *       for (tile = proact::producer_block(lc); tile < ntiles; tile += proact::producer_grid(lc)) {
+ *           ... proact::wait_range(lc, in_region, off, bytes) ...  // consumer wait (a7), 1 thread
+ *           ... proact::put(lc, out_region, byte_off, value) ...   // instrumented store (a2)
+ *           __syncthreads();
+ *           if (threadIdx.x == 0) proact::commit_span(lc, out_region, tile_off, tile_bytes); // a3
+ *       }
+ *   }
+ *
+ * Host side: proact_launch() fills `lc` (include/proact.h).
+ *
+ * Memory-model protocol (PTX ISA memory consistency model; DESIGN.md Sec. "Ordering"):
+ *   producer  weak stores -> bar.sync -> atom.add.release.gpu(counter[c], bytes)         (a2, a3)
+ *   agent     ld.acquire.gpu(counter[c]) == expected[c] -> __syncwarp -> ld.global.cg data
+ *             -> st.global.v4 to every peer mirror -> __syncwarp -> fence.acq_rel.sys
+ *             -> st.relaxed.sys arrive_peer[gchunk] = gen<<1|changed                    (a4-a6)
+ *   consumer  ld.acquire.sys(arrive[gchunk]) >= gen -> bar.sync -> plain loads          (a7)
+ *   credits   kernel end -> sync kernel: fence.acq_rel.sys -> st peer_done[me] = e+1;
+ *             agents wait ld.acquire.sys(done[p]) >= e before overwriting p's replica   (a8)
+ * The paper's counters count writer CTAs down to zero (L127-L129); here they count BYTES up to
+ * expected[c] (reading R1), which needs no block-to-chunk mapping table (Listing 1)
+ * and detects over-counting.  The last arriver is decided from the atomic's return value, never
+ * by re-reading (Listing 1 L207-L208 re-reads counter[chunk], a race; reading R2).
+ */
+#ifndef PROACT_DEVICE_CUH
+#define PROACT_DEVICE_CUH
+
+#include <stdint.h>
+#include "proact.h"
+
+namespace proact {
+
+/* ---------------------------------------------------------------- shared layouts ----------- */
+/* These structs are written by the host runtime (csrc/runtime.cpp) into device memory. */
+
+struct region_dev {
+    char *base;                 /* local full-extent replica */
+    uint64_t own_off;           /* my slice [own_off, own_off + own_bytes) */
+    uint64_t own_bytes;
+    uint64_t total_bytes;
+    uint32_t chunk_bytes;
+    uint32_t n_own;             /* my chunks */
+    uint32_t chunk0;            /* global id of my first chunk */
+    uint32_t n_total;           /* global chunks */
+    uint32_t n_in;              /* chunks pushed INTO me per generation (wait_all); ~0u = n/a */
+    uint32_t flags;             /* PROACT_REGION_* */
+    uint64_t dest_mask;         /* default destinations of my chunks */
+    uint32_t *counter;          /* [n_own] bytes committed this generation (a3) */
+    uint32_t *expected;         /* [n_own] bytes of each chunk */
+    uint32_t *piecedone;        /* [n_own] agent pieces finished this generation */
+    uint32_t *changed_gen;      /* [n_own] generation in which the chunk's data changed */
+    uint32_t *push_gen;         /* [n_own] generation in which the chunk must be pushed (SPARSE) */
+    uint32_t *chunk_dest;       /* [n_own] per-chunk destination override, or nullptr */
+    uint32_t *arrive;           /* [n_total] consumer-side flags: gen << 1 | changed */
+    uint32_t *arrive_count;     /* monotonic count of chunks that arrived from peers */
+    uint32_t *deliv;            /* debug: [n_own * world] deliveries, or nullptr */
+    uint64_t rank_off[PROACT_MAX_RANKS + 1];
+    uint32_t rank_chunk0[PROACT_MAX_RANKS + 1];
+    char *peer_base[PROACT_MAX_RANKS];            /* peers' replica bases (mapped) */
+    uint32_t *peer_arrive[PROACT_MAX_RANKS];      /* peers' arrive[] */
+    uint32_t *peer_arrive_count[PROACT_MAX_RANKS];
+};
+
+struct dev_ctx {
+    int32_t rank;
+    int32_t world;
+    uint64_t watchdog_ns;
+    uint32_t *done;                            /* [world] credits from peers: (epoch+1)<<1|vote */
+    uint32_t *peer_done[PROACT_MAX_RANKS];     /* peers' done[] */
+    uint32_t *err;                             /* device error word (atomics) */
+    uint32_t *err_host;                        /* host-mapped mirror (plain stores) */
+    uint32_t *vote;                            /* [2] local vote words, by epoch parity */
+    uint32_t *vote_host;                       /* host-mapped: (epoch+1)<<1 | global vote */
+    region_dev region[PROACT_MAX_REGIONS];
+};
+
+/* Passed BY VALUE as the first kernel parameter; filled by proact_launch. */
+struct launch_ctx {
+    const dev_ctx *ctx;
+    uint32_t epoch;                            /* phase index on this rank */
+    uint32_t armed;                            /* bit r: region r written by this launch */
+    uint32_t gen[PROACT_MAX_REGIONS];          /* armed: generation produced now; else current */
+    uint32_t gen_epoch[PROACT_MAX_REGIONS];    /* epoch that produced gen[r] */
+    uint16_t mech;                             /* PROACT_MECH_* */
+    uint16_t push;                             /* PROACT_PUSH_* */
+    uint16_t agent_ctas;                       /* leading CTAs that run the agent (FUSED/ELIDE) */
+    uint16_t agent_warps;                      /* warps of those CTAs that poll/push */
+    uint32_t piece_bytes;                      /* agent work unit */
+    uint32_t flags;                            /* reserved */
+};
+
+/* error word encoding: (site << 8) | (-PROACT_ERR_*) */
+enum { SITE_AGENT_POLL = 1, SITE_AGENT_CREDIT = 2, SITE_WAIT_RANGE = 3, SITE_WAIT_ALL = 4,
+       SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7 };
+
+#ifdef __CUDACC__
+
+/* ---------------------------------------------------------------- PTX wrappers ------------- */
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_sys(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_sys(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t atom_add_release_gpu(uint32_t *p, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.release.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ uint32_t atom_add_acqrel_gpu(uint32_t *p, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ void red_add_relaxed_sys(uint32_t *p, uint32_t v)
+{
+    asm volatile("red.relaxed.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ uint4 ld_cg_v4(const uint4 *p)
+{
+    uint4 v;
+    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ void st_v4(uint4 *p, uint4 v)
+{
+    asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+__device__ __forceinline__ uint64_t globaltimer()
+{
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+/* ---------------------------------------------------------------- errors / spinning -------- */
+__device__ __forceinline__ void raise_error(const dev_ctx *C, int site, int status)
+{
+    uint32_t code = ((uint32_t)site << 8) | (uint32_t)(-status);
+    if (atomicCAS(C->err, 0u, code) == 0u) *(volatile uint32_t *)C->err_host = code;
+}
+__device__ __forceinline__ bool error_latched(const dev_ctx *C)
+{
+    return *(volatile uint32_t *)C->err != 0u;
+}
+/* One back-off step of a spin; true = give up (error latched by anyone, or watchdog expired). */
+__device__ __forceinline__ bool spin_step(const dev_ctx *C, uint64_t t0, uint32_t &it, int site)
+{
+    ++it;
+    if ((it & 31u) == 0u) {
+        if (error_latched(C)) return true;
+        if (globaltimer() - t0 > C->watchdog_ns) {
+            raise_error(C, site, PROACT_ERR_TIMEOUT);
+            return true;
+        }
+    }
+    __nanosleep(it < 64 ? 32 : 256);
+    return false;
+}
+
+/* ---------------------------------------------------------------- roles ------------------- */
+__device__ __forceinline__ bool uses_agent(const launch_ctx &lc)
+{
+    return lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE;
+}
+__device__ __forceinline__ uint32_t producer_block(const launch_ctx &lc) { return blockIdx.x - lc.agent_ctas; }
+__device__ __forceinline__ uint32_t producer_grid(const launch_ctx &lc) { return gridDim.x - lc.agent_ctas; }
+
+__device__ __forceinline__ uint32_t chunk_len(const region_dev &R, uint32_t c)
+{
+    uint64_t lo = (uint64_t)c * R.chunk_bytes;
+    uint64_t hi = lo + R.chunk_bytes;
+    if (hi > R.own_bytes) hi = R.own_bytes;
+    return (uint32_t)(hi - lo);
+}
+__device__ __forceinline__ uint32_t dests_of(const launch_ctx &lc, const region_dev &R, uint32_t c)
+{
+    const dev_ctx *C = lc.ctx;
+    uint32_t m = R.chunk_dest ? R.chunk_dest[c] : (uint32_t)R.dest_mask;
+    m &= ~(1u << C->rank);
+    if (C->world < 32) m &= (1u << C->world) - 1u;
+    return m;
+}
+
+/* ---------------------------------------------------------------- producer side (a2, a3) -- */
+
+/* Instrumented store (a2): a weak store into the LOCAL replica at byte offset `off` (relative to
+ * the replica base).  Under PROACT-inline (L143, Listing 1) the same value is also
+ * stored to every destination peer's mirror (naive fine-grained P2P). */
+template <class T>
+__device__ __forceinline__ void put(const launch_ctx &lc, int r, uint64_t off, const T &v)
+{
+    const region_dev &R = lc.ctx->region[r];
+    *reinterpret_cast<T *>(R.base + off) = v;
+    if (lc.mech == PROACT_MECH_INLINE) {
+        uint32_t c = (uint32_t)((off - R.own_off) / R.chunk_bytes);
+        uint32_t m = dests_of(lc, R, c);
+        while (m) {
+            int p = __ffs(m) - 1;
+            m &= m - 1;
+            *reinterpret_cast<T *>(R.peer_base[p] + off) = v;
+        }
+    }
+}
+
+/* Tally commit (a3) for a contiguous span [off, off + nbytes) of region r (offsets relative to
+ * the replica base, inside my slice) whose stores by this CTA are complete.  Call from ONE thread
+ * after a __syncthreads() that follows the stores.  Adds the bytes to every covered chunk's
+ * counter with release semantics; a chunk whose counter would exceed expected latches
+ * PROACT_ERR_PROTOCOL (non-deterministic store count, L129). */
+__device__ __forceinline__ void commit_span(const launch_ctx &lc, int r, uint64_t off, uint64_t nbytes)
+{
+    if (!uses_agent(lc)) return;
+    const region_dev &R = lc.ctx->region[r];
+    uint64_t rel = off - R.own_off;
+    while (nbytes) {
+        uint32_t c = (uint32_t)(rel / R.chunk_bytes);
+        uint64_t end = (uint64_t)(c + 1) * R.chunk_bytes;
+        if (end > R.own_bytes) end = R.own_bytes;
+        uint32_t b = (uint32_t)((end - rel) < nbytes ? (end - rel) : nbytes);
+        uint32_t old = atom_add_release_gpu(&R.counter[c], b);
+        if (old + b > R.expected[c]) raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
+        rel += b;
+        nbytes -= b;
+    }
+}
+
+/* Chunk-state marks for SPARSE regions (SSSP dirty frontier, reading R13).  Plain stores; call
+ * before the commit that covers the chunk (the commit's release publishes them). */
+__device__ __forceinline__ void mark_changed(const launch_ctx &lc, int r, uint64_t off)
+{
+    const region_dev &R = lc.ctx->region[r];
+    R.changed_gen[(off - R.own_off) / R.chunk_bytes] = lc.gen[r];
+}
+__device__ __forceinline__ void mark_push(const launch_ctx &lc, int r, uint64_t off)
+{
+    const region_dev &R = lc.ctx->region[r];
+    R.push_gen[(off - R.own_off) / R.chunk_bytes] = lc.gen[r];
+}
+/* Did my chunk containing `off` change in region r's current generation? */
+__device__ __forceinline__ bool local_changed(const launch_ctx &lc, int r, uint64_t off)
+{
+    const region_dev &R = lc.ctx->region[r];
+    return R.changed_gen[(off - R.own_off) / R.chunk_bytes] == lc.gen[r];
+}
+/* Phase vote (e.g. "something changed"): OR-ed over all ranks by a BARRIER phase_sync. */
+__device__ __forceinline__ void vote(const launch_ctx &lc) { atomicOr(&lc.ctx->vote[lc.epoch & 1u], 1u); }
+
+/* ---------------------------------------------------------------- consumer side (a7) ------- */
+
+/* Wait (ONE thread; the caller then __syncthreads()) until every REMOTE chunk overlapping
+ * [off, off + nbytes) of region r holds the region's current generation lc.gen[r].  FUSED/ELIDE
+ * spin on the per-chunk arrival flags (ld.acquire.sys); INLINE/BULK on the owner's phase credit
+ * (the data is complete when its producer's phase is); LOCAL returns at once.  Returns the OR of
+ * the covered chunks' "changed" bits (FUSED/ELIDE only; 1 otherwise).  Generation 0 (identical
+ * initial replicas, reading R16) never waits.  Must not be used on a region armed by the same
+ * launch (a launch reads the previous generation of what it does not write). */
+__device__ __forceinline__ uint32_t wait_range(const launch_ctx &lc, int r, uint64_t off, uint64_t nbytes)
+{
+    const dev_ctx *C = lc.ctx;
+    const region_dev &R = C->region[r];
+    uint32_t gen = lc.gen[r];
+    if (gen == 0 || nbytes == 0 || lc.mech == PROACT_MECH_LOCAL) return 1u;
+    uint64_t hi = off + nbytes;
+    uint32_t changed = 0;
+    uint64_t t0 = globaltimer();
+    uint32_t it = 0;
+    for (int p = 0; p < C->world; ++p) {
+        uint64_t plo = R.rank_off[p], phi = R.rank_off[p + 1];
+        if (p == C->rank || phi <= off || plo >= hi || plo == phi) continue;
+        if (uses_agent(lc)) {
+            uint64_t a = (off > plo ? off : plo) - plo, b = (hi < phi ? hi : phi) - plo;
+            uint32_t c0 = (uint32_t)(a / R.chunk_bytes), c1 = (uint32_t)((b - 1) / R.chunk_bytes);
+            for (uint32_t c = c0; c <= c1; ++c) {
+                const uint32_t *f = &R.arrive[R.rank_chunk0[p] + c];
+                uint32_t v;
+                while (((v = ld_acquire_sys(f)) >> 1) < gen)
+                    if (spin_step(C, t0, it, SITE_WAIT_RANGE)) return 1u;
+                changed |= v & 1u;
+            }
+        } else {
+            uint32_t need = lc.gen_epoch[r] + 1u;
+            while ((ld_acquire_sys(&C->done[p]) >> 1) < need)
+                if (spin_step(C, t0, it, SITE_WAIT_RANGE)) return 1u;
+            changed = 1u;
+        }
+    }
+    return changed;
+}
+
+/* Wait (ONE thread) until every chunk pushed into this rank for region r's current generation has
+ * arrived: FUSED/ELIDE poll the region's arrival counter (gen * n_in), INLINE/BULK every peer's
+ * credit.  For all-to-all consumers (PageRank, SSSP gathers). */
+__device__ __forceinline__ void wait_all(const launch_ctx &lc, int r)
+{
+    const dev_ctx *C = lc.ctx;
+    const region_dev &R = C->region[r];
+    uint32_t gen = lc.gen[r];
+    if (gen == 0 || lc.mech == PROACT_MECH_LOCAL) return;
+    uint64_t t0 = globaltimer();
+    uint32_t it = 0;
+    if (uses_agent(lc) && R.n_in != 0xFFFFFFFFu) {
+        uint32_t need = gen * R.n_in;
+        while (ld_acquire_sys(R.arrive_count) < need)
+            if (spin_step(C, t0, it, SITE_WAIT_ALL)) return;
+    } else {
+        uint32_t need = lc.gen_epoch[r] + 1u;   /* owner finished the producing phase */
+        for (int p = 0; p < C->world; ++p) {
+            if (p == C->rank) continue;
+            while ((ld_acquire_sys(&C->done[p]) >> 1) < need)
+                if (spin_step(C, t0, it, SITE_WAIT_ALL)) return;
+        }
+    }
+}
+
+/* Changed bit of global chunk g of region r as last published (valid after wait_all/wait_range;
+ * covers my own chunks too: the agent raises my local flag as well). */
+__device__ __forceinline__ uint32_t chunk_flag(const launch_ctx &lc, int r, uint32_t g)
+{
+    return lc.ctx->region[r].arrive[g];
+}
+
+#endif /* __CUDACC__ */
+} /* namespace proact */
+
+#ifdef __CUDACC__
+namespace proact {
+/* The transfer agent (a4-a6); defined in csrc/agent.cuh, included by the library's kernels. */
+__device__ void agent_loop(const launch_ctx &lc);
+
+/* Agent CTAs (the first lc.agent_ctas blocks of a FUSED/ELIDE launch) run the polling agent and
+ * return true; producer CTAs get false.  Call first thing in a producer kernel. */
+__device__ __forceinline__ bool agent_dispatch(const launch_ctx &lc)
+{
+    if (blockIdx.x >= lc.agent_ctas) return false;
+    agent_loop(lc);
+    return true;
+}
+} /* namespace proact */
+#endif
+
+#endif /* PROACT_DEVICE_CUH */

@@ -1,0 +1,122 @@
+"""ctypes binding of libproact.so (argument marshalling only).
+
+Every step of the hot path runs in the library's CUDA kernels; this module only
+declares the C signatures of include/proact.h and include/proact_workloads.h.
+There is no fallback: if the shared library is missing or cannot be loaded the
+import fails loudly (build it with __graft_entry__.build()).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libproact.so")
+
+MAX_RANKS = 16
+MAX_REGIONS = 8
+
+OK = 0
+ERR_INVALID, ERR_CUDA, ERR_NOPEER, ERR_STATE, ERR_TIMEOUT, ERR_PROTOCOL, ERR_NOMEM = range(-1, -8, -1)
+
+MECH_FUSED, MECH_INLINE, MECH_BULK, MECH_LOCAL, MECH_ELIDE = range(5)
+MECH_NAMES = {MECH_FUSED: "fused", MECH_INLINE: "inline", MECH_BULK: "bulk",
+              MECH_LOCAL: "local", MECH_ELIDE: "elide"}
+PUSH_VEC16, PUSH_BULK = 0, 1
+SYNC_SIGNAL, SYNC_BARRIER = 0, 1
+REGION_SPARSE = 1
+
+
+class ProactError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        self.code = code
+        name = _lib.proact_error_string(code).decode() if _lib is not None else str(code)
+        super().__init__(f"{what}: {name} ({code})" if what else f"{name} ({code})")
+
+
+class Config(ctypes.Structure):
+    _fields_ = [("mech", ctypes.c_int32), ("push", ctypes.c_int32),
+                ("agent_warps", ctypes.c_int32), ("block", ctypes.c_int32),
+                ("piece_bytes", ctypes.c_uint32), ("watchdog_ms", ctypes.c_uint32),
+                ("grid_cap", ctypes.c_int32), ("chunk_bytes", ctypes.c_uint32)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class RegionInfo(ctypes.Structure):
+    _fields_ = [("replica_base", ctypes.c_void_p), ("own_offset", ctypes.c_uint64),
+                ("own_bytes", ctypes.c_uint64), ("total_bytes", ctypes.c_uint64),
+                ("chunk_bytes", ctypes.c_uint64), ("n_own_chunks", ctypes.c_uint32),
+                ("n_total_chunks", ctypes.c_uint32), ("first_chunk", ctypes.c_uint32),
+                ("generation", ctypes.c_uint32), ("dest_mask", ctypes.c_uint64),
+                ("rank_offset", ctypes.c_uint64 * (MAX_RANKS + 1))]
+
+
+RUN_FN = ctypes.CFUNCTYPE(ctypes.c_double, ctypes.POINTER(Config), ctypes.c_void_p)
+
+_lib = None
+
+
+def _declare(L):
+    i, u32, u64, sz, vp, cp = (ctypes.c_int, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_size_t,
+                               ctypes.c_void_p, ctypes.c_char_p)
+    sigs = {
+        "proact_init": (i, [i]),
+        "proact_init_ex": (i, [i, i, cp]),
+        "proact_finalize": (i, []),
+        "proact_rank": (i, []),
+        "proact_world": (i, []),
+        "proact_ranks_on_device": (i, []),
+        "proact_error_string": (cp, [i]),
+        "proact_last_cuda_error": (i, []),
+        "proact_set_config": (i, [ctypes.POINTER(Config)]),
+        "proact_get_config": (i, [ctypes.POINTER(Config)]),
+        "proact_register_region": (i, [vp, sz, sz, u64]),
+        "proact_register_region_ex": (i, [vp, sz, sz, u64, u32]),
+        "proact_region_set_chunk_dest": (i, [i, u32, u64]),
+        "proact_region_info_get": (i, [i, ctypes.POINTER(RegionInfo)]),
+        "proact_region_rechunk": (i, [i, sz]),
+        "proact_region_debug_deliveries": (i, [i, ctypes.POINTER(u32), sz]),
+        "proact_launch": (i, [ctypes.POINTER(i), i, vp, ctypes.c_uint, ctypes.c_uint,
+                              ctypes.POINTER(vp), sz, vp]),
+        "proact_phase_sync": (i, [vp, i]),
+        "proact_last_vote": (i, []),
+        "proact_check": (i, []),
+        "proact_launch_count": (u64, []),
+        "proact_epoch": (u32, []),
+        "proact_autotune": (i, [cp, cp, RUN_FN, vp, ctypes.POINTER(Config)]),
+        # workloads
+        "proact_jacobi_phase": (i, [i, i, ctypes.c_longlong, i, vp]),
+        "proact_micro_phase": (i, [i, ctypes.c_uint, ctypes.c_uint, i, i, vp]),
+        "proact_jacobi_solve_host": (i, [vp, vp, ctypes.c_longlong, i, sz, i, vp,
+                                         ctypes.POINTER(ctypes.c_ulonglong),
+                                         ctypes.POINTER(ctypes.c_ulonglong)]),
+    }
+    for name, (res, args) in sigs.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return sorted(sigs)
+
+
+EXPORTED: list[str] = []
+
+
+def load():
+    """Load libproact.so (raises if it is missing: there is no CPU fallback)."""
+    global _lib, EXPORTED
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                              "(the CUDA path has no fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        EXPORTED = _declare(L)
+        _lib = L
+    return _lib
+
+
+def check(rc: int, what: str = "") -> int:
+    if rc < 0:
+        raise ProactError(rc, what)
+    return rc

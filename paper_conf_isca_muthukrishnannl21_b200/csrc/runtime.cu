@@ -1,0 +1,1062 @@
+// runtime.cu -- host runtime of libproact: bootstrap, peer mapping, region registry / readiness
+// tables (a1), launch (fills proact::launch_ctx), phase synchronisation (a8), error surfacing.
+//
+// The paper's runtime is sketched by Listing 1: proact_init() chooses the
+// transfer mechanism from the profiler, allocates one counter per chunk initialised from the
+// profiler and, for polling, a bitmap plus a long-lived polling kernel; main() allocates one
+// replica per GPU (cudaMalloc4GPU) and fills region1[gpu].  This file is the B200 re-design:
+// one rank per GPU (process or thread), a /dev/shm rendezvous, CUDA IPC or direct peer pointers
+// for the replicas, counters counting bytes (reading R1), per-chunk arrival flags and per-rank
+// credits in place of the global barrier (readings R5, R6).  See include/proact.h for the API.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "proact.h"
+#include "proact_device.cuh"
+
+using proact::dev_ctx;
+using proact::launch_ctx;
+using proact::region_dev;
+
+namespace {
+
+constexpr int MAXR = PROACT_MAX_RANKS;
+constexpr int MAXG = PROACT_MAX_REGIONS;
+
+// ------------------------------------------------------------------------------- shm rendezvous
+constexpr size_t SLOT_BYTES = 4096;
+
+struct ShmHeader {
+    std::atomic<uint32_t> arrived;
+    std::atomic<uint32_t> generation;
+    std::atomic<uint32_t> joined;
+    std::atomic<uint32_t> left;
+    uint32_t world;
+    char pad[4096 - 5 * sizeof(uint32_t)];
+};
+
+struct Shm {
+    std::string name;
+    ShmHeader *hdr = nullptr;
+    char *slots = nullptr;
+    size_t size = 0;
+    int world = 0;
+    double timeout_s = 120.0;
+
+    int open(const std::string &job, int world_) {
+        world = world_;
+        std::string key;
+        for (char c : job) key += (isalnum((unsigned char)c) || c == '_' || c == '-') ? c : '_';
+        name = "/proact_" + key;
+        size = sizeof(ShmHeader) + SLOT_BYTES * (size_t)world;
+        int fd = shm_open(name.c_str(), O_CREAT | O_RDWR, 0600);
+        if (fd < 0) return PROACT_ERR_STATE;
+        struct stat st;
+        if (fstat(fd, &st) != 0) { ::close(fd); return PROACT_ERR_STATE; }
+        if ((size_t)st.st_size < size && ftruncate(fd, (off_t)size) != 0) { ::close(fd); return PROACT_ERR_STATE; }
+        void *p = mmap(nullptr, size, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+        ::close(fd);
+        if (p == MAP_FAILED) return PROACT_ERR_STATE;
+        hdr = (ShmHeader *)p;
+        slots = (char *)p + sizeof(ShmHeader);
+        if (const char *t = getenv("PROACT_RDV_TIMEOUT_S")) timeout_s = atof(t);
+        hdr->joined.fetch_add(1);
+        return PROACT_OK;
+    }
+    int barrier() {
+        uint32_t gen = hdr->generation.load(std::memory_order_acquire);
+        if (hdr->arrived.fetch_add(1, std::memory_order_acq_rel) + 1 == (uint32_t)world) {
+            hdr->arrived.store(0, std::memory_order_relaxed);
+            hdr->generation.fetch_add(1, std::memory_order_release);
+            return PROACT_OK;
+        }
+        auto t0 = std::chrono::steady_clock::now();
+        uint32_t spins = 0;
+        while (hdr->generation.load(std::memory_order_acquire) == gen) {
+            if (++spins < 1000) std::this_thread::yield();
+            else std::this_thread::sleep_for(std::chrono::microseconds(50));
+            if ((spins & 1023) == 0 &&
+                std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > timeout_s)
+                return PROACT_ERR_TIMEOUT;
+        }
+        return PROACT_OK;
+    }
+    // all-gather of fixed-size blobs (<= SLOT_BYTES)
+    int allgather(int rank, const void *mine, size_t n, void *all) {
+        if (n > SLOT_BYTES) return PROACT_ERR_INVALID;
+        memcpy(slots + (size_t)rank * SLOT_BYTES, mine, n);
+        int rc = barrier();
+        if (rc) return rc;
+        for (int r = 0; r < world; ++r) memcpy((char *)all + (size_t)r * n, slots + (size_t)r * SLOT_BYTES, n);
+        return barrier();
+    }
+    void close(bool last_unlinks) {
+        if (!hdr) return;
+        uint32_t left = hdr->left.fetch_add(1) + 1;
+        bool last = left == (uint32_t)world;
+        munmap(hdr, size);
+        hdr = nullptr;
+        if (last && last_unlinks) shm_unlink(name.c_str());
+    }
+};
+
+// ------------------------------------------------------------------------------- rank context
+struct PeerInfo {
+    int32_t pid;
+    int32_t device;
+    char uuid[16];
+    cudaIpcMemHandle_t meta_handle;   // my rank metadata block (done[], ...)
+    uint64_t meta_off_done;
+    uint64_t done_ptr;                // raw pointer (valid in my process)
+};
+
+struct RegionExchange {
+    uint64_t bytes, chunk, dest_mask, flags;
+    uint64_t ptr;                     // my slice pointer (valid in my process)
+    cudaIpcMemHandle_t data_handle;   // allocation containing ptr
+    uint64_t data_off;                // ptr - allocation base
+    cudaIpcMemHandle_t meta_handle;   // region metadata block
+    uint64_t meta_ptr;
+    uint64_t off_arrive, off_count;
+    int32_t data_ipc_ok;
+};
+
+struct Region {
+    bool used = false;
+    uint64_t own_off = 0, own_bytes = 0, total = 0, chunk = 0, dest_mask = 0;
+    uint32_t flags = 0, n_own = 0, n_total = 0, chunk0 = 0;
+    char *base = nullptr;
+    void *my_ptr = nullptr;
+    uint64_t rank_off[MAXR + 1] = {0};
+    uint32_t rank_chunk0[MAXR + 1] = {0};
+    char *meta = nullptr;             // library block for this region (device)
+    size_t meta_bytes = 0;
+    std::vector<void *> opened;       // IPC mappings to close
+    std::vector<uint32_t> chunk_dest; // host copy of per-chunk overrides (empty = none)
+    uint32_t *d_chunk_dest = nullptr;
+    uint32_t gen_done = 0;            // completed (launched) generations
+    uint32_t gen_epoch = 0;           // epoch of the latest generation
+    int64_t last_armed_epoch = -1;
+};
+
+struct RankCtx {
+    int rank = -1, world = 0, device = 0;
+    std::string job;
+    Shm shm;
+    proact_config cfg{};
+    int ranks_on_device = 1;
+    bool coop = false;
+    int nsm = 0;
+    bool debug = false;
+    std::vector<PeerInfo> peers;
+    dev_ctx h{};                      // host copy of the device context
+    dev_ctx *d = nullptr;             // device context
+    char *meta = nullptr;             // done[world] | err | vote[2]
+    uint32_t *h_err = nullptr, *d_err_host = nullptr;   // mapped error mirror
+    uint32_t *h_vote = nullptr, *d_vote_host = nullptr; // mapped vote result
+    std::vector<void *> opened;       // IPC mappings of peers' metadata
+    Region regions[MAXG];
+    int nregions = 0;
+    uint32_t epoch = 0;
+    uint32_t armed_epoch_mask = 0;    // regions armed in the current epoch
+    uint32_t bulk_mask = 0;           // regions launched with BULK in the current epoch
+    int bulk_pending = 0;
+    uint64_t launches = 0;
+    int last_cuda = 0;
+    int latched = 0;
+};
+
+thread_local RankCtx *tl = nullptr;
+
+#define CK(call)                                                         \
+    do {                                                                 \
+        cudaError_t e_ = (call);                                         \
+        if (e_ != cudaSuccess) {                                         \
+            if (tl) tl->last_cuda = (int)e_;                             \
+            fprintf(stderr, "[proact] %s failed: %s (%s:%d)\n", #call,  \
+                    cudaGetErrorString(e_), __FILE__, __LINE__);         \
+            return PROACT_ERR_CUDA;                                      \
+        }                                                                \
+    } while (0)
+
+int env_int(const char *name, int dflt) {
+    const char *v = getenv(name);
+    return v && *v ? atoi(v) : dflt;
+}
+
+proact_config default_config() {
+    proact_config c{};
+    c.mech = PROACT_MECH_FUSED;
+    c.push = PROACT_PUSH_VEC16;
+    c.agent_warps = 16;
+    c.block = 256;
+    c.piece_bytes = 64 * 1024;
+    c.watchdog_ms = 20000;
+    c.grid_cap = 0;
+    c.chunk_bytes = 128 * 1024;   // the paper's V100 profiler choice (Table II)
+    return c;
+}
+
+void apply_env(proact_config &c) {
+    c.mech = env_int("PROACT_MECH", c.mech);
+    c.push = env_int("PROACT_PUSH", c.push);
+    c.agent_warps = env_int("PROACT_AGENT_WARPS", c.agent_warps);
+    c.piece_bytes = (uint32_t)env_int("PROACT_PIECE_BYTES", (int)c.piece_bytes);
+    c.watchdog_ms = (uint32_t)env_int("PROACT_WATCHDOG_MS", (int)c.watchdog_ms);
+    c.chunk_bytes = (uint32_t)env_int("PROACT_CHUNK_BYTES", (int)c.chunk_bytes);
+    if (getenv("PROACT_ELIDE_PUSH") && atoi(getenv("PROACT_ELIDE_PUSH"))) c.mech = PROACT_MECH_ELIDE;
+}
+
+int validate_config(const proact_config &c) {
+    if (c.mech < 0 || c.mech > PROACT_MECH_ELIDE) return PROACT_ERR_INVALID;
+    if (c.push != PROACT_PUSH_VEC16) return PROACT_ERR_INVALID;   // BULK push: not built yet
+    if (c.agent_warps < 1 || c.agent_warps > 1024) return PROACT_ERR_INVALID;
+    if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
+    if (c.piece_bytes < 512 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
+    if (c.watchdog_ms < 1) return PROACT_ERR_INVALID;
+    if (c.chunk_bytes < 4096 || c.chunk_bytes % 16) return PROACT_ERR_INVALID;
+    return PROACT_OK;
+}
+
+int upload_ctx(RankCtx *c) {
+    CK(cudaMemcpy(c->d, &c->h, sizeof(dev_ctx), cudaMemcpyHostToDevice));
+    return PROACT_OK;
+}
+
+int check_latched(RankCtx *c) {
+    if (c->latched) return c->latched;
+    uint32_t code = *(volatile uint32_t *)c->h_err;
+    if (code) {
+        int st = -(int)(code & 0xFF);
+        if (st >= 0 || st < PROACT_ERR_NOMEM) st = PROACT_ERR_PROTOCOL;
+        c->latched = st;
+        fprintf(stderr, "[proact] rank %d: device error latched: %s (site %u)\n", c->rank,
+                proact_error_string(st), code >> 8);
+        return st;
+    }
+    return PROACT_OK;
+}
+
+// map a peer allocation: direct pointer (same process) or IPC
+int map_peer(RankCtx *c, int p, const cudaIpcMemHandle_t &h, uint64_t raw_ptr_of_base_plus_off,
+             uint64_t off_in_alloc, char **out, std::vector<void *> &opened) {
+    const PeerInfo &pi = c->peers[p];
+    if (pi.pid == (int32_t)getpid()) {
+        if (pi.device != c->device) {
+            int can = 0;
+            CK(cudaDeviceCanAccessPeer(&can, c->device, pi.device));
+            if (!can) return PROACT_ERR_NOPEER;
+            cudaError_t e = cudaDeviceEnablePeerAccess(pi.device, 0);
+            if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) { c->last_cuda = e; return PROACT_ERR_NOPEER; }
+            cudaGetLastError();
+        }
+        *out = (char *)(uintptr_t)raw_ptr_of_base_plus_off;
+        return PROACT_OK;
+    }
+    void *base = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+        c->last_cuda = e;
+        fprintf(stderr, "[proact] rank %d: cudaIpcOpenMemHandle(peer %d) failed: %s\n", c->rank, p,
+                cudaGetErrorString(e));
+        return PROACT_ERR_NOPEER;
+    }
+    opened.push_back(base);
+    *out = (char *)base + off_in_alloc;
+    return PROACT_OK;
+}
+
+// Driver entry point resolved through the runtime, so libproact does not link libcuda.so.1 and
+// still loads (for symbol checks) on a machine without a GPU driver.
+typedef CUresult (*pfn_getrange)(CUdeviceptr *, size_t *, CUdeviceptr);
+
+int alloc_base_and_handle(void *ptr, cudaIpcMemHandle_t *h, uint64_t *off, int *ok) {
+    CUdeviceptr base = 0;
+    size_t sz = 0;
+    *ok = 0;
+    memset(h, 0, sizeof(*h));
+    *off = 0;
+    static pfn_getrange getrange = nullptr;
+    if (!getrange) {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
+            return PROACT_OK;
+        getrange = (pfn_getrange)fn;
+    }
+    if (getrange(&base, &sz, (CUdeviceptr)(uintptr_t)ptr) != CUDA_SUCCESS) return PROACT_OK;
+    *off = (uint64_t)((uintptr_t)ptr - (uintptr_t)base);
+    if (cudaIpcGetMemHandle(h, (void *)(uintptr_t)base) == cudaSuccess) *ok = 1;
+    else cudaGetLastError();
+    return PROACT_OK;
+}
+
+uint32_t ceil_div64(uint64_t a, uint64_t b) { return (uint32_t)((a + b - 1) / b); }
+
+// (re)build a region's library block, flags, expected table; fills R and c->h.region[id]
+// except peer pointers.  Returns the exchange record.
+int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
+    R.n_own = ceil_div64(R.own_bytes, R.chunk);
+    size_t n_own = std::max<uint32_t>(R.n_own, 1);
+    // totals / global numbering need every rank's bytes: done by caller before (rank_off filled)
+    size_t n_total = std::max<uint32_t>(R.n_total, 1);
+    size_t deliv = c->debug ? n_own * (size_t)c->world : 0;
+    // layout: counter | expected | piecedone | changed | push | arrive[n_total] | count | deliv
+    size_t off_counter = 0, off_expected = off_counter + 4 * n_own, off_piece = off_expected + 4 * n_own,
+           off_changed = off_piece + 4 * n_own, off_push = off_changed + 4 * n_own,
+           off_arrive = off_push + 4 * n_own, off_count = off_arrive + 4 * n_total,
+           off_deliv = off_count + 64, total = off_deliv + 4 * deliv + 64;
+    if (R.meta) { CK(cudaFree(R.meta)); R.meta = nullptr; }
+    CK(cudaMalloc((void **)&R.meta, total));
+    CK(cudaMemset(R.meta, 0, total));
+    R.meta_bytes = total;
+    std::vector<uint32_t> expected(n_own, 0);
+    for (uint32_t k = 0; k < R.n_own; ++k) {
+        uint64_t lo = (uint64_t)k * R.chunk, hi = std::min<uint64_t>(lo + R.chunk, R.own_bytes);
+        expected[k] = (uint32_t)(hi - lo);
+    }
+    CK(cudaMemcpy(R.meta + off_expected, expected.data(), 4 * n_own, cudaMemcpyHostToDevice));
+    region_dev &D = c->h.region[id];
+    D.base = R.base;
+    D.own_off = R.own_off;
+    D.own_bytes = R.own_bytes;
+    D.total_bytes = R.total;
+    D.chunk_bytes = (uint32_t)R.chunk;
+    D.n_own = R.n_own;
+    D.chunk0 = R.chunk0;
+    D.n_total = R.n_total;
+    D.flags = R.flags;
+    D.dest_mask = R.dest_mask;
+    D.counter = (uint32_t *)(R.meta + off_counter);
+    D.expected = (uint32_t *)(R.meta + off_expected);
+    D.piecedone = (uint32_t *)(R.meta + off_piece);
+    D.changed_gen = (uint32_t *)(R.meta + off_changed);
+    D.push_gen = (uint32_t *)(R.meta + off_push);
+    D.arrive = (uint32_t *)(R.meta + off_arrive);
+    D.arrive_count = (uint32_t *)(R.meta + off_count);
+    D.deliv = deliv ? (uint32_t *)(R.meta + off_deliv) : nullptr;
+    D.chunk_dest = nullptr;
+    R.chunk_dest.clear();
+    if (R.d_chunk_dest) { CK(cudaFree(R.d_chunk_dest)); R.d_chunk_dest = nullptr; }
+    for (int p = 0; p <= c->world; ++p) { D.rank_off[p] = R.rank_off[p]; D.rank_chunk0[p] = R.rank_chunk0[p]; }
+    // arrival flags of existing generations: a fresh table starts at "generation gen_done
+    // complete" so consumers of the current data do not wait (rechunk keeps generations)
+    if (R.gen_done) {
+        std::vector<uint32_t> fl(n_total, R.gen_done << 1 | 1u);
+        CK(cudaMemcpy(R.meta + off_arrive, fl.data(), 4 * n_total, cudaMemcpyHostToDevice));
+        // arrival counter restarts at gen_done * n_in (set after n_in is known, in finish)
+    }
+    memset(&ex, 0, sizeof(ex));
+    CK(cudaIpcGetMemHandle(&ex.meta_handle, R.meta));
+    ex.meta_ptr = (uint64_t)(uintptr_t)R.meta;
+    ex.off_arrive = off_arrive;
+    ex.off_count = off_count;
+    return PROACT_OK;
+}
+
+int finish_region_peers(RankCtx *c, int id, Region &R, const std::vector<RegionExchange> &all) {
+    region_dev &D = c->h.region[id];
+    uint32_t n_in = 0;
+    for (int p = 0; p < c->world; ++p) {
+        D.peer_base[p] = nullptr;
+        D.peer_arrive[p] = nullptr;
+        D.peer_arrive_count[p] = nullptr;
+        if (p == c->rank) {
+            D.peer_base[p] = R.base;
+            D.peer_arrive[p] = D.arrive;
+            D.peer_arrive_count[p] = D.arrive_count;
+            continue;
+        }
+        if (all[p].dest_mask >> c->rank & 1) n_in += R.rank_chunk0[p + 1] - R.rank_chunk0[p];
+        const RegionExchange &e = all[p];
+        char *pd = nullptr, *pm = nullptr;
+        // data: the peer's replica base = its slice pointer - its slice offset
+        if (c->peers[p].pid != (int32_t)getpid() && !e.data_ipc_ok) return PROACT_ERR_NOPEER;
+        int rc = map_peer(c, p, e.data_handle, e.ptr, e.data_off, &pd, R.opened);
+        if (rc) return rc;
+        D.peer_base[p] = pd - R.rank_off[p];
+        rc = map_peer(c, p, e.meta_handle, e.meta_ptr, 0, &pm, R.opened);
+        if (rc) return rc;
+        D.peer_arrive[p] = (uint32_t *)(pm + e.off_arrive);
+        D.peer_arrive_count[p] = (uint32_t *)(pm + e.off_count);
+    }
+    D.n_in = n_in;
+    if (R.gen_done) {
+        uint32_t cnt = R.gen_done * n_in;
+        CK(cudaMemcpy(D.arrive_count, &cnt, 4, cudaMemcpyHostToDevice));
+    }
+    return PROACT_OK;
+}
+
+__global__ void sync_kernel(const dev_ctx *C, uint32_t epoch, int mode)
+{
+    // (a8) credit peers "rank finished phase `epoch`" and optionally wait for everyone (L125)
+    const uint32_t lane = threadIdx.x;
+    uint32_t myvote = C->vote[epoch & 1u] ? 1u : 0u;
+    proact::fence_acq_rel_sys();
+    uint32_t val = ((epoch + 1u) << 1) | myvote;
+    for (int p = lane; p < C->world; p += 32) {
+        if (p == C->rank) proact::st_release_sys(&C->done[p], val);
+        else proact::st_release_sys(C->peer_done[p] + C->rank, val);
+    }
+    __syncwarp();
+    if (mode == PROACT_SYNC_BARRIER) {
+        uint32_t any = 0;
+        uint64_t t0 = proact::globaltimer();
+        uint32_t it = 0;
+        for (int p = lane; p < C->world; p += 32) {
+            uint32_t v;
+            while (((v = proact::ld_acquire_sys(&C->done[p])) >> 1) < epoch + 1u)
+                if (proact::spin_step(C, t0, it, proact::SITE_SYNC)) break;
+            any |= v & 1u;
+        }
+        any = __any_sync(0xFFFFFFFFu, any);
+        if (lane == 0) *(volatile uint32_t *)C->vote_host = ((epoch + 1u) << 1) | any;
+    }
+    if (lane == 0) C->vote[epoch & 1u] = 0u;
+}
+
+__global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t mask)
+{
+    // BULK: before copying epoch-e data into peer p's replica, p must have finished phase e-1
+    const uint32_t lane = threadIdx.x;
+    uint64_t t0 = proact::globaltimer();
+    uint32_t it = 0;
+    for (int p = lane; p < C->world; p += 32) {
+        if (!(mask >> p & 1u) || p == C->rank) continue;
+        while ((proact::ld_acquire_sys(&C->done[p]) >> 1) < epoch)
+            if (proact::spin_step(C, t0, it, proact::SITE_AGENT_CREDIT)) break;
+    }
+}
+
+RankCtx *need_ctx() { return tl; }
+
+}  // namespace
+
+// ================================================================================== C ABI
+extern "C" {
+
+const char *proact_error_string(int code)
+{
+    switch (code) {
+    case PROACT_OK: return "PROACT_OK";
+    case PROACT_ERR_INVALID: return "PROACT_ERR_INVALID";
+    case PROACT_ERR_CUDA: return "PROACT_ERR_CUDA";
+    case PROACT_ERR_NOPEER: return "PROACT_ERR_NOPEER";
+    case PROACT_ERR_STATE: return "PROACT_ERR_STATE";
+    case PROACT_ERR_TIMEOUT: return "PROACT_ERR_TIMEOUT";
+    case PROACT_ERR_PROTOCOL: return "PROACT_ERR_PROTOCOL";
+    case PROACT_ERR_NOMEM: return "PROACT_ERR_NOMEM";
+    default: return "PROACT_ERR_UNKNOWN";
+    }
+}
+
+int proact_last_cuda_error(void) { return tl ? tl->last_cuda : 0; }
+int proact_rank(void) { return tl ? tl->rank : -1; }
+int proact_world(void) { return tl ? tl->world : 0; }
+int proact_ranks_on_device(void) { return tl ? tl->ranks_on_device : 0; }
+uint64_t proact_launch_count(void) { return tl ? tl->launches : 0; }
+uint32_t proact_epoch(void) { return tl ? tl->epoch : 0; }
+
+int proact_init_ex(int ngpus, int rank, const char *job)
+{
+    if (tl) return PROACT_ERR_STATE;
+    if (ngpus < 1 || ngpus > MAXR || rank < 0 || rank >= ngpus) return PROACT_ERR_INVALID;
+    RankCtx *c = new RankCtx();
+    c->rank = rank;
+    c->world = ngpus;
+    c->job = job && *job ? job : "default";
+    c->cfg = default_config();
+    apply_env(c->cfg);
+    if (validate_config(c->cfg)) c->cfg = default_config();
+    c->debug = env_int("PROACT_DEBUG", 0) != 0;
+    tl = c;
+    auto fail = [&](int rc) { tl = nullptr; delete c; return rc; };
+    if (cudaGetDevice(&c->device) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    cudaFree(0);   // make sure the primary context exists on this thread's device
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, c->device) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    c->nsm = prop.multiProcessorCount;
+    int coop_attr = 0;
+    cudaDeviceGetAttribute(&coop_attr, cudaDevAttrCooperativeLaunch, c->device);
+    // rank metadata block: done[MAXR] | err | vote[2]
+    size_t meta_bytes = 4 * MAXR + 64 + 64;
+    if (cudaMalloc((void **)&c->meta, meta_bytes) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    cudaMemset(c->meta, 0, meta_bytes);
+    if (cudaHostAlloc((void **)&c->h_err, 64, cudaHostAllocMapped) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    memset(c->h_err, 0, 64);
+    c->h_vote = c->h_err + 8;
+    cudaHostGetDevicePointer((void **)&c->d_err_host, c->h_err, 0);
+    c->d_vote_host = c->d_err_host + 8;
+    if (cudaMalloc((void **)&c->d, sizeof(dev_ctx)) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    memset(&c->h, 0, sizeof(c->h));
+    c->h.rank = rank;
+    c->h.world = ngpus;
+    c->h.watchdog_ns = (uint64_t)c->cfg.watchdog_ms * 1000000ull;
+    c->h.done = (uint32_t *)c->meta;
+    c->h.err = (uint32_t *)(c->meta + 4 * MAXR);
+    c->h.vote = (uint32_t *)(c->meta + 4 * MAXR + 64);
+    c->h.err_host = c->d_err_host;
+    c->h.vote_host = c->d_vote_host;
+    // rendezvous
+    int rc = c->shm.open(c->job, ngpus);
+    if (rc) return fail(rc);
+    PeerInfo mine{};
+    mine.pid = (int32_t)getpid();
+    mine.device = c->device;
+    memcpy(mine.uuid, &prop.uuid, 16);
+    if (cudaIpcGetMemHandle(&mine.meta_handle, c->meta) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    mine.done_ptr = (uint64_t)(uintptr_t)c->meta;
+    c->peers.resize(ngpus);
+    rc = c->shm.allgather(rank, &mine, sizeof(mine), c->peers.data());
+    if (rc) return fail(rc);
+    c->ranks_on_device = 0;
+    for (int p = 0; p < ngpus; ++p)
+        if (memcmp(c->peers[p].uuid, mine.uuid, 16) == 0) c->ranks_on_device++;
+    c->coop = coop_attr && c->ranks_on_device == 1;
+    for (int p = 0; p < ngpus; ++p) {
+        if (p == rank) { c->h.peer_done[p] = c->h.done; continue; }
+        char *pm = nullptr;
+        rc = map_peer(c, p, c->peers[p].meta_handle, c->peers[p].done_ptr, 0, &pm, c->opened);
+        if (rc) return fail(rc);
+        c->h.peer_done[p] = (uint32_t *)pm;
+    }
+    rc = upload_ctx(c);
+    if (rc) return fail(rc);
+    rc = c->shm.barrier();
+    if (rc) return fail(rc);
+    return PROACT_OK;
+}
+
+int proact_init(int ngpus)
+{
+    int rank = -1;
+    if (getenv("PROACT_RANK")) rank = atoi(getenv("PROACT_RANK"));
+    else if (getenv("RANK")) rank = atoi(getenv("RANK"));
+    else if (cudaGetDevice(&rank) != cudaSuccess) return PROACT_ERR_CUDA;
+    std::string job = "default";
+    if (getenv("PROACT_JOB")) job = getenv("PROACT_JOB");
+    else if (getenv("MASTER_PORT"))
+        job = std::string(getenv("MASTER_ADDR") ? getenv("MASTER_ADDR") : "") + ":" + getenv("MASTER_PORT");
+    return proact_init_ex(ngpus, rank, job.c_str());
+}
+
+int proact_set_config(const proact_config *cfg)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    proact_config n = cfg ? *cfg : default_config();
+    if (!cfg) apply_env(n);
+    int rc = validate_config(n);
+    if (rc) return rc;
+    bool wd = n.watchdog_ms != c->cfg.watchdog_ms;
+    c->cfg = n;
+    if (wd) {
+        c->h.watchdog_ns = (uint64_t)n.watchdog_ms * 1000000ull;
+        cudaSetDevice(c->device);
+        return upload_ctx(c);
+    }
+    return PROACT_OK;
+}
+
+int proact_get_config(proact_config *cfg)
+{
+    RankCtx *c = need_ctx();
+    if (!c || !cfg) return c ? PROACT_ERR_INVALID : PROACT_ERR_STATE;
+    *cfg = c->cfg;
+    return PROACT_OK;
+}
+
+int proact_register_region_ex(void *ptr, size_t bytes, size_t chunk_bytes, uint64_t dest_mask, uint32_t flags)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    cudaSetDevice(c->device);
+    int bad = 0;
+    if (c->nregions >= MAXG) bad = 1;
+    if (((uintptr_t)ptr % 16) || (bytes % 16) || (chunk_bytes % 16) || chunk_bytes < 4096) bad = 1;
+    if (!ptr && bytes) bad = 1;
+    // exchange (even on local failure, so nobody hangs): geometry first
+    struct Geo { uint64_t bytes, chunk, dest, flags; int32_t bad, pad; } g{bytes, chunk_bytes, dest_mask, flags, bad, 0};
+    std::vector<Geo> geos(c->world);
+    int rc = c->shm.allgather(c->rank, &g, sizeof(g), geos.data());
+    if (rc) return rc;
+    for (auto &x : geos) if (x.bad || x.chunk != chunk_bytes) return PROACT_ERR_INVALID;
+    int id = c->nregions;
+    Region &R = c->regions[id];
+    R = Region();
+    R.used = true;
+    R.chunk = chunk_bytes;
+    R.dest_mask = dest_mask;
+    R.flags = flags;
+    R.own_bytes = bytes;
+    R.rank_off[0] = 0;
+    R.rank_chunk0[0] = 0;
+    for (int p = 0; p < c->world; ++p) {
+        R.rank_off[p + 1] = R.rank_off[p] + geos[p].bytes;
+        R.rank_chunk0[p + 1] = R.rank_chunk0[p] + ceil_div64(geos[p].bytes, chunk_bytes);
+    }
+    R.own_off = R.rank_off[c->rank];
+    R.total = R.rank_off[c->world];
+    R.n_total = R.rank_chunk0[c->world];
+    R.chunk0 = R.rank_chunk0[c->rank];
+    R.my_ptr = ptr;
+    R.base = (char *)ptr - R.own_off;
+    RegionExchange ex;
+    rc = build_region_tables(c, id, R, ex);
+    if (rc) return rc;
+    ex.bytes = bytes;
+    ex.chunk = chunk_bytes;
+    ex.dest_mask = dest_mask;
+    ex.flags = flags;
+    ex.ptr = (uint64_t)(uintptr_t)R.base + R.own_off;   // == ptr
+    if (ptr) alloc_base_and_handle(ptr, &ex.data_handle, &ex.data_off, &ex.data_ipc_ok);
+    std::vector<RegionExchange> all(c->world);
+    rc = c->shm.allgather(c->rank, &ex, sizeof(ex), all.data());
+    if (rc) return rc;
+    rc = finish_region_peers(c, id, R, all);
+    if (rc) return rc;
+    rc = upload_ctx(c);
+    if (rc) return rc;
+    c->nregions++;
+    rc = c->shm.barrier();
+    return rc ? rc : id;
+}
+
+int proact_register_region(void *ptr, size_t bytes, size_t chunk_bytes, uint64_t dest_mask)
+{
+    return proact_register_region_ex(ptr, bytes, chunk_bytes, dest_mask, 0);
+}
+
+int proact_region_rechunk(int id, size_t chunk_bytes)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (id < 0 || id >= c->nregions) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CK(cudaDeviceSynchronize());
+    Region &R = c->regions[id];
+    int bad = (chunk_bytes % 16) || chunk_bytes < 4096;
+    struct Geo { uint64_t chunk; int32_t bad, pad; } g{chunk_bytes, bad, 0};
+    std::vector<Geo> geos(c->world);
+    int rc = c->shm.allgather(c->rank, &g, sizeof(g), geos.data());
+    if (rc) return rc;
+    for (auto &x : geos) if (x.bad || x.chunk != chunk_bytes) return PROACT_ERR_INVALID;
+    // peers must stop touching our old flags before we free them
+    rc = c->shm.barrier();
+    if (rc) return rc;
+    for (void *p : R.opened) cudaIpcCloseMemHandle(p);
+    R.opened.clear();
+    R.chunk = chunk_bytes;
+    R.rank_chunk0[0] = 0;
+    for (int p = 0; p < c->world; ++p)
+        R.rank_chunk0[p + 1] = R.rank_chunk0[p] + ceil_div64(R.rank_off[p + 1] - R.rank_off[p], chunk_bytes);
+    R.n_total = R.rank_chunk0[c->world];
+    R.chunk0 = R.rank_chunk0[c->rank];
+    RegionExchange ex;
+    rc = build_region_tables(c, id, R, ex);
+    if (rc) return rc;
+    ex.bytes = R.own_bytes;
+    ex.chunk = chunk_bytes;
+    ex.dest_mask = R.dest_mask;
+    ex.flags = R.flags;
+    ex.ptr = (uint64_t)(uintptr_t)(R.base + R.own_off);
+    if (R.own_bytes) alloc_base_and_handle(R.base + R.own_off, &ex.data_handle, &ex.data_off, &ex.data_ipc_ok);
+    std::vector<RegionExchange> all(c->world);
+    rc = c->shm.allgather(c->rank, &ex, sizeof(ex), all.data());
+    if (rc) return rc;
+    rc = finish_region_peers(c, id, R, all);
+    if (rc) return rc;
+    rc = upload_ctx(c);
+    if (rc) return rc;
+    return c->shm.barrier();
+}
+
+int proact_region_set_chunk_dest(int id, uint32_t chunk, uint64_t mask)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (id < 0 || id >= c->nregions) return PROACT_ERR_INVALID;
+    Region &R = c->regions[id];
+    if (chunk >= R.n_own) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    if (R.chunk_dest.empty()) {
+        R.chunk_dest.assign(R.n_own, (uint32_t)R.dest_mask);
+        CK(cudaMalloc((void **)&R.d_chunk_dest, 4 * (size_t)R.n_own));
+        c->h.region[id].chunk_dest = R.d_chunk_dest;
+        c->h.region[id].n_in = 0xFFFFFFFFu;
+        int rc = upload_ctx(c);
+        if (rc) return rc;
+    }
+    R.chunk_dest[chunk] = (uint32_t)mask;
+    CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * (size_t)R.n_own, cudaMemcpyHostToDevice));
+    return PROACT_OK;
+}
+
+int proact_region_info_get(int id, proact_region_info *out)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (id < 0 || id >= c->nregions || !out) return PROACT_ERR_INVALID;
+    const Region &R = c->regions[id];
+    memset(out, 0, sizeof(*out));
+    out->replica_base = R.base;
+    out->own_offset = R.own_off;
+    out->own_bytes = R.own_bytes;
+    out->total_bytes = R.total;
+    out->chunk_bytes = R.chunk;
+    out->n_own_chunks = R.n_own;
+    out->n_total_chunks = R.n_total;
+    out->first_chunk = R.chunk0;
+    out->generation = R.gen_done;
+    out->dest_mask = R.dest_mask;
+    for (int p = 0; p <= c->world; ++p) out->rank_offset[p] = R.rank_off[p];
+    return PROACT_OK;
+}
+
+int proact_region_debug_deliveries(int id, uint32_t *out, size_t n)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (id < 0 || id >= c->nregions || !out) return PROACT_ERR_INVALID;
+    const region_dev &D = c->h.region[id];
+    size_t need = (size_t)c->regions[id].n_own * c->world;
+    if (!D.deliv || n < need) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CK(cudaDeviceSynchronize());
+    if (need) {
+        CK(cudaMemcpy(out, D.deliv, 4 * need, cudaMemcpyDeviceToHost));
+        CK(cudaMemset(D.deliv, 0, 4 * need));
+    }
+    return PROACT_OK;
+}
+
+int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
+                  void **args, size_t smem, void *stream)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (!kernel || !args || !args[0] || nregions < 0 || (nregions && !regions)) return PROACT_ERR_INVALID;
+    int rc = check_latched(c);
+    if (rc) return rc;
+    cudaSetDevice(c->device);
+    const proact_config &cfg = c->cfg;
+    if (block == 0) block = (unsigned)cfg.block;
+    if (block % 32 || block > 1024) return PROACT_ERR_INVALID;
+    launch_ctx lc;
+    memset(&lc, 0, sizeof(lc));
+    lc.ctx = c->d;
+    lc.epoch = c->epoch;
+    lc.mech = (uint16_t)cfg.mech;
+    lc.push = (uint16_t)cfg.push;
+    lc.piece_bytes = cfg.piece_bytes;
+    uint32_t armed = 0;
+    for (int i = 0; i < nregions; ++i) {
+        int r = regions[i];
+        if (r < 0 || r >= c->nregions) return PROACT_ERR_INVALID;
+        if (c->regions[r].last_armed_epoch == (int64_t)c->epoch) return PROACT_ERR_STATE;
+        armed |= 1u << r;
+    }
+    lc.armed = armed;
+    for (int r = 0; r < c->nregions; ++r) {
+        const Region &R = c->regions[r];
+        lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
+        lc.gen_epoch[r] = (armed >> r & 1) ? c->epoch : R.gen_epoch;
+    }
+    bool agent = (cfg.mech == PROACT_MECH_FUSED || cfg.mech == PROACT_MECH_ELIDE) && armed;
+    unsigned wpc = block / 32;
+    unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
+    lc.agent_ctas = (uint16_t)agent_ctas;
+    lc.agent_warps = (uint16_t)(agent ? cfg.agent_warps : 0);
+    int nb = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
+    if (nb < 1) return PROACT_ERR_INVALID;
+    unsigned cap = (unsigned)std::max(1, nb * c->nsm / std::max(1, c->ranks_on_device));
+    if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
+    unsigned total = agent_ctas + (grid ? grid : cap);
+    if (total > cap) total = cap;
+    if (total <= agent_ctas) return PROACT_ERR_INVALID;
+    *(launch_ctx *)args[0] = lc;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->coop && agent)
+        CK(cudaLaunchCooperativeKernel(kernel, dim3(total), dim3(block), args, smem, s));
+    else
+        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+    for (int r = 0; r < c->nregions; ++r) {
+        if (!(armed >> r & 1)) continue;
+        Region &R = c->regions[r];
+        R.gen_done += 1;
+        R.gen_epoch = c->epoch;
+        R.last_armed_epoch = c->epoch;
+    }
+    c->armed_epoch_mask |= armed;
+    if (cfg.mech == PROACT_MECH_BULK) c->bulk_mask |= armed;
+    c->launches++;
+    return PROACT_OK;
+}
+
+int proact_phase_sync(void *stream, int mode)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (mode != PROACT_SYNC_SIGNAL && mode != PROACT_SYNC_BARRIER) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->bulk_mask) {
+        // cudaMemcpy duplication: copy my slice to each destination after the
+        // producer kernel, once the destination finished reading its previous replica.
+        uint32_t peers = 0;
+        for (int r = 0; r < c->nregions; ++r)
+            if (c->bulk_mask >> r & 1) {
+                const Region &R = c->regions[r];
+                if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
+                else peers |= (uint32_t)R.dest_mask;
+            }
+        peers &= ~(1u << c->rank);
+        if (peers) {
+            credit_wait_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, peers);
+            CK(cudaGetLastError());
+            c->launches++;
+        }
+        for (int r = 0; r < c->nregions; ++r) {
+            if (!(c->bulk_mask >> r & 1)) continue;
+            const Region &R = c->regions[r];
+            const region_dev &D = c->h.region[r];
+            for (int p = 0; p < c->world; ++p) {
+                if (p == c->rank) continue;
+                if (R.chunk_dest.empty()) {
+                    if (!(R.dest_mask >> p & 1) || !R.own_bytes) continue;
+                    CK(cudaMemcpyAsync(D.peer_base[p] + R.own_off, R.base + R.own_off, R.own_bytes,
+                                       cudaMemcpyDeviceToDevice, s));
+                } else {   // per-chunk destinations: copy maximal runs of chunks bound for p
+                    uint32_t k = 0;
+                    while (k < R.n_own) {
+                        if (!(R.chunk_dest[k] >> p & 1)) { ++k; continue; }
+                        uint32_t k1 = k;
+                        while (k1 < R.n_own && (R.chunk_dest[k1] >> p & 1)) ++k1;
+                        uint64_t lo = R.own_off + (uint64_t)k * R.chunk;
+                        uint64_t hi = std::min<uint64_t>(R.own_off + (uint64_t)k1 * R.chunk, R.own_off + R.own_bytes);
+                        CK(cudaMemcpyAsync(D.peer_base[p] + lo, R.base + lo, hi - lo, cudaMemcpyDeviceToDevice, s));
+                        k = k1;
+                    }
+                }
+            }
+        }
+    }
+    sync_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, mode);
+    CK(cudaGetLastError());
+    c->launches++;
+    c->epoch++;
+    c->armed_epoch_mask = 0;
+    c->bulk_mask = 0;
+    return check_latched(c);
+}
+
+int proact_last_vote(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return -1;
+    uint32_t v = *(volatile uint32_t *)c->h_vote;
+    if ((v >> 1) != c->epoch) return -1;   // not the most recent phase
+    return (int)(v & 1u);
+}
+
+int proact_check(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    return check_latched(c);
+}
+
+int proact_finalize(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    int rc = c->shm.barrier();   // every rank stopped touching peers' memory
+    for (int r = 0; r < c->nregions; ++r) {
+        Region &R = c->regions[r];
+        for (void *p : R.opened) cudaIpcCloseMemHandle(p);
+        if (R.meta) cudaFree(R.meta);
+        if (R.d_chunk_dest) cudaFree(R.d_chunk_dest);
+    }
+    for (void *p : c->opened) cudaIpcCloseMemHandle(p);
+    int rc2 = c->shm.barrier();  // nobody uses our memory any more
+    cudaFree(c->d);
+    cudaFree(c->meta);
+    cudaFreeHost(c->h_err);
+    c->shm.close(true);
+    int latched = c->latched;
+    tl = nullptr;
+    delete c;
+    if (rc) return rc;
+    if (rc2) return rc2;
+    return latched;
+}
+
+// --------------------------------------------------------------------------------- profiler (a9)
+static std::mutex g_tune_mu;
+
+static std::string cache_path()
+{
+    const char *p = getenv("PROACT_TUNE_CACHE");
+    return p && *p ? p : "proact_tune.json";
+}
+
+// cache format: one JSON object, key -> {"mech":..,"agent_warps":..,"piece_bytes":..,"chunk_bytes":..,"ms":..}
+static bool cache_lookup(const std::string &key, proact_config *out)
+{
+    FILE *f = fopen(cache_path().c_str(), "r");
+    if (!f) return false;
+    std::string s;
+    char buf[4096];
+    size_t n;
+    while ((n = fread(buf, 1, sizeof buf, f)) > 0) s.append(buf, n);
+    fclose(f);
+    std::string pat = "\"" + key + "\"";
+    size_t k = s.find(pat);
+    if (k == std::string::npos) return false;
+    size_t b = s.find('{', k), e = s.find('}', b);
+    if (b == std::string::npos || e == std::string::npos) return false;
+    std::string obj = s.substr(b, e - b);
+    auto get = [&](const char *f2, long long dflt) {
+        std::string q = std::string("\"") + f2 + "\":";
+        size_t i = obj.find(q);
+        return i == std::string::npos ? dflt : atoll(obj.c_str() + i + q.size());
+    };
+    *out = default_config();
+    out->mech = (int)get("mech", out->mech);
+    out->agent_warps = (int)get("agent_warps", out->agent_warps);
+    out->piece_bytes = (uint32_t)get("piece_bytes", out->piece_bytes);
+    out->chunk_bytes = (uint32_t)get("chunk_bytes", out->chunk_bytes);
+    return true;
+}
+
+static void cache_store(const std::string &key, const proact_config &c, double ms)
+{
+    std::lock_guard<std::mutex> lk(g_tune_mu);
+    std::string path = cache_path(), s;
+    if (FILE *f = fopen(path.c_str(), "r")) {
+        char buf[4096];
+        size_t n;
+        while ((n = fread(buf, 1, sizeof buf, f)) > 0) s.append(buf, n);
+        fclose(f);
+    }
+    // drop an existing entry for key, then append
+    std::string pat = "\"" + key + "\"";
+    size_t k = s.find(pat);
+    if (k != std::string::npos) {
+        size_t e = s.find('}', k);
+        size_t start = k;
+        while (start > 0 && (s[start - 1] == ' ' || s[start - 1] == '\n' || s[start - 1] == ',')) --start;
+        s.erase(start, e + 1 - start);
+    }
+    size_t open = s.find('{');
+    size_t close = s.rfind('}');
+    std::string body = (open != std::string::npos && close != std::string::npos && close > open)
+                           ? s.substr(open + 1, close - open - 1) : "";
+    while (!body.empty() && (body.back() == '\n' || body.back() == ' ' || body.back() == ',')) body.pop_back();
+    char ent[512];
+    snprintf(ent, sizeof ent,
+             "  \"%s\": {\"mech\":%d,\"agent_warps\":%d,\"piece_bytes\":%u,\"chunk_bytes\":%u,\"ms\":%.6f}",
+             key.c_str(), c.mech, c.agent_warps, c.piece_bytes, c.chunk_bytes, ms);
+    std::string out = "{\n" + body + (body.empty() ? "" : ",\n") + ent + "\n}\n";
+    std::string tmp = path + ".tmp";
+    if (FILE *f = fopen(tmp.c_str(), "w")) {
+        fwrite(out.data(), 1, out.size(), f);
+        fclose(f);
+        rename(tmp.c_str(), path.c_str());
+    }
+}
+
+static std::vector<long long> parse_list(const std::string &space, const char *name, std::vector<long long> dflt)
+{
+    std::string q = std::string(name) + "=";
+    size_t i = space.find(q);
+    if (i == std::string::npos) return dflt;
+    size_t e = space.find(';', i);
+    std::string lst = space.substr(i + q.size(), e == std::string::npos ? std::string::npos : e - i - q.size());
+    std::vector<long long> v;
+    size_t p = 0;
+    while (p < lst.size()) {
+        size_t c2 = lst.find(',', p);
+        v.push_back(atoll(lst.substr(p, c2 == std::string::npos ? std::string::npos : c2 - p).c_str()));
+        if (c2 == std::string::npos) break;
+        p = c2 + 1;
+    }
+    return v.empty() ? dflt : v;
+}
+
+int proact_autotune(const char *key, const char *space, proact_run_fn fn, void *user, proact_config *out)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (!key || !fn || !out) return PROACT_ERR_INVALID;
+    // cache hit must be agreed on by every rank
+    proact_config hit;
+    int32_t have = cache_lookup(key, &hit) ? 1 : 0;
+    std::vector<int32_t> haves(c->world);
+    int rc = c->shm.allgather(c->rank, &have, sizeof(have), haves.data());
+    if (rc) return rc;
+    bool all_have = std::all_of(haves.begin(), haves.end(), [](int32_t h) { return h == 1; });
+    if (all_have) {
+        *out = hit;
+        return PROACT_OK;
+    }
+    std::string sp = space ? space : "";
+    // Sec. III-A: mechanism x granularity x transfer threads (Table II ranges 4kB-16MB, 32-8192)
+    auto mechs = parse_list(sp, "mech", {PROACT_MECH_FUSED, PROACT_MECH_INLINE});
+    auto chunks = parse_list(sp, "chunk", {(long long)c->cfg.chunk_bytes});
+    auto warps = parse_list(sp, "warps", {4, 8, 16, 32, 64});
+    auto pieces = parse_list(sp, "piece", {(long long)c->cfg.piece_bytes});
+    proact_config base = c->cfg, best = base;
+    double best_ms = 1e300;
+    for (long long m : mechs)
+        for (long long ch : chunks)
+            for (long long w : warps)
+                for (long long pc : pieces) {
+                    bool agent = m == PROACT_MECH_FUSED || m == PROACT_MECH_ELIDE;
+                    // non-agent mechanisms ignore warps/piece: run them once
+                    if (!agent && (w != warps[0] || pc != pieces[0])) continue;
+                    proact_config t = base;
+                    t.mech = (int)m;
+                    t.chunk_bytes = (uint32_t)ch;
+                    t.agent_warps = (int)w;
+                    t.piece_bytes = (uint32_t)pc;
+                    double ms = -1.0;
+                    if (validate_config(t) == PROACT_OK && proact_set_config(&t) == PROACT_OK) ms = fn(&t, user);
+                    std::vector<double> all(c->world);
+                    rc = c->shm.allgather(c->rank, &ms, sizeof(ms), all.data());
+                    if (rc) { proact_set_config(&base); return rc; }
+                    double worst = 0;
+                    bool ok = true;
+                    for (double x : all) { if (x < 0) ok = false; worst = std::max(worst, x); }
+                    if (ok && worst < best_ms) { best_ms = worst; best = t; }
+                }
+    proact_set_config(&base);
+    if (best_ms >= 1e300) return PROACT_ERR_INVALID;
+    if (c->rank == 0) cache_store(key, best, best_ms);
+    rc = c->shm.barrier();
+    *out = best;
+    return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,122 @@
+"""Workload drivers over the C entry points of include/proact_workloads.h.
+
+Host-side orchestration only (allocation through torch, region registration,
+the phase loop); the arithmetic of every phase runs in libproact's kernels.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import _lib
+from . import runtime as rt
+from ._lib import check
+
+
+def _s(stream) -> ctypes.c_void_p:
+    return ctypes.c_void_p(rt._stream_handle(stream))
+
+
+def row_split(N: int, G: int, g: int) -> tuple[int, int]:
+    """Rows of rank g: [g*N//G, (g+1)*N//G) (also proact_jacobi_solve_host's split)."""
+    return (N * g) // G, (N * (g + 1)) // G
+
+
+# ------------------------------------------------------------------ Jacobi (configs 1-2)
+def jacobi_phase(r_in: int, r_out: int, N: int, rows_per_tile: int = 16, stream=None) -> None:
+    check(rt.lib().proact_jacobi_phase(r_in, r_out, N, rows_per_tile, _s(stream)), "jacobi_phase")
+
+
+class Jacobi:
+    """Two replicated N x N fp32 grids (ping-pong), rows partitioned over the world.
+
+    halo_only=True sets per-chunk destinations so that only chunks holding my first/last row
+    go to the neighbours (reading R8); otherwise full replication (configs 1-2)."""
+
+    def __init__(self, N: int, chunk_bytes: int, x0: torch.Tensor | None = None,
+                 halo_only: bool = False, rows_per_tile: int = 16, device=None):
+        G, g = rt.world(), rt.rank()
+        self.N, self.G, self.g, self.rpt = N, G, g, rows_per_tile
+        dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.bufs = [torch.empty((N, N), dtype=torch.float32, device=dev) for _ in range(2)]
+        if x0 is not None:
+            self.bufs[0].copy_(x0)
+            self.bufs[1].copy_(x0)
+        # replicas must be initialised before registration: once the collective returns, peers
+        # may push into them (credits only guard later generations)
+        torch.cuda.synchronize()
+        self.r0, self.r1 = row_split(N, G, g)
+        rowb = N * 4
+        self.rid = [rt.register_region(b, self.r0 * rowb, (self.r1 - self.r0) * rowb, chunk_bytes)
+                    for b in self.bufs]
+        if halo_only:
+            self.set_halo_only()
+        self.k = 0
+
+    def set_halo_only(self) -> None:
+        rowb = self.N * 4
+        for rid in self.rid:
+            info = rt.region_info(rid)
+            cb = info.chunk_bytes
+            n = info.n_own_chunks
+            for c in range(n):
+                lo, hi = c * cb, min((c + 1) * cb, info.own_bytes)
+                m = 0
+                if self.g > 0 and lo < rowb:                       # holds my first row
+                    m |= 1 << (self.g - 1)
+                if self.g < self.G - 1 and hi > info.own_bytes - rowb:  # holds my last row
+                    m |= 1 << (self.g + 1)
+                rt.set_chunk_dest(rid, c, m)
+
+    def step(self, stream=None, barrier: bool = False) -> None:
+        i = self.k & 1
+        jacobi_phase(self.rid[i], self.rid[i ^ 1], self.N, self.rpt, stream)
+        rt.phase_sync(stream, barrier=barrier)
+        self.k += 1
+
+    @property
+    def current(self) -> torch.Tensor:
+        return self.bufs[self.k & 1]
+
+
+def jacobi_solve_host(x0_host, out_host, N: int, iters: int, chunk_bytes: int,
+                      rows_per_tile: int = 16, stream=None) -> tuple[int, int]:
+    """proact_jacobi_solve_host on host buffers (torch CPU tensors, ideally pinned)."""
+    assert x0_host.dtype == torch.float32 and out_host.dtype == torch.float32
+    assert x0_host.is_contiguous() and out_host.is_contiguous()
+    h2d, d2h = ctypes.c_ulonglong(0), ctypes.c_ulonglong(0)
+    check(rt.lib().proact_jacobi_solve_host(ctypes.c_void_p(x0_host.data_ptr()),
+                                            ctypes.c_void_p(out_host.data_ptr()), N, iters,
+                                            chunk_bytes, rows_per_tile, _s(stream),
+                                            ctypes.byref(h2d), ctypes.byref(d2h)), "jacobi_solve_host")
+    return h2d.value, d2h.value
+
+
+# ------------------------------------------------------------------ microbenchmark (config 5)
+def micro_phase(rid: int, phase: int, seed: int, K: int = 1, scattered: bool = False,
+                stream=None) -> None:
+    check(rt.lib().proact_micro_phase(rid, phase & 0xFFFFFFFF, seed & 0xFFFFFFFF, K,
+                                      int(scattered), _s(stream)), "micro_phase")
+
+
+class Micro:
+    """A replicated region of `words` u32 words, all-gather shape (every rank produces W/G)."""
+
+    def __init__(self, words: int, chunk_bytes: int, device=None, dest_mask: int | None = None):
+        G, g = rt.world(), rt.rank()
+        dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+        # slices are 4-word (16 B) aligned: rank g owns words [lo_g, lo_{g+1})
+        bounds = [((words * p) // G) // 4 * 4 for p in range(G)] + [words]
+        self.lo, self.hi = bounds[g], bounds[g + 1]
+        self.buf = torch.zeros(words, dtype=torch.int32, device=dev)
+        torch.cuda.synchronize()
+        self.rid = rt.register_region(self.buf, self.lo * 4, (self.hi - self.lo) * 4, chunk_bytes,
+                                      dest_mask)
+        self.phase = 0
+
+    def step(self, seed: int, K: int = 1, scattered: bool = False, stream=None,
+             barrier: bool = False) -> None:
+        micro_phase(self.rid, self.phase, seed, K, scattered, stream)
+        rt.phase_sync(stream, barrier=barrier)
+        self.phase += 1

@@ -1,0 +1,135 @@
+"""GPU parity: the CUDA Jacobi path (through the C ABI) vs the CPU oracle, bit-exact.
+
+Reading R10: fixed association, fp32 round-to-nearest, no FMA on both
+sides, so the replicas must equal the oracle bit for bit (the north star's 1e-5
+relative bound is implied).  Multi-rank cases run G ranks as threads on one GPU
+(loopback: peers are other buffers of the same device; every kernel, flag,
+credit and push of the protocol runs unchanged).
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks
+from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+
+pytestmark = pytest.mark.gpu
+
+
+def _run_jacobi(r, G, N, iters, chunk, mech, halo_only=False, rpt=16, check_deliv=False):
+    rt.set_config(mech=mech, watchdog_ms=20000)
+    x0 = torch.from_numpy(synth.jacobi_init(N)).cuda()
+    J = wl.Jacobi(N, chunk, x0=x0, halo_only=halo_only, rows_per_tile=rpt)
+    s = torch.cuda.Stream()
+    deliv = []
+    with torch.cuda.stream(s):
+        for k in range(iters):
+            J.step(s, barrier=(k == iters - 1))
+            if check_deliv:
+                s.synchronize()
+                deliv.append(rt.debug_deliveries(J.rid[(k + 1) & 1]).copy())
+    s.synchronize()
+    rt.check_device()
+    return J.current.cpu().numpy(), (J.r0, J.r1), deliv
+
+
+@pytest.mark.parametrize("mech", [_lib.MECH_FUSED, _lib.MECH_INLINE, _lib.MECH_BULK])
+def test_config1_jacobi_1024_two_ranks_bit_exact(mech):
+    """BASELINE.json config 1: 1024x1024 fp32, 2 row partitions, 10 iterations, full replica."""
+    N, iters = 1024, 10
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(2, _run_jacobi, N, iters, 64 * 1024, mech)
+    for g, (rep, _, _) in enumerate(outs):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), f"rank {g} mech {mech}"
+
+
+@pytest.mark.parametrize("G,N,chunk,rpt", [(1, 2048, 4096, 16), (3, 1000, 12288, 16),
+                                           (4, 520, 4096, 7), (2, 4100, 1 << 20, 32)])
+def test_jacobi_ragged_ranks_chunks_tiles(G, N, chunk, rpt):
+    iters = 6
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(G, _run_jacobi, N, iters, chunk, _lib.MECH_FUSED, rpt=rpt)
+    for g, (rep, _, _) in enumerate(outs):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), f"rank {g}"
+
+
+def test_jacobi_halo_only_owned_rows_and_halos():
+    G, N, iters = 4, 512, 9
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(G, _run_jacobi, N, iters, 8192, _lib.MECH_FUSED, halo_only=True)
+    for g, (rep, (r0, r1), _) in enumerate(outs):
+        lo, hi = max(r0 - 1, 0), min(r1 + 1, N)
+        assert np.array_equal(rep[lo:hi].view(np.uint32), want[lo:hi].view(np.uint32)), g
+
+
+def test_jacobi_exactly_once_delivery():
+    os.environ["PROACT_DEBUG"] = "1"
+    try:
+        G, N, iters = 3, 768, 4
+        outs = run_ranks(G, _run_jacobi, N, iters, 4096, _lib.MECH_FUSED, check_deliv=True)
+    finally:
+        del os.environ["PROACT_DEBUG"]
+    for g, (_, _, deliv) in enumerate(outs):
+        assert len(deliv) == iters
+        for d in deliv:
+            want = np.ones_like(d)
+            want[:, g] = 0
+            assert np.array_equal(d, want), f"rank {g}: {d}"
+
+
+@pytest.mark.parametrize("mech", [_lib.MECH_FUSED, _lib.MECH_LOCAL, _lib.MECH_ELIDE])
+def test_jacobi_single_gpu_mechanisms(mech):
+    N, iters = 1536, 5
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    (rep, _, _), = run_ranks(1, _run_jacobi, N, iters, 128 * 1024, mech)
+    assert np.array_equal(rep.view(np.uint32), want.view(np.uint32))
+
+
+def _window_oracle(N, iters, i, j):
+    """Cell (i, j) after `iters` iterations from the (2*iters+3)^2 window of x0 around it:
+    influence travels one cell per iteration, so the window's false boundary never reaches the
+    centre (needs iters+1 <= i, j <= N-2-iters)."""
+    h = iters + 1
+    x0 = synth.jacobi_init(N, row0=i - h, nrows=2 * h + 1)[:, j - h:j + h + 1]
+    return oracle.jacobi(np.ascontiguousarray(x0), iters)[h, h]
+
+
+@pytest.mark.slow
+def test_config2_full_size_sampled():
+    """Config 2 size (16384^2, 100 iterations) in bench.py's launch configuration (G=1, FUSED),
+    checked on sampled cells computed one by one by the oracle."""
+    N, iters = 16384, 100
+    (rep, _, _), = run_ranks(1, _run_jacobi, N, iters, 128 * 1024, _lib.MECH_FUSED)
+    rng = np.random.default_rng(0)
+    pts = [(int(a), int(b)) for a, b in rng.integers(iters + 1, N - iters - 2, size=(12, 2))]
+    pts += [(iters + 1, iters + 1), (N - iters - 2, N - iters - 2), (8192, 1023), (8191, 1024)]
+    for i, j in pts:
+        assert rep[i, j] == _window_oracle(N, iters, i, j), (i, j)
+    # boundary rows/cols are copied through (Dirichlet)
+    x0 = synth.jacobi_init(N, row0=0, nrows=1)
+    assert np.array_equal(rep[0], x0[0])
+
+
+def test_jacobi_e2e_host_buffers():
+    N, iters = 512, 7
+    x0 = synth.jacobi_init(N)
+    want = oracle.jacobi(x0, iters)
+
+    def body(r, G):
+        xh = torch.from_numpy(x0).pin_memory()
+        out = torch.zeros((N, N), dtype=torch.float32).pin_memory()
+        s = torch.cuda.Stream()
+        h2d, d2h = wl.jacobi_solve_host(xh, out, N, iters, 16384, stream=s)
+        s.synchronize()
+        r0, r1 = wl.row_split(N, G, r)
+        return out.numpy()[r0:r1].copy(), (r0, r1), h2d, d2h
+
+    outs = run_ranks(2, body)
+    for rows, (r0, r1), h2d, d2h in outs:
+        assert np.array_equal(rows, want[r0:r1])
+        assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4

@@ -1,0 +1,103 @@
+"""GPU parity for the transfer microbenchmark (config 5 shape) and protocol invariants.
+
+Replica bytes must equal the closed form (oracle.micro_phase) bit-exactly on
+every rank after every phase; each (chunk, dest) delivered exactly once; a
+watchdog turns a protocol stall into PROACT_ERR_TIMEOUT instead of a hang.
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks, ProactError
+from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+
+pytestmark = pytest.mark.gpu
+SEED = 0x5EED
+
+
+def _run_micro(r, G, words, chunk, mech, phases, K, scattered, piece=None, warps=None):
+    kw = dict(mech=mech)
+    if piece:
+        kw["piece_bytes"] = piece
+    if warps:
+        kw["agent_warps"] = warps
+    rt.set_config(**kw)
+    M = wl.Micro(words, chunk)
+    s = torch.cuda.Stream()
+    snaps = []
+    for p in range(phases):
+        M.step(SEED, K, scattered, stream=s, barrier=True)
+        s.synchronize()
+        snaps.append(M.buf.cpu().numpy().view(np.uint32).copy())
+    rt.check_device()
+    return snaps
+
+
+@pytest.mark.parametrize("G,words,chunk,mech,scattered,piece", [
+    (2, 1 << 20, 4096, _lib.MECH_FUSED, False, None),
+    (2, (1 << 20) + 4 * 37, 65536, _lib.MECH_FUSED, True, 16384),
+    (4, 3_000_000, 1 << 20, _lib.MECH_FUSED, False, 65536),
+    (3, 777_776, 12288, _lib.MECH_INLINE, True, None),
+    (4, 1 << 21, 4 << 20, _lib.MECH_BULK, False, None),
+    (1, 1 << 20, 4096, _lib.MECH_FUSED, False, None),
+])
+def test_micro_replicas_equal_closed_form(G, words, chunk, mech, scattered, piece):
+    phases, K = 3, 2
+    outs = run_ranks(G, _run_micro, words, chunk, mech, phases, K, scattered, piece=piece)
+    for p in range(phases):
+        want = oracle.micro_phase(words, p, SEED, K)
+        for g in range(G):
+            assert np.array_equal(outs[g][p], want), (p, g)
+
+
+def test_micro_exactly_once_and_counters():
+    os.environ["PROACT_DEBUG"] = "1"
+
+    def body(r, G):
+        rt.set_config(mech=_lib.MECH_FUSED, piece_bytes=8192, agent_warps=3)
+        M = wl.Micro(1 << 20, 65536)
+        s = torch.cuda.Stream()
+        out = []
+        for p in range(3):
+            M.step(SEED, 1, False, stream=s, barrier=True)
+            s.synchronize()
+            out.append(rt.debug_deliveries(M.rid).copy())
+        return out
+
+    try:
+        outs = run_ranks(3, body)
+    finally:
+        del os.environ["PROACT_DEBUG"]
+    for g, ds in enumerate(outs):
+        for d in ds:
+            want = np.ones_like(d)
+            want[:, g] = 0
+            assert np.array_equal(d, want)
+
+
+def test_watchdog_turns_a_stall_into_timeout():
+    """A consumer waiting for data that no producer will ever publish must time out, not hang
+    (fault injection T5): rank 1 never launches phase 0, rank 0 waits for its credit."""
+
+    def body(r, G):
+        rt.set_config(mech=_lib.MECH_FUSED, watchdog_ms=300)
+        M = wl.Micro(1 << 16, 4096)
+        s = torch.cuda.Stream()
+        if r == 0:
+            wl.micro_phase(M.rid, 0, SEED, stream=s)
+            try:
+                rt.phase_sync(s, barrier=True)   # waits for rank 1's credit forever
+                s.synchronize()
+                rt.check_device()
+            except ProactError as e:
+                return e.code
+            return 0
+        s.synchronize()
+        return None
+
+    res = run_ranks(2, body)
+    assert res[0] == _lib.ERR_TIMEOUT
