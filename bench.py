@@ -1,0 +1,327 @@
+#!/usr/bin/env python
+"""bench.py -- PROACT hot path on B200: BASELINE.json's metric on config 2 (Jacobi 16384^2).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl proact|reference]
+                    [--mech fused|inline|bulk|local|elide] [--chunk BYTES] [--iters I]
+
+One STEP = one full solve of BASELINE.json config 2: I = 100 Jacobi phases of the
+16384 x 16384 fp32 grid, rows strong-scaled over the N ranks, each phase = producer
+kernel with fused transfer agent (tracking, polling, pushes, arrival flags) + phase
+sync (credits).  value = iterations/s of the whole job (K*I / max-over-ranks time).
+The grid (1 GiB per buffer) is far larger than L2 (126 MB), so no flush is needed.
+
+Extra keys: roofline (dominant kernel = jacobi_kernel, HBM bound, measured live with
+CUDA events on its stream), cpu_baseline (the oracle, rank 0, bounded sample), e2e
+(proact_jacobi_solve_host with pinned host buffers: H2D of the grid + I phases + D2H),
+clocks (nvidia-smi sampled during the timed region), gpu_launches, overhead (the
+same step with the uninstrumented LOCAL mechanism: the paper's tracking-overhead
+decomposition, Sec. V-C).
+
+--impl reference: the CPU oracle (oracle/) timed as it stands on the host cores, on
+the same config/metric; rank 0 only under torchrun.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "strong-scaling speedup and iters/sec at 1/2/4/8 B200; NVLink GB/s vs 900 GB/s"
+N_GRID = 16384
+ITERS = 100
+WORKLOAD = "jacobi2d_5pt_fp32_16384x16384_100it (BASELINE.json config 2, full replication)"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+def _traffic_from_profiles():
+    """dram bytes per launch of jacobi_kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_jacobi_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.path = f"/tmp/proact_clocks_{os.getpid()}.csv"
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(5)
+            except Exception:
+                self.proc.kill()
+            self.f.close()
+
+    def summary(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        try:
+            os.remove(self.path)
+        except OSError:
+            pass
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(N: int, budget_s: float = 12.0) -> dict:
+    """The oracle as it stands (oracle.jacobi_step, OpenMP over all host cores) on the full
+    16384^2 grid, iterated until ~budget_s of CPU work (bounded sample)."""
+    import numpy as np
+    import oracle
+    import synth
+    x = synth.jacobi_init(N)
+    oracle.jacobi_step(x)   # page in / warm
+    t0 = time.perf_counter()
+    k = 0
+    while True:
+        x = oracle.jacobi_step(x)
+        k += 1
+        if time.perf_counter() - t0 > budget_s or k >= ITERS:
+            break
+    dt = time.perf_counter() - t0
+    del np
+    return {"value": k / dt, "unit": "iters/s", "cores": oracle.get_threads(), "kind": "oracle",
+            "sample": f"{k} Jacobi iterations of the full {N}x{N} fp32 grid (oracle.jacobi_step)"}
+
+
+def run_reference(args, dist_rank: int) -> None:
+    if dist_rank != 0:
+        return
+    N = args.n
+    cb = cpu_baseline(N, budget_s=max(2.0, 60.0 / max(1, args.steps + args.warmup)))
+    # each step: a bounded sample of the workload (cb's iterations), timed on the host
+    import oracle
+    import synth
+    x = synth.jacobi_init(N)
+    per = max(1, int(round(cb["value"] * 3.0)))   # ~3 s of oracle work per step
+    for _ in range(args.warmup):
+        x = oracle.jacobi_step(x)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for _ in range(per):
+            x = oracle.jacobi_step(x)
+    dt = time.perf_counter() - t0
+    v = args.steps * per / dt
+    cbr = dict(cb)
+    cbr["value"] = v
+    cbr["sample"] = f"{args.steps} steps x {per} oracle Jacobi iterations of the {N}x{N} grid"
+    line = {"metric": METRIC, "value": v, "unit": "iters/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1000.0 * dt / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "impl": "reference", "config": {"workload": WORKLOAD, "N": N, "iters_per_step": per},
+            "cpu_baseline": cbr, "e2e": {"value": v, "unit": "iters/s", "h2d_bytes_per_step": 0,
+                                         "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="proact", choices=["proact", "reference"])
+    ap.add_argument("--mech", default="fused")
+    ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--warps", type=int, default=0)
+    ap.add_argument("--rpt", type=int, default=16)
+    ap.add_argument("--iters", type=int, default=ITERS)
+    ap.add_argument("--n", type=int, default=N_GRID)
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_muthukrishnannl21_b200 import _lib
+    from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+    from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+    import synth
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        job = f"bench_{os.environ.get('MASTER_ADDR', '')}_{os.environ.get('MASTER_PORT', '')}"
+    else:
+        job = rt.new_job_key()
+    rt.init(world, rank, job)
+    mech = {v: k for k, v in _lib.MECH_NAMES.items()}[args.mech]
+    cfg = rt.get_config()
+    chunk = args.chunk or cfg["chunk_bytes"]
+    kw = {"mech": mech}
+    if args.warps:
+        kw["agent_warps"] = args.warps
+    cfg = rt.set_config(**kw)
+    N, I = args.n, args.iters
+    x0 = torch.from_numpy(synth.jacobi_init(N)).cuda()
+    J = wl.Jacobi(N, chunk, x0=x0, rows_per_tile=args.rpt)
+    del x0
+    s = torch.cuda.Stream()
+
+    def step():
+        for k in range(I):
+            J.step(s, barrier=(k == I - 1))
+
+    def timed(fn, K):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(K):
+            fn()
+        e1.record(s)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ms = e0.elapsed_time(e1)
+        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    l0 = rt.launch_count()
+    with Clocks(local) as clk:
+        ms = timed(step, args.steps)
+    launches = rt.launch_count() - l0
+    rt.check_device()
+    value = args.steps * I / (ms / 1000.0)
+
+    # ---- roofline of the dominant kernel: per-launch CUDA events around jacobi_kernel
+    evs = []
+    for k in range(2 * 10):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        i = J.k & 1
+        a.record(s)
+        wl.jacobi_phase(J.rid[i], J.rid[i ^ 1], N, J.rpt, s)
+        b.record(s)
+        rt.phase_sync(s, barrier=False)
+        J.k += 1
+        evs.append((a, b))
+    torch.cuda.synchronize()
+    kms = statistics.mean(a.elapsed_time(b) for a, b in evs)
+    nrows = J.r1 - J.r0
+    alg_bytes = 8.0 * N * nrows          # read x^k + write x^{k+1} of my rows
+    peaks, src = _peaks()
+    peak = float(peaks.get("hbm_gbs", 6650.0))
+    achieved = alg_bytes / (kms / 1000.0) / 1e9
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": _traffic_from_profiles(),
+                "kernel": "jacobi_kernel", "kernel_ms": kms, "alg_bytes_per_launch": alg_bytes,
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({src})"}
+
+    # ---- tracking overhead: same step, uninstrumented LOCAL mechanism (G=1 only meaningful)
+    overhead = None
+    if world == 1:
+        rt.set_config(mech=_lib.MECH_LOCAL)
+        step()
+        ms_local = timed(step, max(2, args.steps // 2))
+        v_local = max(2, args.steps // 2) * I / (ms_local / 1000.0)
+        overhead = {"local_iters_per_s": v_local, "fused_iters_per_s": value,
+                    "tracking_overhead_frac": v_local / value - 1.0}
+        rt.set_config(mech=mech)
+
+    # ---- e2e through the C-ABI host-buffer entry point
+    e2e = None
+    if not args.no_e2e:
+        xh = torch.from_numpy(synth.jacobi_init(N)).pin_memory()
+        out = torch.empty((N, N), dtype=torch.float32).pin_memory()
+        nb = [0, 0]
+
+        def e2e_step():
+            h, d = wl.jacobi_solve_host(xh, out, N, I, chunk, args.rpt, s)
+            nb[0], nb[1] = h, d
+
+        e2e_step()
+        torch.cuda.synchronize()
+        ems = timed(e2e_step, max(2, min(args.steps, 3)))
+        e2e = {"value": max(2, min(args.steps, 3)) * I / (ems / 1000.0), "unit": "iters/s",
+               "h2d_bytes_per_step": nb[0], "d2h_bytes_per_step": nb[1],
+               "api": "proact_jacobi_solve_host"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(N)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "iters/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+                "dtype": "f32", "data": "synthetic",
+                "config": {"workload": WORKLOAD, "N": N, "iters_per_step": I, "ranks": world,
+                           "mech": args.mech, "chunk_bytes": chunk,
+                           "agent_warps": cfg["agent_warps"], "piece_bytes": cfg["piece_bytes"],
+                           "rows_per_tile": args.rpt, "replication": "full",
+                           "l2": "inputs > L2 (two 1 GiB grids), no flush",
+                           "parallelism": f"rows{world}"},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead}
+        print(json.dumps(line), flush=True)
+    torch.cuda.synchronize()
+    rt.finalize()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

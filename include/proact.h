@@ -195,6 +195,10 @@ int proact_last_vote(void);
  * the device.  INVALID if debug counters are off or n is too small. */
 int proact_region_debug_deliveries(int region, uint32_t *out, size_t n);
 
+/* COLLECTIVE host-side barrier of all ranks (no device work): e.g. to read replicas from the
+ * host between phases without a peer's next phase overwriting them. */
+int proact_host_barrier(void);
+
 /* Non-blocking check of the device error word. */
 int proact_check(void);
 /* Kernels launched by this rank so far (producer/agent grids, sync kernels, helper kernels). */

@@ -83,6 +83,7 @@ def _declare(L):
         "proact_phase_sync": (i, [vp, i]),
         "proact_last_vote": (i, []),
         "proact_check": (i, []),
+        "proact_host_barrier": (i, []),
         "proact_launch_count": (u64, []),
         "proact_epoch": (u32, []),
         "proact_autotune": (i, [cp, cp, RUN_FN, vp, ctypes.POINTER(Config)]),

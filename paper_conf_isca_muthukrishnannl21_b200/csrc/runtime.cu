@@ -904,12 +904,17 @@ int proact_finalize(void)
     cudaFree(c->meta);
     cudaFreeHost(c->h_err);
     c->shm.close(true);
-    int latched = c->latched;
     tl = nullptr;
     delete c;
     if (rc) return rc;
-    if (rc2) return rc2;
-    return latched;
+    return rc2;   // a device error latched earlier was already reported by the call that saw it
+}
+
+int proact_host_barrier(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    return c->shm.barrier();
 }
 
 // --------------------------------------------------------------------------------- profiler (a9)

@@ -26,6 +26,7 @@ namespace {
 // lanes whose spans fall in the same chunk are merged into one release atomic (a3).
 __device__ __forceinline__ void warp_commit(const launch_ctx &lc, int r, bool has, uint64_t off, uint32_t nb)
 {
+    if (!proact::uses_agent(lc)) return;
     const region_dev &R = lc.ctx->region[r];
     uint64_t rel = off - R.own_off;
     uint32_t c = has ? (uint32_t)(rel / R.chunk_bytes) : 0xFFFFFFFFu;

@@ -139,6 +139,10 @@ def last_vote() -> int:
     return lib().proact_last_vote()
 
 
+def host_barrier() -> None:
+    check(lib().proact_host_barrier(), "proact_host_barrier")
+
+
 def check_device() -> None:
     check(lib().proact_check(), "proact_check")
 

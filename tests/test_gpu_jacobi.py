@@ -33,6 +33,7 @@ def _run_jacobi(r, G, N, iters, chunk, mech, halo_only=False, rpt=16, check_deli
             if check_deliv:
                 s.synchronize()
                 deliv.append(rt.debug_deliveries(J.rid[(k + 1) & 1]).copy())
+                rt.host_barrier()
     s.synchronize()
     rt.check_device()
     return J.current.cpu().numpy(), (J.r0, J.r1), deliv

@@ -33,6 +33,7 @@ def _run_micro(r, G, words, chunk, mech, phases, K, scattered, piece=None, warps
         M.step(SEED, K, scattered, stream=s, barrier=True)
         s.synchronize()
         snaps.append(M.buf.cpu().numpy().view(np.uint32).copy())
+        rt.host_barrier()   # no peer may start phase p+1 (and overwrite) before every snapshot
     rt.check_device()
     return snaps
 
@@ -66,6 +67,7 @@ def test_micro_exactly_once_and_counters():
             M.step(SEED, 1, False, stream=s, barrier=True)
             s.synchronize()
             out.append(rt.debug_deliveries(M.rid).copy())
+            rt.host_barrier()
         return out
 
     try:
