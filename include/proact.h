@@ -72,6 +72,14 @@ enum {
     PROACT_PUSH_BULK = 1     /* cp.async.bulk (TMA) global->smem->peer global, one lane issues */
 };
 
+/* ---- agent discovery of completed chunks (a4) ------------------------------------------- */
+enum {
+    PROACT_DISCOVER_QUEUE = 0, /* the last committer of a chunk enqueues its pieces; agent warps
+                                  pop them in completion order (O(1) per chunk, no scanning) */
+    PROACT_DISCOVER_SCAN = 1   /* agent warps poll the readiness counters of statically owned
+                                  32-unit windows and claim ready ones with a warp ballot */
+};
+
 /* ---- phase synchronisation modes (a8) ----------------------------------------------------- */
 enum {
     PROACT_SYNC_SIGNAL = 0,  /* credit peers "phase e done"; consumers rely on arrival flags */
@@ -91,10 +99,12 @@ typedef struct proact_config {
     int32_t push;          /* PROACT_PUSH_* */
     int32_t agent_warps;   /* transfer warps (Table II "transfer thread count" / 32) */
     int32_t block;         /* threads per CTA of fused launches (agent CTAs use the same) */
-    uint32_t piece_bytes;  /* agent work unit inside a chunk (multiple of 16) */
+    uint32_t piece_bytes;  /* agent work unit inside a chunk (multiple of 16, >= 4096) */
     uint32_t watchdog_ms;  /* device spin budget before PROACT_ERR_TIMEOUT */
     int32_t grid_cap;      /* 0 = fill the device share; else max CTAs of a fused launch */
     uint32_t chunk_bytes;  /* preferred chunk size for workload drivers (profiler axis) */
+    int32_t discovery;     /* PROACT_DISCOVER_*: how agents find completed chunks (a4) */
+    int32_t reserved;
 } proact_config;
 
 /* Geometry of a registered region as seen by the calling rank. */

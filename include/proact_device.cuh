@@ -61,6 +61,10 @@ struct region_dev {
     uint32_t *arrive;           /* [n_total] consumer-side flags: gen << 1 | changed */
     uint32_t *arrive_count;     /* monotonic count of chunks that arrived from peers */
     uint32_t *deliv;            /* debug: [n_own * world] deliveries, or nullptr */
+    unsigned long long *queue;  /* [qcap] ready units (gen << 32 | unit), QUEUE discovery */
+    uint32_t *qctl;             /* [8]: tail[2], head[2] by generation parity, agents_done */
+    uint32_t qcap;              /* queue capacity in units */
+    uint32_t pad_q;
     uint64_t rank_off[PROACT_MAX_RANKS + 1];
     uint32_t rank_chunk0[PROACT_MAX_RANKS + 1];
     char *peer_base[PROACT_MAX_RANKS];            /* peers' replica bases (mapped) */
@@ -93,7 +97,8 @@ struct launch_ctx {
     uint16_t agent_ctas;                       /* leading CTAs that run the agent (FUSED/ELIDE) */
     uint16_t agent_warps;                      /* warps of those CTAs that poll/push */
     uint32_t piece_bytes;                      /* agent work unit */
-    uint32_t flags;                            /* reserved */
+    uint16_t discovery;                        /* PROACT_DISCOVER_* */
+    uint16_t flags;                            /* reserved */
 };
 
 /* error word encoding: (site << 8) | (-PROACT_ERR_*) */
@@ -113,6 +118,12 @@ __device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t *p)
 {
     uint32_t v;
     asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_gpu(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ uint32_t ld_relaxed_sys(const uint32_t *p)
@@ -236,6 +247,41 @@ __device__ __forceinline__ void put(const launch_ctx &lc, int r, uint64_t off, c
     }
 }
 
+/* Pieces of my chunk c under piece size `piece` (agent work units). */
+__device__ __forceinline__ uint32_t pieces_of(const region_dev &R, uint32_t c, uint32_t piece)
+{
+    return (chunk_len(R, c) + piece - 1) / piece;
+}
+__device__ __forceinline__ uint32_t piece_size(const launch_ctx &lc, const region_dev &R)
+{
+    return lc.piece_bytes < R.chunk_bytes ? lc.piece_bytes : R.chunk_bytes;
+}
+
+/* Add `b` committed bytes to my chunk c of region r (a3).  The RMW is acq_rel: release publishes
+ * this CTA's stores; acquire lets the LAST committer (old + b == expected, decided from the
+ * returned value, reading R2) hand the chunk to the agent with everything ordered before it:
+ * under QUEUE discovery it enqueues the chunk's pieces with release stores. */
+__device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32_t c, uint32_t b)
+{
+    const region_dev &R = lc.ctx->region[r];
+    const uint32_t old = atom_add_acqrel_gpu(&R.counter[c], b);
+    const uint32_t ex = R.expected[c];
+    if (old + b > ex) {
+        raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
+    } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE) {
+        const uint32_t piece = piece_size(lc, R);
+        const uint32_t P = (R.chunk_bytes + piece - 1) / piece;
+        const uint32_t np = pieces_of(R, c, piece);
+        const uint32_t gen = lc.gen[r];
+        const uint32_t idx = atomicAdd(&R.qctl[gen & 1u], np);
+        fence_acq_rel_gpu();   // one release fence for all np entries (fence + relaxed stores)
+        for (uint32_t k = 0; k < np; ++k) {
+            const unsigned long long e = ((unsigned long long)gen << 32) | (unsigned long long)(c * P + k);
+            asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(R.queue + idx + k), "l"(e) : "memory");
+        }
+    }
+}
+
 /* Tally commit (a3) for a contiguous span [off, off + nbytes) of region r (offsets relative to
  * the replica base, inside my slice) whose stores by this CTA are complete.  Call from ONE thread
  * after a __syncthreads() that follows the stores.  Adds the bytes to every covered chunk's
@@ -251,8 +297,7 @@ __device__ __forceinline__ void commit_span(const launch_ctx &lc, int r, uint64_
         uint64_t end = (uint64_t)(c + 1) * R.chunk_bytes;
         if (end > R.own_bytes) end = R.own_bytes;
         uint32_t b = (uint32_t)((end - rel) < nbytes ? (end - rel) : nbytes);
-        uint32_t old = atom_add_release_gpu(&R.counter[c], b);
-        if (old + b > R.expected[c]) raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
+        commit_chunk(lc, r, c, b);
         rel += b;
         nbytes -= b;
     }

@@ -211,6 +211,7 @@ proact_config default_config() {
     c.watchdog_ms = 20000;
     c.grid_cap = 0;
     c.chunk_bytes = 128 * 1024;   // the paper's V100 profiler choice (Table II)
+    c.discovery = PROACT_DISCOVER_QUEUE;
     return c;
 }
 
@@ -221,6 +222,7 @@ void apply_env(proact_config &c) {
     c.piece_bytes = (uint32_t)env_int("PROACT_PIECE_BYTES", (int)c.piece_bytes);
     c.watchdog_ms = (uint32_t)env_int("PROACT_WATCHDOG_MS", (int)c.watchdog_ms);
     c.chunk_bytes = (uint32_t)env_int("PROACT_CHUNK_BYTES", (int)c.chunk_bytes);
+    c.discovery = env_int("PROACT_DISCOVERY", c.discovery);
     if (getenv("PROACT_ELIDE_PUSH") && atoi(getenv("PROACT_ELIDE_PUSH"))) c.mech = PROACT_MECH_ELIDE;
 }
 
@@ -229,7 +231,8 @@ int validate_config(const proact_config &c) {
     if (c.push != PROACT_PUSH_VEC16) return PROACT_ERR_INVALID;   // BULK push: not built yet
     if (c.agent_warps < 1 || c.agent_warps > 1024) return PROACT_ERR_INVALID;
     if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
-    if (c.piece_bytes < 512 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
+    if (c.piece_bytes < 4096 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
+    if (c.discovery != PROACT_DISCOVER_QUEUE && c.discovery != PROACT_DISCOVER_SCAN) return PROACT_ERR_INVALID;
     if (c.watchdog_ms < 1) return PROACT_ERR_INVALID;
     if (c.chunk_bytes < 4096 || c.chunk_bytes % 16) return PROACT_ERR_INVALID;
     return PROACT_OK;
@@ -318,11 +321,20 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
     // totals / global numbering need every rank's bytes: done by caller before (rank_off filled)
     size_t n_total = std::max<uint32_t>(R.n_total, 1);
     size_t deliv = c->debug ? n_own * (size_t)c->world : 0;
-    // layout: counter | expected | piecedone | changed | push | arrive[n_total] | count | deliv
-    size_t off_counter = 0, off_expected = off_counter + 4 * n_own, off_piece = off_expected + 4 * n_own,
-           off_changed = off_piece + 4 * n_own, off_push = off_changed + 4 * n_own,
-           off_arrive = off_push + 4 * n_own, off_count = off_arrive + 4 * n_total,
-           off_deliv = off_count + 64, total = off_deliv + 4 * deliv + 64;
+    // queue capacity: units with pieces >= 4096 B (validate_config) never exceed this
+    uint64_t qcap = 0;
+    for (uint32_t k = 0; k < R.n_own; ++k) {
+        uint64_t lo = (uint64_t)k * R.chunk, hi = std::min<uint64_t>(lo + R.chunk, R.own_bytes);
+        qcap += (hi - lo + 4095) / 4096;
+    }
+    qcap = std::max<uint64_t>(qcap, 1);
+    // layout: queue (8-aligned) | counter | expected | piecedone | changed | push | arrive[n_total]
+    //         | count | qctl[8] | deliv
+    size_t off_queue = 0, off_counter = off_queue + 8 * qcap, off_expected = off_counter + 4 * n_own,
+           off_piece = off_expected + 4 * n_own, off_changed = off_piece + 4 * n_own,
+           off_push = off_changed + 4 * n_own, off_arrive = off_push + 4 * n_own,
+           off_count = off_arrive + 4 * n_total, off_qctl = off_count + 64, off_deliv = off_qctl + 64,
+           total = off_deliv + 4 * deliv + 64;
     if (R.meta) { CK(cudaFree(R.meta)); R.meta = nullptr; }
     CK(cudaMalloc((void **)&R.meta, total));
     CK(cudaMemset(R.meta, 0, total));
@@ -352,6 +364,9 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
     D.arrive = (uint32_t *)(R.meta + off_arrive);
     D.arrive_count = (uint32_t *)(R.meta + off_count);
     D.deliv = deliv ? (uint32_t *)(R.meta + off_deliv) : nullptr;
+    D.queue = (unsigned long long *)(R.meta + off_queue);
+    D.qctl = (uint32_t *)(R.meta + off_qctl);
+    D.qcap = (uint32_t)qcap;
     D.chunk_dest = nullptr;
     R.chunk_dest.clear();
     if (R.d_chunk_dest) { CK(cudaFree(R.d_chunk_dest)); R.d_chunk_dest = nullptr; }
@@ -767,6 +782,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     lc.mech = (uint16_t)cfg.mech;
     lc.push = (uint16_t)cfg.push;
     lc.piece_bytes = cfg.piece_bytes;
+    lc.discovery = (uint16_t)cfg.discovery;
     uint32_t armed = 0;
     for (int i = 0; i < nregions; ++i) {
         int r = regions[i];
@@ -780,7 +796,11 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
         lc.gen_epoch[r] = (armed >> r & 1) ? c->epoch : R.gen_epoch;
     }
-    bool agent = (cfg.mech == PROACT_MECH_FUSED || cfg.mech == PROACT_MECH_ELIDE) && armed;
+    // a single rank has nothing to send or receive: no tracking is needed at all, the fused
+    // launch degenerates to the plain kernel (ELIDE keeps the agent: it measures tracking).
+    // (Not done for G > 1 even if my masks are empty: lc.mech also drives my consumer waits.)
+    if (cfg.mech == PROACT_MECH_FUSED && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
+    bool agent = (lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE) && armed;
     unsigned wpc = block / 32;
     unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
     lc.agent_ctas = (uint16_t)agent_ctas;

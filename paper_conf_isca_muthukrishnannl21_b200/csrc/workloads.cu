@@ -34,11 +34,7 @@ __device__ __forceinline__ void warp_commit(const launch_ctx &lc, int r, bool ha
     uint32_t key = single ? c : 0xFFFFFFFFu;
     uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
     if (single) {
-        if ((__ffs(grp) - 1) == (int)(threadIdx.x & 31)) {
-            uint32_t b = nb * __popc(grp);
-            uint32_t old = proact::atom_add_release_gpu(&R.counter[c], b);
-            if (old + b > R.expected[c]) proact::raise_error(lc.ctx, proact::SITE_COMMIT, PROACT_ERR_PROTOCOL);
-        }
+        if ((__ffs(grp) - 1) == (int)(threadIdx.x & 31)) proact::commit_chunk(lc, r, c, nb * __popc(grp));
     } else if (has) {
         proact::commit_span(lc, r, off, nb);
     }
@@ -70,99 +66,189 @@ __device__ __forceinline__ float ld_f(const float *p)
 }
 
 // ---------------------------------------------------------------- Jacobi
-constexpr int JB = 256;           // threads per CTA
-constexpr int JW = 4 * JB;        // strip width in columns (float4 per thread) = 4 KiB of a row
+// Tile = rows_per_tile rows x one 1024-column strip (4 KiB of a row).  Warp-specialised CTA:
+// one producer warp streams the tile's input rows (plus the two halo rows) into a JS-deep
+// shared-memory ring with 1D bulk async copies (cp.async.bulk = TMA engine, completion on a
+// per-slot "full" mbarrier); eight compute warps consume them (each thread: 4 columns, float4
+// up/cur/dn rolled in registers, horizontal neighbours by warp shuffle, warp-edge lanes from
+// shared memory) and release slots on per-slot "empty" mbarriers.  The row stream runs across
+// the CTA's tiles without draining.  Every input row is read from HBM once per tile (+2 halo
+// rows per tile, L2 hits); outputs are 16-byte stores.
+constexpr int JC = 8;                   // compute warps
+constexpr int JB = (JC + 1) * 32;       // + one producer warp
+constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
+constexpr int JS = 8;                   // ring depth (rows in flight per CTA)
+constexpr int SLOT = JW + 8;            // floats per slot: columns [c0-4, c0+JW+4)
+constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8;
 
-struct Row { float4 v; float l, r; };
-
-// Row k of the input as seen by this thread: 4 cells at column j and (warp-edge lanes) the
-// left/right scalars.  `local` rows (mine, written by my previous phase) use the read-only
-// path; halo rows pushed by a peer during this kernel use plain (coherent) loads.
-__device__ __forceinline__ Row load_row(const float *in, int64_t N, int64_t k, int64_t j, bool act,
-                                        bool local, uint32_t lane)
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt)
 {
-    Row o;
-    o.v = make_float4(0.f, 0.f, 0.f, 0.f);
-    o.l = 0.f;
-    o.r = 0.f;
-    if (k < 0 || k >= N || !act) return o;
-    const float *p = in + k * N + j;
-    if (local) {
-        o.v = ld_nc_f4(p);
-        if (lane == 0 && j > 0) o.l = ld_nc_f(p - 1);
-        if (lane == 31 && j + 4 < N) o.r = ld_nc_f(p + 4);
-    } else {
-        o.v = ld_f4(p);
-        if (lane == 0 && j > 0) o.l = ld_f(p - 1);
-        if (lane == 31 && j + 4 < N) o.r = ld_f(p + 4);
-    }
-    return o;
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b)
+{
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
+{
+    uint32_t done;
+    do {
+        asm volatile("{\n\t.reg .pred p;\n\t"
+                     "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                     "selp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes, uint64_t *bar)
+{
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(sdst)), "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ float4 lds128(const float *p) { return *reinterpret_cast<const float4 *>(p); }
+
+struct JTile {
+    int i0, i1, c0, c1, kfirst, klast;
+};
+
+// Tile t of this rank: interior bands first, the two halo-dependent edge bands last (a7).
+__device__ __forceinline__ JTile jtile(int t, int nstrips, int nbands, int rb, int row0, int rend, int N)
+{
+    const int bi = t / nstrips, strip = t - bi * nstrips;
+    int band;
+    if (nbands <= 2) band = bi;
+    else if (bi < nbands - 2) band = bi + 1;
+    else band = bi == nbands - 2 ? 0 : nbands - 1;
+    JTile T;
+    T.i0 = row0 + band * rb;
+    T.i1 = min(T.i0 + rb, rend);
+    T.c0 = strip * JW;
+    T.c1 = min(T.c0 + JW, N);
+    T.kfirst = T.i0 > 0 ? T.i0 - 1 : 0;
+    T.klast = T.i1 < N - 1 ? T.i1 : N - 1;
+    return T;
 }
 
-__global__ void __launch_bounds__(JB) jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
+// Producer warp (one lane): the CTA's row stream, slot by slot.
+__device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_jacobi_params &p, float *ring,
+                                           uint64_t *full, uint64_t *empty, int t_first, int P, int ntiles,
+                                           int nstrips, int nbands)
+{
+    const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows), rb = p.rows_per_tile;
+    const char *in = lc.ctx->region[p.region_in].base;
+    uint32_t q = 0;
+    for (int t = t_first; t < ntiles; t += P) {
+        const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+        const int lo = T.c0 >= 4 ? T.c0 - 4 : 0, hi = min(T.c0 + JW + 4, N);
+        const uint32_t bytes = (uint32_t)(hi - lo) * 4;
+        for (int k = T.kfirst; k <= T.klast; ++k, ++q) {
+            const uint32_t slot = q % JS;
+            if (q >= JS) mbar_wait(&empty[slot], ((q / JS) - 1) & 1u);
+            const uint64_t goff = ((uint64_t)k * N + lo) * 4;
+            if (k < row0 || k >= rend) {   // (a7) halo row produced by a peer: wait, then
+                proact::wait_range(lc, p.region_in, goff, bytes);
+                asm volatile("fence.proxy.async;" ::: "memory");   // generic -> async proxy
+            }
+            mbar_expect_tx(&full[slot], bytes);
+            bulk_g2s(ring + slot * SLOT + (lo - (T.c0 - 4)), in + goff, bytes, &full[slot]);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(JB, 4) jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 {
     if (proact::agent_dispatch(lc)) return;
-    const region_dev &Ri = lc.ctx->region[p.region_in];
-    const float *in = reinterpret_cast<const float *>(Ri.base);
-    const int64_t N = p.N, row0 = p.row0, rend = p.row0 + p.nrows;
+    extern __shared__ __align__(128) unsigned char jsm[];
+    float *ring = reinterpret_cast<float *>(jsm);
+    uint64_t *full = reinterpret_cast<uint64_t *>(jsm + (size_t)JS * SLOT * 4);
+    uint64_t *empty = full + JS;
+    const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows);
     const int rb = p.rows_per_tile;
-    const uint32_t lane = threadIdx.x & 31u;
-    const int64_t nstrips = (N + JW - 1) / JW;
-    const int64_t nbands = (p.nrows + rb - 1) / rb;
-    const int64_t ntiles = nbands * nstrips;
-    for (int64_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
-        // interior bands first, the two halo-dependent edge bands last (they wait on flags)
-        int64_t bi = t / nstrips, strip = t % nstrips, band;
-        if (nbands <= 2) band = bi;
-        else if (bi < nbands - 2) band = bi + 1;
-        else band = bi == nbands - 2 ? 0 : nbands - 1;
-        const int64_t i0 = row0 + band * rb, i1 = min(i0 + (int64_t)rb, rend);
-        const int64_t c0 = strip * JW, c1 = min(c0 + (int64_t)JW, N);
-        const bool top_halo = i0 == row0 && i0 > 0, bot_halo = i1 == rend && i1 < N;
-        if (top_halo || bot_halo) {   // (a7) wait for the neighbours' boundary rows of gen-1
-            if (threadIdx.x == 0) {
-                const int64_t a = c0 > 0 ? c0 - 1 : 0, b = c1 < N ? c1 + 1 : N;
-                if (top_halo) proact::wait_range(lc, p.region_in, (uint64_t)((i0 - 1) * N + a) * 4, (uint64_t)(b - a) * 4);
-                if (bot_halo) proact::wait_range(lc, p.region_in, (uint64_t)(i1 * N + a) * 4, (uint64_t)(b - a) * 4);
-            }
-            __syncthreads();
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int nstrips = (N + JW - 1) / JW;
+    const int nbands = ((int)p.nrows + rb - 1) / rb;
+    const int ntiles = nbands * nstrips;
+    const int P = (int)proact::producer_grid(lc);
+    const int t_first = (int)proact::producer_block(lc);
+    if (tid == 0) {
+        for (int s = 0; s < JS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], JC);
         }
-        const int64_t j = c0 + 4 * (int64_t)threadIdx.x;
-        const bool act = j < c1;
-        Row up = load_row(in, N, i0 - 1, j, act, i0 - 1 >= row0, lane);
-        Row cur = load_row(in, N, i0, j, act, true, lane);
-        Row dn = load_row(in, N, i0 + 1, j, act, i0 + 1 < rend, lane);
-        for (int64_t i = i0; i < i1; ++i) {
-            Row nx;
-            if (i + 2 <= i1) nx = load_row(in, N, i + 2, j, act, i + 2 < rend, lane);
-            // horizontal neighbours: lanes exchange, warp-edge lanes use their scalars
-            float lft = __shfl_up_sync(0xFFFFFFFFu, cur.v.w, 1);
-            float rgt = __shfl_down_sync(0xFFFFFFFFu, cur.v.x, 1);
-            if (lane == 0) lft = cur.l;
-            if (lane == 31) rgt = cur.r;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (warp == JC) {
+        if (lane == 0) jacobi_stream(lc, p, ring, full, empty, t_first, P, ntiles, nstrips, nbands);
+        return;
+    }
+    char *outb = lc.ctx->region[p.region_out].base;
+    uint32_t q = 0;   // next stream item (same sequence as the producer warp's)
+    for (int t = t_first; t < ntiles; t += P) {
+        const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+        const int x = 4 * tid, j = T.c0 + x;
+        const bool act = j < T.c1;
+        const float *ringf = ring + 4 + x;
+        float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur, dn = up;
+        if (T.i0 > 0) {   // top halo / previous row: registers only, release at once
+            mbar_wait(&full[q % JS], (q / JS) & 1u);
+            if (act) up = lds128(ringf + (q % JS) * SLOT);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[q % JS]);
+            ++q;
+        }
+        uint32_t qcur = q;
+        mbar_wait(&full[q % JS], (q / JS) & 1u);
+        cur = act ? lds128(ringf + (q % JS) * SLOT) : up;
+        ++q;
+        for (int i = T.i0; i < T.i1; ++i) {
+            const uint32_t qdn = q;
+            const bool has_dn = i + 1 <= T.klast;
+            if (has_dn) {
+                mbar_wait(&full[q % JS], (q / JS) & 1u);
+                if (act) dn = lds128(ringf + (q % JS) * SLOT);
+                ++q;
+            }
+            const float *cs = ringf + (qcur % JS) * SLOT;
+            float lft = __shfl_up_sync(0xFFFFFFFFu, cur.w, 1);
+            float rgt = __shfl_down_sync(0xFFFFFFFFu, cur.x, 1);
+            if (lane == 0) lft = cs[-1];
+            if (lane == 31) rgt = cs[4];
             if (act) {
                 float4 o;
                 if (i == 0 || i == N - 1) {
-                    o = cur.v;
+                    o = cur;
                 } else {
-                    o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.v.x, dn.v.x), __fadd_rn(lft, cur.v.y)));
-                    o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.v.y, dn.v.y), __fadd_rn(cur.v.x, cur.v.z)));
-                    o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.v.z, dn.v.z), __fadd_rn(cur.v.y, cur.v.w)));
-                    o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.v.w, dn.v.w), __fadd_rn(cur.v.z, rgt)));
-                    if (j == 0) o.x = cur.v.x;
-                    if (j + 3 == N - 1) o.w = cur.v.w;
+                    o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.x, dn.x), __fadd_rn(lft, cur.y)));
+                    o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.y, dn.y), __fadd_rn(cur.x, cur.z)));
+                    o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.z, dn.z), __fadd_rn(cur.y, cur.w)));
+                    o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.w, dn.w), __fadd_rn(cur.z, rgt)));
+                    if (j == 0) o.x = cur.x;
+                    if (j + 3 == N - 1) o.w = cur.w;
                 }
-                proact::put(lc, p.region_out, (uint64_t)(i * N + j) * 4, o);
+                const uint64_t off = ((uint64_t)i * N + j) * 4;
+                if (lc.mech == PROACT_MECH_INLINE) proact::put(lc, p.region_out, off, o);
+                else *reinterpret_cast<float4 *>(outb + off) = o;
+            }
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&empty[qcur % JS]);                    // row i: done
+                if (has_dn && i + 1 == T.i1) mbar_arrive(&empty[qdn % JS]);   // bottom halo row
             }
             up = cur;
             cur = dn;
-            dn = nx;
+            qcur = qdn;
         }
-        __syncthreads();
-        if (threadIdx.x < 32) {   // (a3) one span per row of the tile, merged per chunk
-            for (int64_t k0 = i0; k0 < i1; k0 += 32) {
-                const int64_t i = k0 + lane;
-                warp_commit(lc, p.region_out, i < i1, (uint64_t)(i * N + c0) * 4, (uint32_t)((c1 - c0) * 4));
+        // (a3) the tile's stores are complete in every compute warp -> commit, merged per chunk
+        asm volatile("bar.sync 1, %0;" ::"r"(JC * 32) : "memory");
+        if (warp == 0) {
+            for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
+                const int i = k0 + lane;
+                warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4, (uint32_t)(T.c1 - T.c0) * 4);
             }
         }
     }
@@ -250,7 +336,7 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
-    return proact_launch(regs, 1, (const void *)jacobi_kernel, 0, JB, args, 0, stream);
+    return proact_launch(regs, 1, (const void *)jacobi_kernel, 0, JB, args, JSMEM, stream);
 }
 
 int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int scattered, void *stream)

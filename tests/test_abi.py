@@ -62,6 +62,6 @@ def test_binding_fails_loudly_without_library(monkeypatch, tmp_path):
 
 
 def test_struct_layouts_match_header():
-    # proact_config: 8 x 4-byte fields; proact_region_info: see include/proact.h
-    assert ctypes.sizeof(_lib.Config) == 32
+    # proact_config: 10 x 4-byte fields; proact_region_info: see include/proact.h
+    assert ctypes.sizeof(_lib.Config) == 40
     assert ctypes.sizeof(_lib.RegionInfo) == 8 + 8 * 4 + 4 * 4 + 8 + 8 * (_lib.MAX_RANKS + 1)

@@ -55,11 +55,12 @@ def test_micro_replicas_equal_closed_form(G, words, chunk, mech, scattered, piec
             assert np.array_equal(outs[g][p], want), (p, g)
 
 
-def test_micro_exactly_once_and_counters():
+@pytest.mark.parametrize("disc", [_lib.DISCOVER_QUEUE, _lib.DISCOVER_SCAN])
+def test_micro_exactly_once_and_counters(disc):
     os.environ["PROACT_DEBUG"] = "1"
 
     def body(r, G):
-        rt.set_config(mech=_lib.MECH_FUSED, piece_bytes=8192, agent_warps=3)
+        rt.set_config(mech=_lib.MECH_FUSED, piece_bytes=8192, agent_warps=3, discovery=disc)
         M = wl.Micro(1 << 20, 65536)
         s = torch.cuda.Stream()
         out = []
