@@ -11,7 +11,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libproact.so")
+# PROACT_LIB: an alternative build of the same library (tools/ variant sweeps only)
+LIB_PATH = os.environ.get("PROACT_LIB") or os.path.join(_HERE, "libproact.so")
 
 MAX_RANKS = 16
 MAX_REGIONS = 8

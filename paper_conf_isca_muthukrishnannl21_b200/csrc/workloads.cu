@@ -77,7 +77,10 @@ __device__ __forceinline__ float ld_f(const float *p)
 constexpr int JC = 8;                   // compute warps
 constexpr int JB = (JC + 1) * 32;       // + one producer warp
 constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
-constexpr int JS = 8;                   // ring depth (rows in flight per CTA)
+#ifndef PROACT_JACOBI_RING
+#define PROACT_JACOBI_RING 16
+#endif
+constexpr int JS = PROACT_JACOBI_RING;  // ring depth (rows in flight per CTA)
 constexpr int SLOT = JW + 8;            // floats per slot: columns [c0-4, c0+JW+4)
 constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8;
 
@@ -336,6 +339,12 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
+    static bool attr = false;   // > 48 KiB of dynamic shared memory needs the opt-in
+    if (!attr) {
+        if (cudaFuncSetAttribute(jacobi_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) != cudaSuccess)
+            return PROACT_ERR_CUDA;
+        attr = true;
+    }
     return proact_launch(regs, 1, (const void *)jacobi_kernel, 0, JB, args, JSMEM, stream);
 }
 
