@@ -402,10 +402,8 @@ __device__ __forceinline__ uint32_t chunk_flag(const launch_ctx &lc, int r, uint
 } /* namespace proact */
 
 #ifdef __CUDACC__
+#include "proact_agent.cuh"
 namespace proact {
-/* The transfer agent (a4-a6); defined in csrc/agent.cuh, included by the library's kernels. */
-__device__ void agent_loop(const launch_ctx &lc);
-
 /* Agent CTAs (the first lc.agent_ctas blocks of a FUSED/ELIDE launch) run the polling agent and
  * return true; producer CTAs get false.  Call first thing in a producer kernel. */
 __device__ __forceinline__ bool agent_dispatch(const launch_ctx &lc)

@@ -59,6 +59,41 @@ int proact_jacobi_solve_host(const float *h_x0, float *h_out, long long N, int i
                              size_t chunk_bytes, int rows_per_tile, void *stream,
                              unsigned long long *bytes_h2d, unsigned long long *bytes_d2h);
 
+/* ---- graph workloads (Sec. IV-C L265 PageRank, L267 SSSP; configs 3-4) --------- */
+
+/* Destination partition of a graph for G ranks: bounds[0..G] (host array of G+1) receive vertex
+ * boundaries, multiples of `align` vertices (use chunk_bytes/4 so that every rank's slice of a
+ * replicated 4-byte vertex vector starts on a chunk boundary), chosen so that in-edge counts are
+ * as even as possible.  d_dst: device array of E destination ids.  Synchronises `stream`. */
+int proact_graph_partition(const uint32_t *d_dst, unsigned long long E, unsigned V, int G, unsigned align,
+                           unsigned *bounds, void *stream);
+
+/* Build this rank's in-edge CSC for destinations [v0, v1) from a device edge list (d_src,
+ * d_dst, optional d_w weights, E edges, V vertices; self loops allowed, duplicates kept) plus the
+ * global out-degree.  Library-owned device memory; returns a graph id >= 0 (NOMEM if 4 graphs
+ * exist).  The edge list may be freed afterwards.  Synchronises `stream`. */
+int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w,
+                       unsigned long long E, unsigned V, unsigned v0, unsigned v1, void *stream);
+int proact_graph_free(int graph);
+int proact_graph_info(int graph, unsigned long long *e_own, unsigned *v0, unsigned *nv);
+
+/* PageRank (readings R11/R12).  The replicated region holds contrib[u] = r[u]/out(u) (fp32, 0
+ * for dangling u) over all V vertices; its owned slice must be [4*v0, 4*v1).  init writes
+ * contrib^0 = fp32(1/V)/out(u) into the WHOLE local replica (identical on every rank).  A phase
+ * computes, for my vertices, r'[v] = (float)((1-d)/V + d * sum_{u->v} contrib[u]) with an fp64
+ * sum, keeps r' locally and writes contrib'[v] = r'[v]/out(v) into region_out.
+ * pagerank_ranks copies my r' (nv floats) to device memory d_out. */
+int proact_pagerank_init(int graph, int region, void *stream);
+int proact_pagerank_phase(int graph, int region_in, int region_out, double damping, void *stream);
+int proact_pagerank_ranks(int graph, float *d_out, void *stream);
+
+/* SSSP, synchronous Bellman-Ford round (reading R13): for my vertices
+ * d'[v] = min(d[v], min_{u->v, d[u] != INT32_MAX} d[u] + w), int32, relaxing only sources whose
+ * chunk changed in the previous round (all of them when first != 0).  Regions should be
+ * registered with PROACT_REGION_SPARSE and chunk_bytes a multiple of 4096.  A round that
+ * changes anything casts a proact::vote (read it with a BARRIER phase_sync + proact_last_vote). */
+int proact_sssp_phase(int graph, int region_in, int region_out, int first, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -96,6 +96,17 @@ def _declare(L):
         "proact_jacobi_solve_host": (i, [vp, vp, ctypes.c_longlong, i, sz, i, vp,
                                          ctypes.POINTER(ctypes.c_ulonglong),
                                          ctypes.POINTER(ctypes.c_ulonglong)]),
+        "proact_graph_partition": (i, [vp, ctypes.c_ulonglong, ctypes.c_uint, i, ctypes.c_uint,
+                                       ctypes.POINTER(ctypes.c_uint), vp]),
+        "proact_graph_build": (i, [vp, vp, vp, ctypes.c_ulonglong, ctypes.c_uint, ctypes.c_uint,
+                                   ctypes.c_uint, vp]),
+        "proact_graph_free": (i, [i]),
+        "proact_graph_info": (i, [i, ctypes.POINTER(ctypes.c_ulonglong), ctypes.POINTER(ctypes.c_uint),
+                                  ctypes.POINTER(ctypes.c_uint)]),
+        "proact_pagerank_init": (i, [i, i, vp]),
+        "proact_pagerank_phase": (i, [i, i, i, ctypes.c_double, vp]),
+        "proact_pagerank_ranks": (i, [i, vp, vp]),
+        "proact_sssp_phase": (i, [i, i, i, i, vp]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)

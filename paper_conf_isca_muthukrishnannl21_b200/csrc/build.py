@@ -14,9 +14,9 @@ PKG = os.path.dirname(HERE)
 ROOT = os.path.dirname(PKG)
 INC = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libproact.so")
-SOURCES = ["runtime.cu", "workloads.cu"]
-DEPS = SOURCES + ["agent.cuh"]
-HEADERS = ["proact.h", "proact_device.cuh", "proact_workloads.h"]
+SOURCES = ["runtime.cu", "workloads.cu", "graph.cu"]
+DEPS = SOURCES
+HEADERS = ["proact.h", "proact_device.cuh", "proact_agent.cuh", "proact_workloads.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC,-O2", "-Xptxas", "-v", "--expt-relaxed-constexpr"]

@@ -11,7 +11,6 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include "agent.cuh"
 #include "proact.h"
 #include "proact_device.cuh"
 #include "proact_workloads.h"

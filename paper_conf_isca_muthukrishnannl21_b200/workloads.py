@@ -120,3 +120,117 @@ class Micro:
         micro_phase(self.rid, self.phase, seed, K, scattered, stream)
         rt.phase_sync(stream, barrier=barrier)
         self.phase += 1
+
+
+# ------------------------------------------------------------------ graphs (configs 3-4)
+def _u32_dev(a) -> torch.Tensor:
+    """A host numpy uint32 / int32 array (or a CUDA tensor) as a contiguous CUDA int32 tensor."""
+    if isinstance(a, torch.Tensor):
+        t = a
+    else:
+        import numpy as np
+        t = torch.from_numpy(np.ascontiguousarray(a).view(np.int32))
+    return t.to(device="cuda", dtype=torch.int32).contiguous()
+
+
+class _Graph:
+    """Edge list -> this rank's destination partition + in-edge CSC (library-owned)."""
+
+    def __init__(self, V: int, src, dst, w, chunk_bytes: int, stream=None):
+        G, g = rt.world(), rt.rank()
+        self.V = V
+        s = _s(stream)
+        d_src, d_dst = _u32_dev(src), _u32_dev(dst)
+        d_w = _u32_dev(w) if w is not None else None
+        E = d_src.numel()
+        bounds = (ctypes.c_uint * (G + 1))()
+        check(rt.lib().proact_graph_partition(ctypes.c_void_p(d_dst.data_ptr()), E, V, G, chunk_bytes // 4,
+                                               bounds, s), "graph_partition")
+        self.bounds = list(bounds)
+        self.v0, self.v1 = self.bounds[g], self.bounds[g + 1]
+        self.gid = check(rt.lib().proact_graph_build(
+            ctypes.c_void_p(d_src.data_ptr()), ctypes.c_void_p(d_dst.data_ptr()),
+            ctypes.c_void_p(d_w.data_ptr() if d_w is not None else 0), E, V, self.v0, self.v1, s),
+            "graph_build")
+        e_own = ctypes.c_ulonglong(0)
+        check(rt.lib().proact_graph_info(self.gid, ctypes.byref(e_own), None, None), "graph_info")
+        self.e_own = e_own.value
+        self.E = E
+        del d_src, d_dst, d_w
+        torch.cuda.synchronize()
+
+    def free(self):
+        rt.lib().proact_graph_free(self.gid)
+
+
+class PageRank(_Graph):
+    """Destination-partitioned PageRank over a replicated contrib = r/out vector (config 3)."""
+
+    def __init__(self, V: int, src, dst, chunk_bytes: int, damping: float = 0.85, stream=None):
+        super().__init__(V, src, dst, None, chunk_bytes, stream)
+        self.d = damping
+        self.bufs = [torch.zeros(V, dtype=torch.float32, device="cuda") for _ in range(2)]
+        torch.cuda.synchronize()
+        self.rid = [rt.register_region(b, self.v0 * 4, (self.v1 - self.v0) * 4, chunk_bytes) for b in self.bufs]
+        check(rt.lib().proact_pagerank_init(self.gid, self.rid[0], _s(stream)), "pagerank_init")
+        self.k = 0
+
+    def step(self, stream=None, barrier: bool = False) -> None:
+        i = self.k & 1
+        check(rt.lib().proact_pagerank_phase(self.gid, self.rid[i], self.rid[i ^ 1], self.d, _s(stream)),
+              "pagerank_phase")
+        rt.phase_sync(stream, barrier=barrier)
+        self.k += 1
+
+    def ranks(self, stream=None) -> torch.Tensor:
+        out = torch.empty(self.v1 - self.v0, dtype=torch.float32, device="cuda")
+        check(rt.lib().proact_pagerank_ranks(self.gid, ctypes.c_void_p(out.data_ptr()), _s(stream)),
+              "pagerank_ranks")
+        return out
+
+
+INF32 = 2**31 - 1
+
+
+class SSSP(_Graph):
+    """Synchronous Bellman-Ford over a replicated int32 distance vector, SPARSE regions (config 4)."""
+
+    def __init__(self, V: int, src, dst, w, source: int, chunk_bytes: int, stream=None):
+        super().__init__(V, src, dst, w, chunk_bytes, stream)
+        self.bufs = []
+        for _ in range(2):
+            b = torch.full((V,), INF32, dtype=torch.int32, device="cuda")
+            b[source] = 0
+            self.bufs.append(b)
+        torch.cuda.synchronize()
+        self.rid = [rt.register_region(b, self.v0 * 4, (self.v1 - self.v0) * 4, chunk_bytes,
+                                       flags=_lib.REGION_SPARSE) for b in self.bufs]
+        self.k = 0
+
+    def step(self, stream=None) -> bool:
+        """One round with a BARRIER sync; returns True if any rank changed a distance."""
+        i = self.k & 1
+        check(rt.lib().proact_sssp_phase(self.gid, self.rid[i], self.rid[i ^ 1], int(self.k == 0), _s(stream)),
+              "sssp_phase")
+        rt.phase_sync(stream, barrier=True)
+        self.k += 1
+        if stream is None:
+            torch.cuda.current_stream().synchronize()
+        else:
+            stream.synchronize()
+        v = rt.last_vote()
+        if v < 0:
+            raise RuntimeError("vote not available")
+        return bool(v)
+
+    def run(self, max_rounds: int = 0, stream=None) -> int:
+        """Rounds until (and including) the first round that changes nothing (reading R13)."""
+        cap = max_rounds if max_rounds > 0 else self.V
+        for r in range(cap):
+            if not self.step(stream):
+                return r + 1
+        return cap
+
+    @property
+    def current(self) -> torch.Tensor:
+        return self.bufs[self.k & 1]
