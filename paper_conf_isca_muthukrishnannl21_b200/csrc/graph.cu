@@ -527,7 +527,9 @@ int proact_pagerank_phase(int graph, int region_in, int region_out, double dampi
 
 int proact_pagerank_ranks(int graph, float *d_out, void *stream)
 {
-    if (graph < 0 || graph >= MAXGRAPH || !graphs[graph].used || !d_out) return PROACT_ERR_INVALID;
+    if (graph < 0 || graph >= MAXGRAPH || !graphs[graph].used) return PROACT_ERR_INVALID;
+    if (graphs[graph].nv == 0) return PROACT_OK;   // empty slice: nothing to copy
+    if (!d_out) return PROACT_ERR_INVALID;
     GCK(cudaMemcpyAsync(d_out, graphs[graph].r_own, 4 * (size_t)graphs[graph].nv, cudaMemcpyDeviceToDevice,
                         (cudaStream_t)stream));
     return PROACT_OK;

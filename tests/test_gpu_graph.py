@@ -91,3 +91,29 @@ def test_sssp_disconnected_and_tiny():
     for rounds, d, _, _ in outs:
         assert rounds == want_rounds and np.array_equal(d, want)
         assert np.all(d[V // 2:] == oracle.INF)
+
+
+@pytest.mark.slow
+def test_config3_pagerank_full_size():
+    """BASELINE.json config 3 at full size (RMAT-24, ef16, 20 iterations), every vertex."""
+    src, dst = synth.rmat(24, 16)
+    V, iters = 1 << 24, 20
+    outs = run_ranks(1, _pr_body, V, src, dst, iters, 128 * 1024, _lib.MECH_FUSED)
+    want = oracle.pagerank(V, src, dst, iters).astype(np.float64)
+    (_, _, got), = outs
+    rel = np.abs(got.astype(np.float64) - want) / want
+    assert rel.max() <= 1e-5, rel.max()
+
+
+@pytest.mark.slow
+def test_config4_sssp_full_size():
+    """BASELINE.json config 4 at full size (RMAT-24, int32, to convergence), bit-exact."""
+    src, dst = synth.rmat(24, 16)
+    V = 1 << 24
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    outs = run_ranks(1, _sssp_body, V, src, dst, w, s0, 128 * 1024, _lib.MECH_FUSED)
+    want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
+    (rounds, d, _, _), = outs
+    assert rounds == want_rounds
+    assert np.array_equal(d, want)

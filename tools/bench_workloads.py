@@ -1,0 +1,191 @@
+#!/usr/bin/env python
+"""Secondary benchmarks (configs 3-5 of BASELINE.json) -- one JSON line per run.
+
+    python tools/bench_workloads.py --workload pagerank|sssp|micro [--scale 24] [--steps K]
+           [--warmup W] [--chunk BYTES] [--mech fused] [--ranks G] [--no-cpu]
+
+pagerank: step = 20 PageRank iterations on RMAT-scale (edge factor 16), value = iters/s.
+sssp:     step = Bellman-Ford to convergence (rounds as the oracle), value = rounds/s.
+micro:    step = one phase of the transfer microbenchmark (R bytes, all-gather shape) over
+          --ranks loopback ranks on this GPU; value = replicated bytes/s (HBM-to-HBM here:
+          with one GPU there is no NVLink, so this measures the protocol, not the link).
+Roofline: the phase kernel's algorithmic bytes per launch / CUDA-event time (DESIGN.md Sec.
+"Roofline accounting").  cpu_baseline: the oracle on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks  # noqa: E402
+from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt  # noqa: E402
+from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl  # noqa: E402
+
+
+def peak_hbm():
+    try:
+        return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+    except Exception:
+        return 6650.0
+
+
+def ev():
+    return torch.cuda.Event(enable_timing=True)
+
+
+def pagerank(args, src, dst, V):
+    def body(r, G):
+        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+        s = torch.cuda.Stream()
+        P = wl.PageRank(V, src, dst, args.chunk, stream=s)
+        I = 20
+
+        def step():
+            for k in range(I):
+                P.step(s, barrier=(k == I - 1))
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
+        e0, e1 = ev(), ev()
+        e0.record(s)
+        for _ in range(args.steps):
+            step()
+        e1.record(s)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        ks = []
+        for _ in range(10):
+            a, b = ev(), ev()
+            i = P.k & 1
+            a.record(s)
+            _lib.check(rt.lib().proact_pagerank_phase(P.gid, P.rid[i], P.rid[i ^ 1], P.d, wl._s(s)), "pr")
+            b.record(s)
+            rt.phase_sync(s)
+            P.k += 1
+            ks.append((a, b))
+        torch.cuda.synchronize()
+        kms = statistics.median(a.elapsed_time(b) for a, b in ks)
+        out = {"ms": ms, "kms": kms, "e_own": P.e_own, "nv": P.v1 - P.v0, "iters": args.steps * I}
+        P.free()
+        return out
+    res = run_ranks(args.ranks, body)
+    ms = max(r["ms"] for r in res)
+    kms = max(r["kms"] for r in res)
+    alg = max(8.0 * r["e_own"] + 16.0 * r["nv"] for r in res)
+    line = {"workload": f"pagerank_rmat{args.scale}_ef16_20it (BASELINE.json config 3)",
+            "value": res[0]["iters"] / (ms / 1000.0), "unit": "iters/s", "ranks": args.ranks,
+            "mech": args.mech, "chunk_bytes": args.chunk, "edges": int(src.size),
+            "roofline": {"bound": "hbm", "kernel": "pagerank_kernel", "kernel_ms": kms,
+                         "alg_bytes_per_launch": alg, "achieved": alg / kms / 1e6, "peak": peak_hbm(),
+                         "unit": "GB/s", "frac": alg / kms / 1e6 / peak_hbm(),
+                         "note": "8 B/edge (index + gathered contrib) + 16 B/vertex; gathers hit L2"}}
+    if not args.no_cpu:
+        import oracle
+        t0 = time.perf_counter()
+        oracle.pagerank(V, src, dst, 2)
+        t1 = time.perf_counter()
+        oracle.pagerank(V, src, dst, 4)
+        t2 = time.perf_counter()
+        per = max(1e-9, ((t2 - t1) - (t1 - t0)) / 2)
+        line["cpu_baseline"] = {"value": 1.0 / per, "unit": "iters/s", "cores": oracle.get_threads(),
+                                "kind": "oracle", "sample": "oracle.pagerank 4 vs 2 iterations (CSC build cancels)"}
+    return line
+
+
+def sssp(args, src, dst, V):
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+
+    def body(r, G):
+        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+        st = torch.cuda.Stream()
+        rounds = None
+        times = []
+        for k in range(args.warmup + args.steps):
+            S = wl.SSSP(V, src, dst, w, s0, args.chunk, stream=st)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            rounds = S.run(stream=st)
+            times.append(time.perf_counter() - t0)
+            S.free()
+        return {"rounds": rounds, "t": sum(times[args.warmup:])}
+    res = run_ranks(args.ranks, body)
+    t = max(r["t"] for r in res)
+    rounds = res[0]["rounds"]
+    line = {"workload": f"sssp_rmat{args.scale}_ef16 (BASELINE.json config 4)",
+            "value": args.steps * rounds / t, "unit": "rounds/s", "rounds": rounds, "ranks": args.ranks,
+            "mech": args.mech, "chunk_bytes": args.chunk, "edges": int(src.size),
+            "timing": "host wall clock per run (a BARRIER + host vote read every round)"}
+    if not args.no_cpu:
+        import oracle
+        t0 = time.perf_counter()
+        _, orounds, _ = oracle.sssp(V, src, dst, w, s0, max_rounds=3)
+        dt = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": orounds / dt, "unit": "rounds/s", "cores": 1, "kind": "oracle",
+                                "sample": "first 3 rounds of oracle.sssp (serial edge loop)"}
+    return line
+
+
+def micro(args):
+    R = args.bytes
+    W = R // 4
+
+    def body(r, G):
+        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+        M = wl.Micro(W, args.chunk)
+        s = torch.cuda.Stream()
+        for _ in range(args.warmup):
+            M.step(0x5EED, 1, False, stream=s, barrier=True)
+        torch.cuda.synchronize()
+        rt.host_barrier()
+        e0, e1 = ev(), ev()
+        e0.record(s)
+        for _ in range(args.steps):
+            M.step(0x5EED, 1, False, stream=s, barrier=True)
+        e1.record(s)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1)
+    ms = max(run_ranks(args.ranks, body))
+    G = args.ranks
+    repl = (G - 1) * R * args.steps   # bytes that cross "links" (to the G-1 other replicas)
+    return {"workload": f"micro R={R} chunk={args.chunk} loopback G={G}", "value": repl / (ms / 1000.0) / 1e9,
+            "unit": "GB/s replicated (HBM loopback)", "ms_per_phase": ms / args.steps, "mech": args.mech}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="pagerank", choices=["pagerank", "sssp", "micro"])
+    ap.add_argument("--scale", type=int, default=24)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=1)
+    ap.add_argument("--chunk", type=int, default=128 * 1024)
+    ap.add_argument("--mech", default="fused")
+    ap.add_argument("--ranks", type=int, default=1)
+    ap.add_argument("--bytes", type=int, default=256 << 20)
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.workload == "micro":
+        print(json.dumps(micro(args)), flush=True)
+        return
+    t0 = time.perf_counter()
+    src, dst = synth.rmat(args.scale, 16)
+    V = 1 << args.scale
+    gen_s = time.perf_counter() - t0
+    line = pagerank(args, src, dst, V) if args.workload == "pagerank" else sssp(args, src, dst, V)
+    line["rmat_gen_s"] = gen_s
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()
