@@ -177,16 +177,45 @@ struct SsspParams {
     int pad;
 };
 
-__device__ __forceinline__ float ld_nc_f(const float *p)
+// L2 policies: the CSC stream (read once per phase) is evict-first, the gathered vertex vector
+// (64 MiB at RMAT-24, fits the 126 MB L2) evict-last.
+__device__ __forceinline__ uint64_t pol_first()
 {
-    float v;
-    asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_last()
+{
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint32_t ld_stream_u(const uint32_t *p, uint64_t pol)
+{
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
-__device__ __forceinline__ int32_t ld_nc_i(const int32_t *p)
+__device__ __forceinline__ int32_t ld_stream_i(const int32_t *p, uint64_t pol)
 {
     int32_t v;
-    asm volatile("ld.global.nc.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+// The gathered vector: written by peers' agents during the previous phase (all arrived: the CTA
+// waited with wait_all before its first load, and nothing rewrites it this phase), so the
+// read-only path is coherent here.
+__device__ __forceinline__ float ld_gather_f(const float *p, uint64_t pol)
+{
+    float v;
+    asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ int32_t ld_gather_i(const int32_t *p, uint64_t pol)
+{
+    int32_t v;
+    asm volatile("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
 __device__ __forceinline__ uint32_t ld_nc_u(const uint32_t *p)
@@ -219,37 +248,67 @@ __device__ __forceinline__ double block_sum_f64(double x, double *red)
     return t;   // valid in thread 0
 }
 
-__global__ void __launch_bounds__(GB) pagerank_kernel(launch_ctx lc, PrParams p)
+// sum over edges [e0, e1) with stride `step` starting at `first`, 4 gathers in flight per lane
+__device__ __forceinline__ double pr_sum(const uint32_t *rowidx, const float *cin, uint32_t first, uint32_t e1,
+                                         uint32_t step, uint64_t pf, uint64_t pl)
+{
+    double s = 0.0;
+    uint32_t e = first;
+    for (; e + 3 * step < e1; e += 4 * step) {
+        const uint32_t u0 = ld_stream_u(rowidx + e, pf), u1 = ld_stream_u(rowidx + e + step, pf);
+        const uint32_t u2 = ld_stream_u(rowidx + e + 2 * step, pf), u3 = ld_stream_u(rowidx + e + 3 * step, pf);
+        const float c0 = ld_gather_f(cin + u0, pl), c1 = ld_gather_f(cin + u1, pl);
+        const float c2 = ld_gather_f(cin + u2, pl), c3 = ld_gather_f(cin + u3, pl);
+        s += (double)c0;
+        s += (double)c1;
+        s += (double)c2;
+        s += (double)c3;
+    }
+    for (; e < e1; e += step) s += (double)ld_gather_f(cin + ld_stream_u(rowidx + e, pf), pl);
+    return s;
+}
+
+// Light vertices of a tile are fetched dynamically by 8-lane groups (balances skewed degrees);
+// hubs are queued and reduced by the whole CTA afterwards.
+__global__ void __launch_bounds__(GB, 6) pagerank_kernel(launch_ctx lc, PrParams p)
 {
     if (proact::agent_dispatch(lc)) return;
     __shared__ uint32_t heavy[MAXHEAVY];
-    __shared__ uint32_t nheavy;
+    __shared__ uint32_t nheavy, next;
     __shared__ double red[GB / 32];
     const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
     const uint32_t ntiles = (p.g.nv + GT - 1) / GT;
-    const uint32_t grp = threadIdx.x / GL, sub = threadIdx.x % GL;
-    const uint32_t gmask = 0xFFu << ((threadIdx.x & 31) & ~(GL - 1));
+    const uint32_t sub = threadIdx.x % GL, lead = (threadIdx.x & 31) & ~(GL - 1);
+    const uint32_t gmask = 0xFFu << lead;
+    const uint64_t pf = pol_first(), pl = pol_last();
     bool waited = false;
     for (uint32_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
         if (!waited) {   // (a7) every chunk of the previous generation is in my replica
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
             waited = true;
         }
-        if (threadIdx.x == 0) nheavy = 0;
+        if (threadIdx.x == 0) {
+            nheavy = 0;
+            next = 0;
+        }
         __syncthreads();
         const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
-        for (uint32_t v = lo + grp; v < hi; v += GB / GL) {
+        for (;;) {
+            uint32_t k = 0;
+            if (sub == 0) k = atomicAdd(&next, 1u);
+            k = __shfl_sync(gmask, k, lead);
+            const uint32_t v = lo + k;
+            if (v >= hi) break;
             const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
             if (e1 - e0 > HEAVY) {
                 bool queued = false;
                 if (sub == 0) {
-                    const uint32_t k = atomicAdd(&nheavy, 1u);
-                    if (k < MAXHEAVY) { heavy[k] = v; queued = true; }
+                    const uint32_t h = atomicAdd(&nheavy, 1u);
+                    if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
                 }
-                if (__shfl_sync(gmask, queued, (threadIdx.x & 31) & ~(GL - 1))) continue;
+                if (__shfl_sync(gmask, queued, lead)) continue;
             }
-            double s = 0.0;
-            for (uint32_t e = e0 + sub; e < e1; e += GL) s += (double)ld_nc_f(cin + ld_nc_u(p.g.rowidx + e));
+            double s = pr_sum(p.g.rowidx, cin, e0 + sub, e1, GL, pf, pl);
             for (int o = GL / 2; o > 0; o >>= 1) s += __shfl_xor_sync(gmask, s, o);
             if (sub == 0) pr_finish(lc, p, v, s);
         }
@@ -258,8 +317,7 @@ __global__ void __launch_bounds__(GB) pagerank_kernel(launch_ctx lc, PrParams p)
         for (uint32_t h = 0; h < nh; ++h) {   // hubs: the whole CTA, fp64 tree reduction
             const uint32_t v = heavy[h];
             const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
-            double s = 0.0;
-            for (uint32_t e = e0 + threadIdx.x; e < e1; e += GB) s += (double)ld_nc_f(cin + ld_nc_u(p.g.rowidx + e));
+            double s = pr_sum(p.g.rowidx, cin, e0 + threadIdx.x, e1, GB, pf, pl);
             s = block_sum_f64(s, red);
             if (threadIdx.x == 0) pr_finish(lc, p, v, s);
         }
@@ -268,24 +326,34 @@ __global__ void __launch_bounds__(GB) pagerank_kernel(launch_ctx lc, PrParams p)
     }
 }
 
-// SSSP: is source chunk g (global id) "changed" in region r's current generation?
-__device__ __forceinline__ bool src_changed(const launch_ctx &lc, const region_dev &R, int r, uint32_t g)
+// relax edges [first, e1) stride `step` into best; sources filtered by the changed-chunk bitmap
+__device__ __forceinline__ int32_t sssp_relax(const SsspParams &p, const uint32_t *chg, uint32_t cshift,
+                                              uint32_t cdiv, const int32_t *din, uint32_t first, uint32_t e1,
+                                              uint32_t step, int32_t best, uint64_t pf, uint64_t pl)
 {
-    if (g >= R.chunk0 && g < R.chunk0 + R.n_own) return R.changed_gen[g - R.chunk0] == lc.gen[r];
-    if (!proact::uses_agent(lc)) return true;   // no per-chunk flags without the agent
-    return ld_nc_u(R.arrive + g) & 1u;
-}
-
-__device__ __forceinline__ int32_t sssp_relax(const launch_ctx &lc, const SsspParams &p, const region_dev &Ri,
-                                              const int32_t *din, uint32_t e, int32_t best)
-{
-    const uint32_t u = ld_nc_u(p.g.rowidx + e);
-    if (!p.first && !src_changed(lc, Ri, p.region_in, (uint32_t)(((uint64_t)u * 4) / Ri.chunk_bytes)))
-        return best;
-    const int32_t du = ld_nc_i(din + u);
-    if (du == INT32_MAX) return best;
-    const int64_t cand = (int64_t)du + (int64_t)ld_nc_i(p.g.w + e);
-    return cand < (int64_t)best ? (int32_t)cand : best;
+    for (uint32_t e = first; e < e1; e += 2 * step) {
+        const bool has1 = e + step < e1;
+        const uint32_t u0 = ld_stream_u(p.g.rowidx + e, pf);
+        const uint32_t u1 = has1 ? ld_stream_u(p.g.rowidx + e + step, pf) : 0u;
+        const uint32_t g0 = cdiv ? u0 / cdiv : u0 >> cshift, g1 = cdiv ? u1 / cdiv : u1 >> cshift;
+        const bool a0 = p.first || (chg[g0 >> 5] >> (g0 & 31) & 1u);
+        const bool a1 = has1 && (p.first || (chg[g1 >> 5] >> (g1 & 31) & 1u));
+        if (a0) {
+            const int32_t du = ld_gather_i(din + u0, pl);
+            if (du != INT32_MAX) {
+                const int64_t cand = (int64_t)du + (int64_t)ld_stream_i(p.g.w + e, pf);
+                if (cand < (int64_t)best) best = (int32_t)cand;
+            }
+        }
+        if (a1) {
+            const int32_t du = ld_gather_i(din + u1, pl);
+            if (du != INT32_MAX) {
+                const int64_t cand = (int64_t)du + (int64_t)ld_stream_i(p.g.w + e + step, pf);
+                if (cand < (int64_t)best) best = (int32_t)cand;
+            }
+        }
+    }
+    return best;
 }
 
 __device__ __forceinline__ int32_t block_min_i32(int32_t x, int32_t *red)
@@ -302,40 +370,69 @@ __device__ __forceinline__ int32_t block_min_i32(int32_t x, int32_t *red)
     return t;
 }
 
-__global__ void __launch_bounds__(GB) sssp_kernel(launch_ctx lc, SsspParams p)
+constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
+
+__global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p)
 {
     if (proact::agent_dispatch(lc)) return;
     __shared__ uint32_t heavy[MAXHEAVY];
-    __shared__ uint32_t nheavy;
+    __shared__ uint32_t nheavy, next;
     __shared__ int32_t red[GB / 32];
+    __shared__ uint32_t chg[CHG_WORDS];
     const region_dev &Ri = lc.ctx->region[p.region_in];
     const int32_t *din = reinterpret_cast<const int32_t *>(Ri.base);
     const uint32_t ntiles = (p.g.nv + GT - 1) / GT;
-    const uint32_t grp = threadIdx.x / GL, sub = threadIdx.x % GL;
-    const uint32_t gmask = 0xFFu << ((threadIdx.x & 31) & ~(GL - 1));
-    bool waited = false;
+    const uint32_t sub = threadIdx.x % GL, lead = (threadIdx.x & 31) & ~(GL - 1);
+    const uint32_t gmask = 0xFFu << lead;
+    const uint64_t pf = pol_first(), pl = pol_last();
+    // source vertex -> global chunk id: rank slices are chunk-aligned, so it is u*4/chunk_bytes
+    const uint32_t cv = Ri.chunk_bytes / 4;   // vertices per chunk
+    const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
+    bool ready = false;
     for (uint32_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
-        if (!waited) {
+        if (!ready) {   // (a7) wait for the previous generation, then snapshot its changed bits
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
-            waited = true;
+            __syncthreads();
+            const uint32_t gen = lc.gen[p.region_in];
+            const bool agent = proact::uses_agent(lc);
+            for (uint32_t wi = threadIdx.x; wi < CHG_WORDS && wi * 32 < Ri.n_total; wi += GB) {
+                uint32_t bits = 0;
+                for (uint32_t b = 0; b < 32; ++b) {
+                    const uint32_t g = wi * 32 + b;
+                    if (g >= Ri.n_total) break;
+                    bool c;
+                    if (g >= Ri.chunk0 && g < Ri.chunk0 + Ri.n_own) c = Ri.changed_gen[g - Ri.chunk0] == gen;
+                    else c = !agent || (ld_nc_u(Ri.arrive + g) & 1u);   // no flags without the agent
+                    bits |= (uint32_t)c << b;
+                }
+                chg[wi] = bits;
+            }
+            ready = true;
         }
-        if (threadIdx.x == 0) nheavy = 0;
+        if (threadIdx.x == 0) {
+            nheavy = 0;
+            next = 0;
+        }
         __syncthreads();
         const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
         bool changed = false;
-        for (uint32_t v = lo + grp; v < hi; v += GB / GL) {
+        for (;;) {
+            uint32_t k = 0;
+            if (sub == 0) k = atomicAdd(&next, 1u);
+            k = __shfl_sync(gmask, k, lead);
+            const uint32_t v = lo + k;
+            if (v >= hi) break;
             const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
             if (e1 - e0 > HEAVY) {
                 bool queued = false;
                 if (sub == 0) {
-                    const uint32_t k = atomicAdd(&nheavy, 1u);
-                    if (k < MAXHEAVY) { heavy[k] = v; queued = true; }
+                    const uint32_t h = atomicAdd(&nheavy, 1u);
+                    if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
                 }
-                if (__shfl_sync(gmask, queued, (threadIdx.x & 31) & ~(GL - 1))) continue;
+                if (__shfl_sync(gmask, queued, lead)) continue;
             }
             const int32_t old = din[v];
-            int32_t best = old;
-            for (uint32_t e = e0 + sub; e < e1; e += GL) best = sssp_relax(lc, p, Ri, din, e, best);
+            int32_t best = sssp_relax(p, chg, cshift, cdiv, din, e0 + sub, e1, GL, old, pf, pl);
             for (int o = GL / 2; o > 0; o >>= 1) best = min(best, __shfl_xor_sync(gmask, best, o));
             if (sub == 0) {
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
@@ -348,8 +445,7 @@ __global__ void __launch_bounds__(GB) sssp_kernel(launch_ctx lc, SsspParams p)
             const uint32_t v = heavy[h];
             const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
             const int32_t old = din[v];
-            int32_t best = INT32_MAX;
-            for (uint32_t e = e0 + threadIdx.x; e < e1; e += GB) best = sssp_relax(lc, p, Ri, din, e, best);
+            int32_t best = sssp_relax(p, chg, cshift, cdiv, din, e0 + threadIdx.x, e1, GB, INT32_MAX, pf, pl);
             best = min(block_min_i32(best, red), old);
             if (threadIdx.x == 0) {
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
@@ -545,7 +641,7 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     rc = proact_region_info_get(region_out, &ro);
     if (rc) return rc;
     if (ro.total_bytes != 4ull * p.g.V || ro.own_offset != 4ull * p.g.v0 || ro.own_bytes != 4ull * p.g.nv ||
-        ro.chunk_bytes % 4096)
+        ro.chunk_bytes % 4096 || ro.n_total_chunks > 32u * CHG_WORDS)
         return PROACT_ERR_INVALID;
     p.region_in = region_in;
     p.region_out = region_out;
