@@ -113,6 +113,19 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def max_over_ranks(ms: float, world: int) -> float:
+    """Max of a per-rank time over all ranks (the contract's whole-job time); works with the
+    nccl (CUDA tensor) and gloo (CPU tensor) backends."""
+    if world <= 1:
+        return float(ms)
+    import torch
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([float(ms)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def cpu_baseline(N: int, budget_s: float = 12.0) -> dict:
     """The oracle as it stands (oracle.jacobi_step, OpenMP over all host cores) on the full
     16384^2 grid, iterated until ~budget_s of CPU work (bounded sample)."""
@@ -178,6 +191,8 @@ def main():
     ap.add_argument("--n", type=int, default=N_GRID)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for the timing barrier / max-over-ranks only")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -195,9 +210,15 @@ def main():
     from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
     import synth
 
-    torch.cuda.set_device(local)
+    # PROACT_BENCH_SAME_DEVICE=1: every rank on GPU 0 (tests of the multi-process path on a
+    # one-GPU box; ranks then time-slice, so such numbers are not performance)
+    dev = 0 if os.environ.get("PROACT_BENCH_SAME_DEVICE") == "1" else local
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group("gloo")
         job = f"bench_{os.environ.get('MASTER_ADDR', '')}_{os.environ.get('MASTER_PORT', '')}"
     else:
         job = rt.new_job_key()
@@ -231,17 +252,13 @@ def main():
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        ms = e0.elapsed_time(e1)
-        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
-        if world > 1:
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return max_over_ranks(e0.elapsed_time(e1), world)
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     l0 = rt.launch_count()
-    with Clocks(local) as clk:
+    with Clocks(dev) as clk:
         ms = timed(step, args.steps)
     launches = rt.launch_count() - l0
     rt.check_device()

@@ -209,6 +209,15 @@ int proact_region_debug_deliveries(int region, uint32_t *out, size_t n);
  * host between phases without a peer's next phase overwriting them. */
 int proact_host_barrier(void);
 
+/* ---- host-only helpers (no CUDA; also used internally, exposed for tests) --------------- */
+/* Slice plan of a region: rank_off[0..world] (prefix sums of bytes[]) and rank_chunk0[0..world]
+ * (global id of each rank's first chunk; a rank's chunks are ceil(bytes/chunk_bytes)). */
+int proact_plan_slices(int world, const uint64_t *bytes, uint64_t chunk_bytes, uint64_t *rank_off,
+                       uint32_t *rank_chunk0);
+/* All-gather of n bytes (<= 4096) per rank through the job-keyed /dev/shm rendezvous that
+ * proact_init uses (COLLECTIVE over `world` callers with distinct ranks). */
+int proact_rdv_allgather(const char *job, int world, int rank, const void *mine, size_t n, void *all);
+
 /* Non-blocking check of the device error word. */
 int proact_check(void);
 /* Kernels launched by this rank so far (producer/agent grids, sync kernels, helper kernels). */

@@ -68,6 +68,9 @@ int proact_jacobi_solve_host(const float *h_x0, float *h_out, long long N, int i
 int proact_graph_partition(const uint32_t *d_dst, unsigned long long E, unsigned V, int G, unsigned align,
                            unsigned *bounds, void *stream);
 
+/* Host-only core of proact_graph_partition: bounds from an in-degree histogram (V entries). */
+int proact_partition_bounds(const uint32_t *indeg, unsigned V, int G, unsigned align, unsigned *bounds);
+
 /* Build this rank's in-edge CSC for destinations [v0, v1) from a device edge list (d_src,
  * d_dst, optional d_w weights, E edges, V vertices; self loops allowed, duplicates kept) plus the
  * global out-degree.  Library-owned device memory; returns a graph id >= 0 (NOMEM if 4 graphs

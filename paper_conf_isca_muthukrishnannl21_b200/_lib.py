@@ -88,6 +88,9 @@ def _declare(L):
         "proact_check": (i, []),
         "proact_host_barrier": (i, []),
         "proact_launch_count": (u64, []),
+        "proact_plan_slices": (i, [i, ctypes.POINTER(u64), u64, ctypes.POINTER(u64), ctypes.POINTER(u32)]),
+        "proact_rdv_allgather": (i, [cp, i, i, vp, sz, vp]),
+        "proact_partition_bounds": (i, [vp, ctypes.c_uint, i, ctypes.c_uint, ctypes.POINTER(ctypes.c_uint)]),
         "proact_epoch": (u32, []),
         "proact_autotune": (i, [cp, cp, RUN_FN, vp, ctypes.POINTER(Config)]),
         # workloads

@@ -509,16 +509,23 @@ int proact_graph_partition(const uint32_t *d_dst, unsigned long long E, unsigned
     GCK(cudaMemcpyAsync(h.data(), indeg, 4 * (size_t)V, cudaMemcpyDeviceToHost, s));
     GCK(cudaStreamSynchronize(s));
     GCK(cudaFree(indeg));
-    // bounds[g]: the align-multiple vertex closest to where the in-edge prefix reaches g*E/G
+    return proact_partition_bounds(h.data(), V, G, align, bounds);
+}
+
+int proact_partition_bounds(const uint32_t *indeg, unsigned V, int G, unsigned align, unsigned *bounds)
+{
+    if (!indeg || !bounds || G < 1 || align == 0) return PROACT_ERR_INVALID;
+    // bounds[g]: the align-multiple vertex whose in-edge prefix is closest to g*E/G (monotone)
     std::vector<uint64_t> cum((size_t)V + 1, 0);
-    for (uint32_t v = 0; v < V; ++v) cum[v + 1] = cum[v] + h[v];
+    for (uint32_t v = 0; v < V; ++v) cum[v + 1] = cum[v] + indeg[v];
+    auto dist = [&](uint64_t x, uint64_t t) { return cum[x] > t ? cum[x] - t : t - cum[x]; };
     bounds[0] = 0;
     for (int g = 1; g < G; ++g) {
         const uint64_t target = cum[V] * (uint64_t)g / (uint64_t)G;
-        uint32_t v = (uint32_t)(std::lower_bound(cum.begin(), cum.end(), target) - cum.begin());
-        uint64_t a = (uint64_t)v / align * align, b = std::min<uint64_t>(a + align, V);
-        uint32_t pick = (uint32_t)((target - cum[a] <= cum[b] - target) ? a : b);
-        bounds[g] = std::max<unsigned>(pick, bounds[g - 1]);
+        const uint64_t v = (uint64_t)(std::lower_bound(cum.begin(), cum.end(), target) - cum.begin());
+        const uint64_t a = v / align * align, b = std::min<uint64_t>(a + align, V);
+        const uint32_t pick = (uint32_t)(dist(a, target) <= dist(b, target) ? a : b);
+        bounds[g] = std::min<unsigned>(V, std::max<unsigned>(pick, bounds[g - 1]));
     }
     bounds[G] = V;
     return PROACT_OK;

@@ -622,11 +622,10 @@ int proact_register_region_ex(void *ptr, size_t bytes, size_t chunk_bytes, uint6
     R.dest_mask = dest_mask;
     R.flags = flags;
     R.own_bytes = bytes;
-    R.rank_off[0] = 0;
-    R.rank_chunk0[0] = 0;
-    for (int p = 0; p < c->world; ++p) {
-        R.rank_off[p + 1] = R.rank_off[p] + geos[p].bytes;
-        R.rank_chunk0[p + 1] = R.rank_chunk0[p] + ceil_div64(geos[p].bytes, chunk_bytes);
+    {
+        uint64_t bytes_of[MAXR];
+        for (int p = 0; p < c->world; ++p) bytes_of[p] = geos[p].bytes;
+        proact_plan_slices(c->world, bytes_of, chunk_bytes, R.rank_off, R.rank_chunk0);
     }
     R.own_off = R.rank_off[c->rank];
     R.total = R.rank_off[c->world];
@@ -680,9 +679,11 @@ int proact_region_rechunk(int id, size_t chunk_bytes)
     for (void *p : R.opened) cudaIpcCloseMemHandle(p);
     R.opened.clear();
     R.chunk = chunk_bytes;
-    R.rank_chunk0[0] = 0;
-    for (int p = 0; p < c->world; ++p)
-        R.rank_chunk0[p + 1] = R.rank_chunk0[p] + ceil_div64(R.rank_off[p + 1] - R.rank_off[p], chunk_bytes);
+    {
+        uint64_t bytes_of[MAXR];
+        for (int p = 0; p < c->world; ++p) bytes_of[p] = R.rank_off[p + 1] - R.rank_off[p];
+        proact_plan_slices(c->world, bytes_of, chunk_bytes, R.rank_off, R.rank_chunk0);
+    }
     R.n_total = R.rank_chunk0[c->world];
     R.chunk0 = R.rank_chunk0[c->rank];
     RegionExchange ex;
@@ -928,6 +929,31 @@ int proact_finalize(void)
     delete c;
     if (rc) return rc;
     return rc2;   // a device error latched earlier was already reported by the call that saw it
+}
+
+int proact_plan_slices(int world, const uint64_t *bytes, uint64_t chunk_bytes, uint64_t *rank_off,
+                       uint32_t *rank_chunk0)
+{
+    if (world < 1 || world > MAXR || !bytes || !rank_off || !rank_chunk0 || chunk_bytes == 0) return PROACT_ERR_INVALID;
+    rank_off[0] = 0;
+    rank_chunk0[0] = 0;
+    for (int p = 0; p < world; ++p) {
+        rank_off[p + 1] = rank_off[p] + bytes[p];
+        rank_chunk0[p + 1] = rank_chunk0[p] + ceil_div64(bytes[p], chunk_bytes);
+    }
+    return PROACT_OK;
+}
+
+int proact_rdv_allgather(const char *job, int world, int rank, const void *mine, size_t n, void *all)
+{
+    if (!job || world < 1 || world > MAXR || rank < 0 || rank >= world || !mine || !all) return PROACT_ERR_INVALID;
+    Shm shm;
+    int rc = shm.open(job, world);
+    if (rc) return rc;
+    rc = shm.allgather(rank, mine, n, all);
+    int rc2 = shm.barrier();
+    shm.close(true);
+    return rc ? rc : rc2;
 }
 
 int proact_host_barrier(void)

@@ -1,0 +1,84 @@
+"""Runtime pieces beyond the kernels: the profiler (a9) and bench.py's multi-process path."""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks
+from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_autotune_sweeps_caches_and_keeps_results_correct(tmp_path, monkeypatch):
+    """proact_autotune (Sec. III-A): brute force over mechanism x chunk x
+    agent warps, max-over-ranks time, JSON cache keyed by workload; results stay bit-exact for
+    every point (the callback checks them)."""
+    cache = tmp_path / "tune.json"
+    monkeypatch.setenv("PROACT_TUNE_CACHE", str(cache))
+    W = 1 << 20
+    seen = []
+
+    def body(r, G):
+        M = wl.Micro(W, 65536)
+        s = torch.cuda.Stream()
+
+        def run(cfg):
+            if cfg["chunk_bytes"] != rt.region_info(M.rid).chunk_bytes:
+                rt.rechunk(M.rid, cfg["chunk_bytes"])
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            for _ in range(3):
+                M.step(0x5EED, 1, False, stream=s, barrier=True)
+            b.record(s)
+            s.synchronize()
+            rt.host_barrier()
+            want = oracle.micro_phase(W, M.phase - 1, 0x5EED, 1)
+            assert np.array_equal(M.buf.cpu().numpy().view(np.uint32), want)
+            rt.host_barrier()
+            if r == 0:
+                seen.append(dict(cfg))
+            return a.elapsed_time(b)
+
+        best = rt.autotune("micro_1M_G2", run, "mech=0,1;warps=4,16;chunk=65536,262144")
+        again = rt.autotune("micro_1M_G2", run, None)   # cached: no new runs
+        return best, again
+
+    n_before = len(seen)
+    outs = run_ranks(2, body)
+    (best0, again0), (best1, _) = outs
+    assert best0 == best1 and again0["mech"] == best0["mech"]
+    assert best0["mech"] in (_lib.MECH_FUSED, _lib.MECH_INLINE)
+    assert best0["chunk_bytes"] in (65536, 262144)
+    # FUSED: 2 chunks x 2 warps points; INLINE: 2 chunks (warps ignored) -> 6 runs, cache hit after
+    assert len(seen) - n_before == 6
+    d = json.loads(cache.read_text())
+    assert "micro_1M_G2" in d and d["micro_1M_G2"]["chunk_bytes"] == best0["chunk_bytes"]
+
+
+@pytest.mark.slow
+def test_bench_two_processes_json_line():
+    """bench.py --gpus 2 under torchrun (both ranks on this one GPU: CUDA IPC, time-sliced)."""
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ, PROACT_BENCH_SAME_DEVICE="1", PROACT_WATCHDOG_MS="120000")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "1", "--warmup", "3", "--n", "1024", "--iters", "4", "--backend", "gloo",
+           "--no-cpu", "--no-e2e"]
+    r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout + r.stderr
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "strong"
