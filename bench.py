@@ -188,7 +188,7 @@ def main():
     ap.add_argument("--warps", type=int, default=0)
     ap.add_argument("--rpt", type=int, default=16)
     ap.add_argument("--iters", type=int, default=ITERS)
-    ap.add_argument("--n", type=int, default=N_GRID)
+    ap.add_argument("--grid-n", dest="n", type=int, default=N_GRID)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],

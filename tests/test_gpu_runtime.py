@@ -74,7 +74,7 @@ def test_bench_two_processes_json_line():
     env = dict(os.environ, PROACT_BENCH_SAME_DEVICE="1", PROACT_WATCHDOG_MS="120000")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
-           "--gpus", "2", "--steps", "1", "--warmup", "3", "--n", "1024", "--iters", "4", "--backend", "gloo",
+           "--gpus", "2", "--steps", "1", "--warmup", "3", "--grid-n", "1024", "--iters", "4", "--backend", "gloo",
            "--no-cpu", "--no-e2e"]
     r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout + r.stderr
