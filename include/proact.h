@@ -38,6 +38,7 @@ extern "C" {
 #endif
 
 #define PROACT_MAX_RANKS 16
+#define PROACT_BULK_SMEM (32 * 1024)   /* min dynamic smem of a launch with TMA pushes */
 #define PROACT_MAX_REGIONS 8
 
 /* ---- status codes ------------------------------------------------------------------------ */
@@ -69,7 +70,9 @@ enum {
 /* ---- agent push instruction (a5) -------------------------------------------------------- */
 enum {
     PROACT_PUSH_VEC16 = 0,   /* 16-byte ld.global.cg / st.global.v4, 512 B per warp instruction */
-    PROACT_PUSH_BULK = 1     /* cp.async.bulk (TMA) global->smem->peer global, one lane issues */
+    PROACT_PUSH_BULK = 1     /* cp.async.bulk (TMA): global->smem stage, then one smem->global bulk
+                                store per destination; one agent warp per CTA (lane 0 issues),
+                                the CTA's dynamic shared memory is its staging ring */
 };
 
 /* ---- agent discovery of completed chunks (a4) ------------------------------------------- */
@@ -78,6 +81,16 @@ enum {
                                   pop them in completion order (O(1) per chunk, no scanning) */
     PROACT_DISCOVER_SCAN = 1   /* agent warps poll the readiness counters of statically owned
                                   32-unit windows and claim ready ones with a warp ballot */
+};
+
+/* ---- where the transfer agent runs ----------------------------------------------------- */
+enum {
+    PROACT_AGENT_FUSED = 0,    /* leading CTAs of the producer's own grid (cooperative launch on a
+                                  dedicated GPU: co-residency guaranteed); shares its registers */
+    PROACT_AGENT_SEPARATE = 1  /* its own small kernel, launched first on a high-priority stream
+                                  (the paper's "independently launched long-lived kernel", L137),
+                                  with its own registers and a 128 KiB TMA staging ring; the
+                                  producer grid leaves room for it */
 };
 
 /* ---- phase synchronisation modes (a8) ----------------------------------------------------- */
@@ -104,7 +117,7 @@ typedef struct proact_config {
     int32_t grid_cap;      /* 0 = fill the device share; else max CTAs of a fused launch */
     uint32_t chunk_bytes;  /* preferred chunk size for workload drivers (profiler axis) */
     int32_t discovery;     /* PROACT_DISCOVER_*: how agents find completed chunks (a4) */
-    int32_t reserved;
+    int32_t agent_kernel;  /* PROACT_AGENT_*: where the agent warps run */
 } proact_config;
 
 /* Geometry of a registered region as seen by the calling rank. */

@@ -25,6 +25,7 @@ MECH_NAMES = {MECH_FUSED: "fused", MECH_INLINE: "inline", MECH_BULK: "bulk",
               MECH_LOCAL: "local", MECH_ELIDE: "elide"}
 PUSH_VEC16, PUSH_BULK = 0, 1
 DISCOVER_QUEUE, DISCOVER_SCAN = 0, 1
+AGENT_FUSED, AGENT_SEPARATE = 0, 1
 SYNC_SIGNAL, SYNC_BARRIER = 0, 1
 REGION_SPARSE = 1
 
@@ -41,7 +42,7 @@ class Config(ctypes.Structure):
                 ("agent_warps", ctypes.c_int32), ("block", ctypes.c_int32),
                 ("piece_bytes", ctypes.c_uint32), ("watchdog_ms", ctypes.c_uint32),
                 ("grid_cap", ctypes.c_int32), ("chunk_bytes", ctypes.c_uint32),
-                ("discovery", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("discovery", ctypes.c_int32), ("agent_kernel", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

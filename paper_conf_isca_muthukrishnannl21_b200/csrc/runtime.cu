@@ -181,6 +181,8 @@ struct RankCtx {
     uint64_t launches = 0;
     int last_cuda = 0;
     int latched = 0;
+    cudaStream_t side = nullptr;      // high-priority stream of the SEPARATE agent kernel
+    cudaEvent_t ev_start = nullptr, ev_done = nullptr;
 };
 
 thread_local RankCtx *tl = nullptr;
@@ -212,6 +214,7 @@ proact_config default_config() {
     c.grid_cap = 0;
     c.chunk_bytes = 128 * 1024;   // the paper's V100 profiler choice (Table II)
     c.discovery = PROACT_DISCOVER_QUEUE;
+    c.agent_kernel = PROACT_AGENT_FUSED;
     return c;
 }
 
@@ -223,16 +226,18 @@ void apply_env(proact_config &c) {
     c.watchdog_ms = (uint32_t)env_int("PROACT_WATCHDOG_MS", (int)c.watchdog_ms);
     c.chunk_bytes = (uint32_t)env_int("PROACT_CHUNK_BYTES", (int)c.chunk_bytes);
     c.discovery = env_int("PROACT_DISCOVERY", c.discovery);
+    c.agent_kernel = env_int("PROACT_AGENT_KERNEL", c.agent_kernel);
     if (getenv("PROACT_ELIDE_PUSH") && atoi(getenv("PROACT_ELIDE_PUSH"))) c.mech = PROACT_MECH_ELIDE;
 }
 
 int validate_config(const proact_config &c) {
     if (c.mech < 0 || c.mech > PROACT_MECH_ELIDE) return PROACT_ERR_INVALID;
-    if (c.push != PROACT_PUSH_VEC16) return PROACT_ERR_INVALID;   // BULK push: not built yet
+    if (c.push != PROACT_PUSH_VEC16 && c.push != PROACT_PUSH_BULK) return PROACT_ERR_INVALID;
     if (c.agent_warps < 1 || c.agent_warps > 1024) return PROACT_ERR_INVALID;
     if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
     if (c.piece_bytes < 4096 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
     if (c.discovery != PROACT_DISCOVER_QUEUE && c.discovery != PROACT_DISCOVER_SCAN) return PROACT_ERR_INVALID;
+    if (c.agent_kernel != PROACT_AGENT_FUSED && c.agent_kernel != PROACT_AGENT_SEPARATE) return PROACT_ERR_INVALID;
     if (c.watchdog_ms < 1) return PROACT_ERR_INVALID;
     if (c.chunk_bytes < 4096 || c.chunk_bytes % 16) return PROACT_ERR_INVALID;
     return PROACT_OK;
@@ -461,6 +466,10 @@ __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t ma
     }
 }
 
+// PROACT_AGENT_SEPARATE: the transfer agent as its own kernel (own registers, TMA staging ring)
+constexpr size_t AGENT_SMEM = 128 * 1024 + 256;
+__global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc) { proact::agent_loop(lc); }
+
 RankCtx *need_ctx() { return tl; }
 
 }  // namespace
@@ -555,6 +564,16 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     }
     rc = upload_ctx(c);
     if (rc) return fail(rc);
+    {
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        if (cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        if (cudaEventCreateWithFlags(&c->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        if (cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM) !=
+            cudaSuccess)
+            return fail(PROACT_ERR_CUDA);
+    }
     rc = c->shm.barrier();
     if (rc) return fail(rc);
     return PROACT_OK;
@@ -802,24 +821,50 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     // (Not done for G > 1 even if my masks are empty: lc.mech also drives my consumer waits.)
     if (cfg.mech == PROACT_MECH_FUSED && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
     bool agent = (lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE) && armed;
-    unsigned wpc = block / 32;
+    const bool separate = agent && cfg.agent_kernel == PROACT_AGENT_SEPARATE;
+    // VEC16: agent_warps warps packed into CTAs; BULK (TMA): one agent warp per CTA, which
+    // uses the CTA's whole dynamic shared memory as its staging ring (>= PROACT_BULK_SMEM)
+    const unsigned agent_block = separate ? 256u : block;
+    unsigned wpc = cfg.push == PROACT_PUSH_BULK ? 1 : agent_block / 32;
     unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
-    lc.agent_ctas = (uint16_t)agent_ctas;
+    if (agent && !separate && cfg.push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
     lc.agent_warps = (uint16_t)(agent ? cfg.agent_warps : 0);
     int nb = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
     if (nb < 1) return PROACT_ERR_INVALID;
     unsigned cap = (unsigned)std::max(1, nb * c->nsm / std::max(1, c->ranks_on_device));
     if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
-    unsigned total = agent_ctas + (grid ? grid : cap);
-    if (total > cap) total = cap;
-    if (total <= agent_ctas) return PROACT_ERR_INVALID;
-    *(launch_ctx *)args[0] = lc;
     cudaStream_t s = (cudaStream_t)stream;
-    if (c->coop && agent)
-        CK(cudaLaunchCooperativeKernel(kernel, dim3(total), dim3(block), args, smem, s));
-    else
+    if (separate) {
+        // the agent kernel first, on its own high-priority stream (ordered after my earlier
+        // work), so its CTAs are resident before the producer grid fills the device; the
+        // producer grid leaves one slot per agent CTA; my stream waits for the agent.
+        launch_ctx la = lc;
+        la.agent_ctas = (uint16_t)agent_ctas;
+        const size_t asmem = cfg.push == PROACT_PUSH_BULK ? AGENT_SMEM : 0;
+        CK(cudaEventRecord(c->ev_start, s));
+        CK(cudaStreamWaitEvent(c->side, c->ev_start, 0));
+        agent_kernel<<<agent_ctas, agent_block, asmem, c->side>>>(la);
+        CK(cudaGetLastError());
+        CK(cudaEventRecord(c->ev_done, c->side));
+        c->launches++;
+        lc.agent_ctas = 0;
+        unsigned total = grid ? grid : cap;
+        if (total + agent_ctas > cap) total = cap > agent_ctas ? cap - agent_ctas : 1;
+        *(launch_ctx *)args[0] = lc;
         CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+        CK(cudaStreamWaitEvent(s, c->ev_done, 0));
+    } else {
+        lc.agent_ctas = (uint16_t)agent_ctas;
+        unsigned total = agent_ctas + (grid ? grid : cap);
+        if (total > cap) total = cap;
+        if (total <= agent_ctas) return PROACT_ERR_INVALID;
+        *(launch_ctx *)args[0] = lc;
+        if (c->coop && agent)
+            CK(cudaLaunchCooperativeKernel(kernel, dim3(total), dim3(block), args, smem, s));
+        else
+            CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+    }
     for (int r = 0; r < c->nregions; ++r) {
         if (!(armed >> r & 1)) continue;
         Region &R = c->regions[r];
@@ -924,6 +969,9 @@ int proact_finalize(void)
     cudaFree(c->d);
     cudaFree(c->meta);
     cudaFreeHost(c->h_err);
+    if (c->side) cudaStreamDestroy(c->side);
+    if (c->ev_start) cudaEventDestroy(c->ev_start);
+    if (c->ev_done) cudaEventDestroy(c->ev_done);
     c->shm.close(true);
     tl = nullptr;
     delete c;

@@ -21,8 +21,8 @@ from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
 pytestmark = pytest.mark.gpu
 
 
-def _run_jacobi(r, G, N, iters, chunk, mech, halo_only=False, rpt=16, check_deliv=False):
-    rt.set_config(mech=mech, watchdog_ms=20000)
+def _run_jacobi(r, G, N, iters, chunk, mech, halo_only=False, rpt=16, check_deliv=False, **cfg):
+    rt.set_config(mech=mech, watchdog_ms=20000, **cfg)
     x0 = torch.from_numpy(synth.jacobi_init(N)).cuda()
     J = wl.Jacobi(N, chunk, x0=x0, halo_only=halo_only, rows_per_tile=rpt)
     s = torch.cuda.Stream()
@@ -57,6 +57,16 @@ def test_jacobi_ragged_ranks_chunks_tiles(G, N, chunk, rpt):
     outs = run_ranks(G, _run_jacobi, N, iters, chunk, _lib.MECH_FUSED, rpt=rpt)
     for g, (rep, _, _) in enumerate(outs):
         assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), f"rank {g}"
+
+
+@pytest.mark.parametrize("cfg", [dict(push=1), dict(agent_kernel=1), dict(push=1, agent_kernel=1),
+                                 dict(discovery=1, agent_warps=5)])
+def test_config1_jacobi_agent_variants(cfg):
+    N, iters = 1024, 10
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(2, _run_jacobi, N, iters, 64 * 1024, _lib.MECH_FUSED, **cfg)
+    for g, (rep, _, _) in enumerate(outs):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), (g, cfg)
 
 
 def test_jacobi_halo_only_owned_rows_and_halos():

@@ -19,8 +19,8 @@ pytestmark = pytest.mark.gpu
 SEED = 0x5EED
 
 
-def _run_micro(r, G, words, chunk, mech, phases, K, scattered, piece=None, warps=None):
-    kw = dict(mech=mech)
+def _run_micro(r, G, words, chunk, mech, phases, K, scattered, piece=None, warps=None, push=0, akern=0):
+    kw = dict(mech=mech, push=push, agent_kernel=akern)
     if piece:
         kw["piece_bytes"] = piece
     if warps:
@@ -51,6 +51,19 @@ def test_micro_replicas_equal_closed_form(G, words, chunk, mech, scattered, piec
     outs = run_ranks(G, _run_micro, words, chunk, mech, phases, K, scattered, piece=piece)
     for p in range(phases):
         want = oracle.micro_phase(words, p, SEED, K)
+        for g in range(G):
+            assert np.array_equal(outs[g][p], want), (p, g)
+
+
+@pytest.mark.parametrize("push,akern", [(0, 0), (1, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("G,words,chunk", [(2, (1 << 21) + 4 * 5, 1 << 20), (3, 1 << 20, 16384)])
+def test_micro_push_modes_and_agent_kernels(G, words, chunk, push, akern):
+    """TMA bulk pushes and the separate agent kernel give the same bytes as the SIMT/fused path."""
+    phases = 3
+    outs = run_ranks(G, _run_micro, words, chunk, _lib.MECH_FUSED, phases, 1, False, piece=65536, warps=4,
+                     push=push, akern=akern)
+    for p in range(phases):
+        want = oracle.micro_phase(words, p, SEED, 1)
         for g in range(G):
             assert np.array_equal(outs[g][p], want), (p, g)
 
