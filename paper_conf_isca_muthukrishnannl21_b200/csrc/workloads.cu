@@ -74,14 +74,14 @@ __device__ __forceinline__ float ld_f(const float *p)
 // the CTA's tiles without draining.  Every input row is read from HBM once per tile (+2 halo
 // rows per tile, L2 hits); outputs are 16-byte stores.
 constexpr int JC = 8;                   // compute warps
-constexpr int JB = (JC + 1) * 32;       // + one producer warp
+constexpr int JB = (JC + 2) * 32;       // + one producer (TMA) warp + one committer warp
 constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
 #ifndef PROACT_JACOBI_RING
 #define PROACT_JACOBI_RING 16
 #endif
 constexpr int JS = PROACT_JACOBI_RING;  // ring depth (rows in flight per CTA)
 constexpr int SLOT = JW + 8;            // floats per slot: columns [c0-4, c0+JW+4)
-constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8;
+constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8 + 4 * 8;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt)
@@ -161,13 +161,16 @@ __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_ja
     }
 }
 
-__global__ void __launch_bounds__(JB, 4) jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
+__global__ void __launch_bounds__(JB, 3) jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 {
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ __align__(128) unsigned char jsm[];
     float *ring = reinterpret_cast<float *>(jsm);
     uint64_t *full = reinterpret_cast<uint64_t *>(jsm + (size_t)JS * SLOT * 4);
     uint64_t *empty = full + JS;
+    uint64_t *tdone = empty + JS;    // [2] compute warps finished tile k (k & 1)
+    uint64_t *cdone = tdone + 2;     // [2] committer finished tile k (k & 1)
+    const bool tally = proact::uses_agent(lc);
     const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows);
     const int rb = p.rows_per_tile;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -181,6 +184,10 @@ __global__ void __launch_bounds__(JB, 4) jacobi_kernel(launch_ctx lc, proact_jac
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], JC);
         }
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(&tdone[s], JC);
+            mbar_init(&cdone[s], 1);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -188,8 +195,27 @@ __global__ void __launch_bounds__(JB, 4) jacobi_kernel(launch_ctx lc, proact_jac
         if (lane == 0) jacobi_stream(lc, p, ring, full, empty, t_first, P, ntiles, nstrips, nbands);
         return;
     }
+    if (warp == JC + 1) {
+        // (a3) committer warp: after the compute warps' mbarrier arrival for tile k (release ->
+        // acquire at CTA scope), commit the tile's rows with release RMWs, merged per chunk.
+        // The compute warps never stall on the commit's fence latency.
+        if (!tally) return;
+        uint32_t k = 0;
+        for (int t = t_first; t < ntiles; t += P, ++k) {
+            const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+            mbar_wait(&tdone[k & 1u], (k >> 1) & 1u);
+            for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
+                const int i = k0 + lane;
+                warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4, (uint32_t)(T.c1 - T.c0) * 4);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&cdone[k & 1u]);
+        }
+        return;
+    }
     char *outb = lc.ctx->region[p.region_out].base;
-    uint32_t q = 0;   // next stream item (same sequence as the producer warp's)
+    uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
+    uint32_t kt = 0;   // tiles handed to the committer
     for (int t = t_first; t < ntiles; t += P) {
         const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
         const int x = 4 * tid, j = T.c0 + x;
@@ -245,13 +271,11 @@ __global__ void __launch_bounds__(JB, 4) jacobi_kernel(launch_ctx lc, proact_jac
             cur = dn;
             qcur = qdn;
         }
-        // (a3) the tile's stores are complete in every compute warp -> commit, merged per chunk
-        asm volatile("bar.sync 1, %0;" ::"r"(JC * 32) : "memory");
-        if (warp == 0) {
-            for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
-                const int i = k0 + lane;
-                warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4, (uint32_t)(T.c1 - T.c0) * 4);
-            }
+        if (tally) {   // hand the tile to the committer warp; never run > 2 tiles ahead of it
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&tdone[kt & 1u]);
+            ++kt;
+            if (kt >= 2) mbar_wait(&cdone[kt & 1u], ((kt - 2) >> 1) & 1u);
         }
     }
 }
@@ -274,38 +298,46 @@ __device__ __forceinline__ uint32_t micro_value(uint32_t k, uint32_t phase, uint
 }
 
 constexpr int MB = 256;            // threads; one 4 KiB tile (1024 words) per CTA pass (L279)
+constexpr int MBLK = 8;            // tiles per CTA block: one commit per 32 KiB block
 
-__global__ void __launch_bounds__(MB) micro_kernel(launch_ctx lc, proact_micro_params p)
+__global__ void __launch_bounds__(MB, 4) micro_kernel(launch_ctx lc, proact_micro_params p)
 {
     if (proact::agent_dispatch(lc)) return;
     const region_dev &R = lc.ctx->region[p.region];
     const uint64_t w_lo = R.own_off / 4, w_hi = (R.own_off + R.own_bytes) / 4;
     const uint64_t ntiles = (w_hi - w_lo + 1023) / 1024;
-    for (uint64_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
-        const uint64_t t0 = w_lo + t * 1024, t1 = min(t0 + 1024, w_hi);
-        if (!p.scattered) {
-            const uint64_t k = t0 + 4 * threadIdx.x;
-            if (k + 4 <= t1) {
-                uint4 v;
-                v.x = micro_value((uint32_t)k, p.phase, p.seed, p.K);
-                v.y = micro_value((uint32_t)k + 1, p.phase, p.seed, p.K);
-                v.z = micro_value((uint32_t)k + 2, p.phase, p.seed, p.K);
-                v.w = micro_value((uint32_t)k + 3, p.phase, p.seed, p.K);
-                proact::put(lc, p.region, k * 4, v);
+    const uint64_t nblk = (ntiles + MBLK - 1) / MBLK;
+    for (uint64_t bk = proact::producer_block(lc); bk < nblk; bk += proact::producer_grid(lc)) {
+        const uint64_t tb0 = bk * MBLK, tb1 = min(tb0 + MBLK, ntiles);
+        for (uint64_t t = tb0; t < tb1; ++t) {   // the paper's 4 KiB per source block pass
+            const uint64_t t0 = w_lo + t * 1024, t1 = min(t0 + 1024, w_hi);
+            if (!p.scattered) {
+                const uint64_t k = t0 + 4 * threadIdx.x;
+                if (k + 4 <= t1) {
+                    uint4 v;
+                    v.x = micro_value((uint32_t)k, p.phase, p.seed, p.K);
+                    v.y = micro_value((uint32_t)k + 1, p.phase, p.seed, p.K);
+                    v.z = micro_value((uint32_t)k + 2, p.phase, p.seed, p.K);
+                    v.w = micro_value((uint32_t)k + 3, p.phase, p.seed, p.K);
+                    proact::put(lc, p.region, k * 4, v);
+                } else {
+                    for (uint64_t q = k; q < t1 && q < k + 4; ++q)
+                        proact::put(lc, p.region, q * 4, micro_value((uint32_t)q, p.phase, p.seed, p.K));
+                }
             } else {
-                for (uint64_t q = k; q < t1 && q < k + 4; ++q)
-                    proact::put(lc, p.region, q * 4, micro_value((uint32_t)q, p.phase, p.seed, p.K));
-            }
-        } else {
-            // scattered store order inside the 4 KiB tile: position (j*389) mod 1024 (bijection)
-            for (int s = 0; s < 4; ++s) {
-                const uint32_t jj = threadIdx.x + MB * s;
-                const uint64_t q = t0 + ((jj * 389u) & 1023u);
-                if (q < t1) proact::put(lc, p.region, q * 4, micro_value((uint32_t)q, p.phase, p.seed, p.K));
+                // scattered store order inside the 4 KiB tile: position (j*389) mod 1024 (bijection)
+                for (int s = 0; s < 4; ++s) {
+                    const uint32_t jj = threadIdx.x + MB * s;
+                    const uint64_t q = t0 + ((jj * 389u) & 1023u);
+                    if (q < t1) proact::put(lc, p.region, q * 4, micro_value((uint32_t)q, p.phase, p.seed, p.K));
+                }
             }
         }
         __syncthreads();
-        if (threadIdx.x == 0) proact::commit_span(lc, p.region, t0 * 4, (t1 - t0) * 4);
+        if (threadIdx.x == 0) {
+            const uint64_t a = w_lo + tb0 * 1024, b = min(w_lo + tb1 * 1024, w_hi);
+            proact::commit_span(lc, p.region, a * 4, (b - a) * 4);
+        }
     }
 }
 
