@@ -38,7 +38,7 @@ extern "C" {
 #endif
 
 #define PROACT_MAX_RANKS 16
-#define PROACT_BULK_SMEM (32 * 1024)   /* min dynamic smem of a launch with TMA pushes */
+#define PROACT_BULK_SMEM (33 * 1024)   /* min dynamic smem of a launch with TMA pushes */
 #define PROACT_MAX_REGIONS 8
 
 /* ---- status codes ------------------------------------------------------------------------ */
@@ -217,6 +217,11 @@ int proact_last_vote(void);
  * (n_own_chunks * world uint32, row-major) to host memory `out` and zero them.  Synchronises
  * the device.  INVALID if debug counters are off or n is too small. */
 int proact_region_debug_deliveries(int region, uint32_t *out, size_t n);
+
+/* Debug (PROACT_DEBUG=2 at init): agent cycle accounting since the last call, 8 counters:
+ * [0] discovery-wait cycles, [1] batch-processing cycles, [2] batches, [3] units,
+ * [4] TMA push-pipeline cycles, [5] store-drain cycles.  Synchronises the device; resets. */
+int proact_debug_agent_prof(unsigned long long *out8);
 
 /* COLLECTIVE host-side barrier of all ranks (no device work): e.g. to read replicas from the
  * host between phases without a peer's next phase overwriting them. */

@@ -82,6 +82,7 @@ struct dev_ctx {
     uint32_t *err_host;                        /* host-mapped mirror (plain stores) */
     uint32_t *vote;                            /* [2] local vote words, by epoch parity */
     uint32_t *vote_host;                       /* host-mapped: (epoch+1)<<1 | global vote */
+    unsigned long long *prof;                  /* PROACT_DEBUG=2: agent cycle accounting [8] */
     region_dev region[PROACT_MAX_REGIONS];
 };
 
@@ -103,7 +104,7 @@ struct launch_ctx {
 
 /* error word encoding: (site << 8) | (-PROACT_ERR_*) */
 enum { SITE_AGENT_POLL = 1, SITE_AGENT_CREDIT = 2, SITE_WAIT_RANGE = 3, SITE_WAIT_ALL = 4,
-       SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7 };
+       SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7, SITE_AGENT_PUSH = 8 };
 
 #ifdef __CUDACC__
 

@@ -88,6 +88,7 @@ def _declare(L):
         "proact_last_vote": (i, []),
         "proact_check": (i, []),
         "proact_host_barrier": (i, []),
+        "proact_debug_agent_prof": (i, [ctypes.POINTER(ctypes.c_ulonglong)]),
         "proact_launch_count": (u64, []),
         "proact_plan_slices": (i, [i, ctypes.POINTER(u64), u64, ctypes.POINTER(u64), ctypes.POINTER(u32)]),
         "proact_rdv_allgather": (i, [cp, i, i, vp, sz, vp]),

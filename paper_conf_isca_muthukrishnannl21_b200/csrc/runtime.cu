@@ -467,7 +467,9 @@ __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t ma
 }
 
 // PROACT_AGENT_SEPARATE: the transfer agent as its own kernel (own registers, TMA staging ring)
-constexpr size_t AGENT_SMEM = 128 * 1024 + 256;
+// staging ring: 8 x 16 KiB (+ metadata) for up to 32 agent CTAs, 8 x 8 KiB beyond (2 per SM)
+constexpr size_t AGENT_SMEM = 128 * 1024 + 1024;
+constexpr size_t AGENT_SMEM_SMALL = 64 * 1024 + 1024;
 __global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc) { proact::agent_loop(lc); }
 
 RankCtx *need_ctx() { return tl; }
@@ -539,6 +541,11 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     c->h.vote = (uint32_t *)(c->meta + 4 * MAXR + 64);
     c->h.err_host = c->d_err_host;
     c->h.vote_host = c->d_vote_host;
+    c->h.prof = nullptr;
+    if (env_int("PROACT_DEBUG", 0) >= 2) {
+        if (cudaMalloc((void **)&c->h.prof, 64) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        cudaMemset(c->h.prof, 0, 64);
+    }
     // rendezvous
     int rc = c->shm.open(c->job, ngpus);
     if (rc) return fail(rc);
@@ -841,7 +848,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         // producer grid leaves one slot per agent CTA; my stream waits for the agent.
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
-        const size_t asmem = cfg.push == PROACT_PUSH_BULK ? AGENT_SMEM : 0;
+        const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         CK(cudaEventRecord(c->ev_start, s));
         CK(cudaStreamWaitEvent(c->side, c->ev_start, 0));
         agent_kernel<<<agent_ctas, agent_block, asmem, c->side>>>(la);
@@ -1002,6 +1009,18 @@ int proact_rdv_allgather(const char *job, int world, int rank, const void *mine,
     int rc2 = shm.barrier();
     shm.close(true);
     return rc ? rc : rc2;
+}
+
+int proact_debug_agent_prof(unsigned long long *out8)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (!c->h.prof || !out8) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CK(cudaDeviceSynchronize());
+    CK(cudaMemcpy(out8, c->h.prof, 64, cudaMemcpyDeviceToHost));
+    CK(cudaMemset(c->h.prof, 0, 64));
+    return PROACT_OK;
 }
 
 int proact_host_barrier(void)

@@ -9,7 +9,14 @@ exercised on the single-GPU boxes this project is tested on.
 """
 from __future__ import annotations
 
+import os
 import threading
+
+# Several ranks in one process share the device's hardware work queues; with the default 8
+# connections, streams of different ranks alias onto one queue and a rank's stream waiting on
+# a cross-rank flag can block another rank's queued launch (a false dependency -> deadlock).
+# 32 connections (the maximum) must be requested before the CUDA context is created.
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 import torch
 
@@ -45,7 +52,12 @@ def run_ranks(G: int, fn, *args, device: int = 0, job: str | None = None, timeou
         t.join(timeout)
     if any(t.is_alive() for t in th):
         raise TimeoutError(f"loopback ranks did not finish within {timeout}s")
-    for e in errors:
-        if e is not None:
-            raise e
+    bad = [(r, e) for r, e in enumerate(errors) if e is not None]
+    if bad:
+        if len(bad) > 1:   # a rank's failure often makes the others time out: report them all
+            import sys
+            for r, e in bad[1:]:
+                print(f"[loopback] rank {r} also failed: {type(e).__name__}: {e}", file=sys.stderr)
+        r0, e0 = min(bad, key=lambda x: 0 if not isinstance(x[1], Exception) or "TIMEOUT" not in str(x[1]) else 1)
+        raise e0
     return results

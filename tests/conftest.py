@@ -1,6 +1,10 @@
 import os
 import sys
 
+# loopback ranks (threads on one GPU) need more hardware queues than the default 8: set before
+# any CUDA context exists (see paper_conf_isca_muthukrishnannl21_b200/loopback.py)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))

@@ -17,6 +17,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # loopback ranks: see loopback.py
 import statistics
 import sys
 import time

@@ -2,6 +2,7 @@
 import itertools
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # loopback ranks: see loopback.py
 import statistics
 import sys
 

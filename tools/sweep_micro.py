@@ -5,6 +5,7 @@ replicated GB/s = (G-1) * R / phase time, per mechanism / chunk / agent warps / 
 import itertools
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # loopback ranks: see loopback.py
 import statistics
 import sys
 
@@ -42,6 +43,9 @@ def body(r, G_):
             rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[mech], agent_warps=w, discovery=d,
                           piece_bytes=pc, push=pu, agent_kernel=ak)
             ts = []
+            if os.environ.get("PROACT_DEBUG") == "2":
+                import ctypes
+                rt.lib().proact_debug_agent_prof((ctypes.c_ulonglong * 8)())
             for k in range(PH):
                 rt.host_barrier()
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -50,7 +54,13 @@ def body(r, G_):
                 b.record(s)
                 s.synchronize()
                 ts.append(a.elapsed_time(b))
-            out.append({"chunk": ch, "mech": mech, "warps": w, "disc": d, "piece": pc, "push": pu, "akern": ak,
+            prof = None
+            if os.environ.get("PROACT_DEBUG") == "2":
+                import ctypes
+                arr = (ctypes.c_ulonglong * 8)()
+                rt.lib().proact_debug_agent_prof(arr)
+                prof = list(arr)[:6]
+            out.append({"prof": prof, "chunk": ch, "mech": mech, "warps": w, "disc": d, "piece": pc, "push": pu, "akern": ak,
                         "ms": statistics.median(ts[2:])})
     return out
 
