@@ -206,15 +206,15 @@ int env_int(const char *name, int dflt) {
 proact_config default_config() {
     proact_config c{};
     c.mech = PROACT_MECH_FUSED;
-    c.push = PROACT_PUSH_VEC16;
-    c.agent_warps = 16;
+    c.push = PROACT_PUSH_BULK;
+    c.agent_warps = 16;         // with PUSH_BULK + SEPARATE: 16 agent CTAs, one TMA issuer each
     c.block = 256;
     c.piece_bytes = 64 * 1024;
     c.watchdog_ms = 20000;
     c.grid_cap = 0;
     c.chunk_bytes = 128 * 1024;   // the paper's V100 profiler choice (Table II)
     c.discovery = PROACT_DISCOVER_QUEUE;
-    c.agent_kernel = PROACT_AGENT_FUSED;
+    c.agent_kernel = PROACT_AGENT_SEPARATE;
     return c;
 }
 
@@ -856,8 +856,29 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         CK(cudaEventRecord(c->ev_done, c->side));
         c->launches++;
         lc.agent_ctas = 0;
+        // producer slots an agent CTA displaces on its SM (shared memory / registers / threads)
+        unsigned lost = 1;
+        {
+            cudaFuncAttributes fa, aa;
+            int smem_sm = 0, regs_sm = 0, thr_sm = 0;
+            if (cudaFuncGetAttributes(&fa, kernel) == cudaSuccess &&
+                cudaFuncGetAttributes(&aa, (const void *)agent_kernel) == cudaSuccess &&
+                cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device) == cudaSuccess &&
+                cudaDeviceGetAttribute(&regs_sm, cudaDevAttrMaxRegistersPerMultiprocessor, c->device) == cudaSuccess &&
+                cudaDeviceGetAttribute(&thr_sm, cudaDevAttrMaxThreadsPerMultiProcessor, c->device) == cudaSuccess) {
+                const long ps = (long)fa.sharedSizeBytes + (long)smem + 1024, as = (long)aa.sharedSizeBytes + (long)asmem + 1024;
+                const long pr = (long)fa.numRegs * block, ar = (long)aa.numRegs * agent_block;
+                long fit = nb;
+                if (ps > 0) fit = std::min(fit, (smem_sm - as) / ps);
+                if (pr > 0) fit = std::min(fit, (regs_sm - ar) / pr);
+                fit = std::min(fit, (long)(thr_sm - (long)agent_block) / (long)block);
+                fit = std::max(0L, fit);
+                lost = (unsigned)std::max(1L, (long)nb - fit);
+            }
+        }
         unsigned total = grid ? grid : cap;
-        if (total + agent_ctas > cap) total = cap > agent_ctas ? cap - agent_ctas : 1;
+        const unsigned reserve = std::min(cap - 1, agent_ctas * lost);
+        if (total + reserve > cap) total = cap - reserve;
         *(launch_ctx *)args[0] = lc;
         CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
         CK(cudaStreamWaitEvent(s, c->ev_done, 0));
