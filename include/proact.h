@@ -203,6 +203,11 @@ int proact_region_rechunk(int region, size_t chunk_bytes);
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid,
                   unsigned block, void **args, size_t smem, void *stream);
 
+/* 1 if the next proact_launch of this rank will run tallies and the agent (FUSED with G > 1, or
+ * ELIDE), 0 if not (LOCAL / INLINE / BULK, or FUSED on a single rank): lets a workload pick a
+ * kernel instantiation without the tally machinery. */
+int proact_launch_tallies(void);
+
 /* Close phase e on `stream` (a8): peers get the credit "rank finished phase e" (write-after-read
  * guard for ping-pong replicas, reading R6), a BULK launch's copies are issued first, and in
  * BARRIER mode the stream also waits for every peer's credit (L125).  Then the rank's epoch

@@ -85,6 +85,7 @@ def _declare(L):
         "proact_launch": (i, [ctypes.POINTER(i), i, vp, ctypes.c_uint, ctypes.c_uint,
                               ctypes.POINTER(vp), sz, vp]),
         "proact_phase_sync": (i, [vp, i]),
+        "proact_launch_tallies": (i, []),
         "proact_last_vote": (i, []),
         "proact_check": (i, []),
         "proact_host_barrier": (i, []),

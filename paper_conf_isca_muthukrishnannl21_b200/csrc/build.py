@@ -30,13 +30,21 @@ def _stale() -> bool:
     return any(os.path.getmtime(s) > t for s in srcs)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Build libproact.so; `defines` (e.g. ["PROACT_JACOBI_RING=8"]) + `out` build a variant."""
+    global OUT
+    if out is not None:
+        saved, OUT = OUT, out
+        try:
+            return build(True, verbose, defines)
+        finally:
+            OUT = saved
     if not force and not _stale():
         return OUT
     objs = []
     for s in SOURCES:
         obj = os.path.join(HERE, s.replace(".cu", ".o"))
-        cmd = [NVCC, *FLAGS, "-I", INC, "-c", os.path.join(HERE, s), "-o", obj]
+        cmd = [NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-I", INC, "-c", os.path.join(HERE, s), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
@@ -58,4 +66,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 if __name__ == "__main__":
-    print(build(force="-f" in sys.argv, verbose="-v" in sys.argv))
+    # python build.py [-f] [-v] [-o OUT.so] [-D NAME=VALUE ...]
+    argv = sys.argv[1:]
+    defs, out = [], None
+    for i, a in enumerate(argv):
+        if a == "-D":
+            defs.append(argv[i + 1])
+        if a == "-o":
+            out = argv[i + 1]
+    print(build(force="-f" in argv, verbose="-v" in argv, defines=defs, out=out))

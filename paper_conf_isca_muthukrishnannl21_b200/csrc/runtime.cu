@@ -790,6 +790,15 @@ int proact_region_debug_deliveries(int id, uint32_t *out, size_t n)
     return PROACT_OK;
 }
 
+int proact_launch_tallies(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return 0;
+    const int m = c->cfg.mech;
+    if (m == PROACT_MECH_ELIDE) return 1;
+    return m == PROACT_MECH_FUSED && c->world > 1;
+}
+
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
                   void **args, size_t smem, void *stream)
 {

@@ -74,7 +74,13 @@ __device__ __forceinline__ float ld_f(const float *p)
 // the CTA's tiles without draining.  Every input row is read from HBM once per tile (+2 halo
 // rows per tile, L2 hits); outputs are 16-byte stores.
 constexpr int JC = 8;                   // compute warps
-constexpr int JB = (JC + 2) * 32;       // + one producer (TMA) warp + one committer warp
+// Two instantiations: TALLY = false (no remote destinations this launch: LOCAL / INLINE / BULK /
+// G = 1) has 8 compute + 1 TMA warp and the register budget of 4 CTAs/SM; TALLY = true adds a
+// committer warp that publishes the tile tallies so the compute warps never wait on a release.
+template <bool TALLY> struct JCfg {
+    static constexpr int threads = (JC + 1 + (TALLY ? 1 : 0)) * 32;
+    static constexpr int minb = TALLY ? 3 : 4;
+};
 constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
 #ifndef PROACT_JACOBI_RING
 #define PROACT_JACOBI_RING 16
@@ -161,7 +167,9 @@ __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_ja
     }
 }
 
-__global__ void __launch_bounds__(JB, 3) jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
+template <bool TALLY>
+__global__ void __launch_bounds__(JCfg<TALLY>::threads, JCfg<TALLY>::minb)
+jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 {
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ __align__(128) unsigned char jsm[];
@@ -170,7 +178,7 @@ __global__ void __launch_bounds__(JB, 3) jacobi_kernel(launch_ctx lc, proact_jac
     uint64_t *empty = full + JS;
     uint64_t *tdone = empty + JS;    // [2] compute warps finished tile k (k & 1)
     uint64_t *cdone = tdone + 2;     // [2] committer finished tile k (k & 1)
-    const bool tally = proact::uses_agent(lc);
+    const bool tally = TALLY && proact::uses_agent(lc);
     const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows);
     const int rb = p.rows_per_tile;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -195,7 +203,7 @@ __global__ void __launch_bounds__(JB, 3) jacobi_kernel(launch_ctx lc, proact_jac
         if (lane == 0) jacobi_stream(lc, p, ring, full, empty, t_first, P, ntiles, nstrips, nbands);
         return;
     }
-    if (warp == JC + 1) {
+    if (TALLY && warp == JC + 1) {
         // (a3) committer warp: after the compute warps' mbarrier arrival for tile k (release ->
         // acquire at CTA scope), commit the tile's rows with release RMWs, merged per chunk.
         // The compute warps never stall on the commit's fence latency.
@@ -372,11 +380,16 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
     int regs[1] = {region_out};
     static bool attr = false;   // > 48 KiB of dynamic shared memory needs the opt-in
     if (!attr) {
-        if (cudaFuncSetAttribute(jacobi_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) != cudaSuccess)
+        if (cudaFuncSetAttribute(jacobi_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) !=
+                cudaSuccess ||
+            cudaFuncSetAttribute(jacobi_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) !=
+                cudaSuccess)
             return PROACT_ERR_CUDA;
         attr = true;
     }
-    return proact_launch(regs, 1, (const void *)jacobi_kernel, 0, JB, args, JSMEM, stream);
+    if (proact_launch_tallies())
+        return proact_launch(regs, 1, (const void *)jacobi_kernel<true>, 0, JCfg<true>::threads, args, JSMEM, stream);
+    return proact_launch(regs, 1, (const void *)jacobi_kernel<false>, 0, JCfg<false>::threads, args, JSMEM, stream);
 }
 
 int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int scattered, void *stream)
