@@ -114,11 +114,18 @@ def _declare(L):
         "proact_pagerank_ranks": (i, [i, vp, vp]),
         "proact_sssp_phase": (i, [i, i, i, i, vp]),
     }
+    missing = []
     for name, (res, args) in sigs.items():
-        f = getattr(L, name)
+        try:
+            f = getattr(L, name)
+        except AttributeError:
+            if LIB_PATH.endswith("libproact.so") and "PROACT_LIB" not in os.environ:
+                raise
+            missing.append(name)   # an older variant build (tools/ sweeps): tolerate
+            continue
         f.restype = res
         f.argtypes = args
-    return sorted(sigs)
+    return sorted(set(sigs) - set(missing))
 
 
 EXPORTED: list[str] = []

@@ -178,7 +178,12 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     uint64_t *empty = full + JS;
     uint64_t *tdone = empty + JS;    // [2] compute warps finished tile k (k & 1)
     uint64_t *cdone = tdone + 2;     // [2] committer finished tile k (k & 1)
-    const bool tally = TALLY && proact::uses_agent(lc);
+#ifndef PROACT_JACOBI_RT_TALLY
+#define PROACT_JACOBI_RT_TALLY 1
+#endif
+    // (the runtime test in the TALLY=false instantiation keeps its compute loop's code identical
+    //  to the measured-fastest build; with tallies off at compile time it was ~15% slower)
+    const bool tally = (TALLY || PROACT_JACOBI_RT_TALLY) && proact::uses_agent(lc);
     const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows);
     const int rb = p.rows_per_tile;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -279,11 +284,19 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             cur = dn;
             qcur = qdn;
         }
-        if (tally) {   // hand the tile to the committer warp; never run > 2 tiles ahead of it
+        if (tally && TALLY) {   // hand the tile to the committer warp; never run > 2 tiles ahead
             __syncwarp();
             if (lane == 0) mbar_arrive(&tdone[kt & 1u]);
             ++kt;
             if (kt >= 2) mbar_wait(&cdone[kt & 1u], ((kt - 2) >> 1) & 1u);
+        } else if (tally) {   // no committer warp: compute warps meet, warp 0 commits
+            asm volatile("bar.sync 1, %0;" ::"r"(JC * 32) : "memory");
+            if (warp == 0)
+                for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
+                    const int i = k0 + lane;
+                    warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4,
+                                (uint32_t)(T.c1 - T.c0) * 4);
+                }
         }
     }
 }
