@@ -293,24 +293,39 @@ __global__ void __launch_bounds__(GB, 6) pagerank_kernel(launch_ctx lc, PrParams
         }
         __syncthreads();
         const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
-        for (;;) {
-            uint32_t k = 0;
-            if (sub == 0) k = atomicAdd(&next, 1u);
-            k = __shfl_sync(gmask, k, lead);
-            const uint32_t v = lo + k;
-            if (v >= hi) break;
-            const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
-            if (e1 - e0 > HEAVY) {
-                bool queued = false;
-                if (sub == 0) {
-                    const uint32_t h = atomicAdd(&nheavy, 1u);
-                    if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
-                }
-                if (__shfl_sync(gmask, queued, lead)) continue;
+        for (;;) {   // a warp takes 4 vertices (one per 8-lane group); control flow stays converged
+            uint32_t k4 = 0;
+            if ((threadIdx.x & 31) == 0) k4 = atomicAdd(&next, 4u);
+            k4 = __shfl_sync(0xFFFFFFFFu, k4, 0);
+            if (lo + k4 >= hi) break;
+            const uint32_t v = lo + k4 + ((threadIdx.x & 31) >> 3);
+            uint32_t e0 = 0, e1 = 0;
+            if (v < hi) {
+                e0 = p.g.colptr[v - p.g.v0];
+                e1 = p.g.colptr[v - p.g.v0 + 1];
             }
-            double s = pr_sum(p.g.rowidx, cin, e0 + sub, e1, GL, pf, pl);
-            for (int o = GL / 2; o > 0; o >>= 1) s += __shfl_xor_sync(gmask, s, o);
-            if (sub == 0) pr_finish(lc, p, v, s);
+            bool queued = false;
+            if (sub == 0 && e1 - e0 > HEAVY) {
+                const uint32_t h = atomicAdd(&nheavy, 1u);
+                if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
+            }
+            queued = __shfl_sync(0xFFFFFFFFu, queued, lead);
+            if (queued) e1 = e0;   // the hub is reduced by the whole CTA below
+            const uint32_t maxd = __reduce_max_sync(0xFFFFFFFFu, e1 - e0);
+            double s = 0.0;
+            for (uint32_t b = sub; b < maxd; b += 4 * GL) {
+                uint32_t u[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const uint32_t e = e0 + b + q * GL;
+                    u[q] = e < e1 ? ld_stream_u(p.g.rowidx + e, pf) : 0xFFFFFFFFu;
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (u[q] != 0xFFFFFFFFu) s += (double)ld_gather_f(cin + u[q], pl);
+            }
+            for (int o = GL / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, o);
+            if (sub == 0 && v < hi && !queued) pr_finish(lc, p, v, s);
         }
         __syncthreads();
         const uint32_t nh = min(nheavy, (uint32_t)MAXHEAVY);
@@ -416,25 +431,32 @@ __global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p
         __syncthreads();
         const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
         bool changed = false;
-        for (;;) {
-            uint32_t k = 0;
-            if (sub == 0) k = atomicAdd(&next, 1u);
-            k = __shfl_sync(gmask, k, lead);
-            const uint32_t v = lo + k;
-            if (v >= hi) break;
-            const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
-            if (e1 - e0 > HEAVY) {
-                bool queued = false;
-                if (sub == 0) {
-                    const uint32_t h = atomicAdd(&nheavy, 1u);
-                    if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
-                }
-                if (__shfl_sync(gmask, queued, lead)) continue;
+        for (;;) {   // a warp takes 4 vertices (one per 8-lane group); control flow stays converged
+            uint32_t k4 = 0;
+            if ((threadIdx.x & 31) == 0) k4 = atomicAdd(&next, 4u);
+            k4 = __shfl_sync(0xFFFFFFFFu, k4, 0);
+            if (lo + k4 >= hi) break;
+            const uint32_t v = lo + k4 + ((threadIdx.x & 31) >> 3);
+            uint32_t e0 = 0, e1 = 0;
+            int32_t old = INT32_MAX;
+            if (v < hi) {
+                e0 = p.g.colptr[v - p.g.v0];
+                e1 = p.g.colptr[v - p.g.v0 + 1];
+                old = din[v];
             }
-            const int32_t old = din[v];
-            int32_t best = sssp_relax(p, chg, cshift, cdiv, din, e0 + sub, e1, GL, old, pf, pl);
-            for (int o = GL / 2; o > 0; o >>= 1) best = min(best, __shfl_xor_sync(gmask, best, o));
-            if (sub == 0) {
+            bool queued = false;
+            if (sub == 0 && e1 - e0 > HEAVY) {
+                const uint32_t h = atomicAdd(&nheavy, 1u);
+                if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
+            }
+            queued = __shfl_sync(0xFFFFFFFFu, queued, lead);
+            if (queued) e1 = e0;
+            const uint32_t maxd = __reduce_max_sync(0xFFFFFFFFu, e1 - e0);
+            int32_t best = old;
+            for (uint32_t b = sub; b < maxd; b += 2 * GL)
+                best = sssp_relax(p, chg, cshift, cdiv, din, e0 + b, min(e1, e0 + b + 2 * GL), GL, best, pf, pl);
+            for (int o = GL / 2; o > 0; o >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, o));
+            if (sub == 0 && v < hi && !queued) {
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
                 changed |= best != old;
             }
