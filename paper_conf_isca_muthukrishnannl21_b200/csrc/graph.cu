@@ -33,8 +33,19 @@ namespace {
 constexpr int GB = 256;            // threads per CTA
 constexpr int GT = 1024;           // vertices per tile (4 KiB of output, the paper's L279)
 constexpr int GL = 8;              // lanes per light vertex
-constexpr uint32_t HEAVY = 2048;   // in-degree above which the whole CTA reduces a vertex
-constexpr int MAXHEAVY = 64;       // per-tile hub list (overflow: the group does it itself)
+constexpr int RUN = 8;             // consecutive in-edges per thread per round (merge path)
+constexpr uint32_t SPLIT = 32768;  // max in-edges per work item: bigger tiles are split
+
+// Work item = (vertex tile, in-edge sub-range).  Tiles whose in-edges exceed SPLIT (hubs) are
+// split over several items (processed by different CTAs, split items first); their partial
+// sums meet in a per-split-tile global accumulator and the last item to arrive finishes the
+// tile.  Every item then carries about the same number of edges: the CTAs stay balanced on a
+// power-law graph.
+struct Item {
+    uint32_t tile, e0, e1;   // edges [e0, e1) (local CSC indices)
+    uint32_t nsplit;         // items of this tile (1 = unsplit)
+    uint32_t slot, pad[3];   // split-tile accumulator slot
+};
 
 struct GraphDev {
     const uint32_t *colptr;   // [nv + 1]
@@ -42,7 +53,11 @@ struct GraphDev {
     const int32_t *w;         // [E_own] weights (SSSP) or nullptr
     const uint32_t *outdeg;   // [V] global out-degree (multi-edges counted)
     float *r_own;             // [nv] PageRank values of my vertices
-    uint32_t V, v0, nv, pad;
+    const Item *items;        // [nitems]
+    unsigned long long *acc_f;   // [nslot * GT] split-tile fixed-point sums (PageRank), zero between launches
+    int32_t *acc_i;           // [nslot * GT] split-tile minima (SSSP), INT32_MAX between launches
+    uint32_t *acc_cnt;        // [nslot] arrivals of a split tile's items
+    uint32_t V, v0, nv, nitems;
 };
 
 struct Graph {
@@ -52,6 +67,11 @@ struct Graph {
     uint32_t *colptr = nullptr, *rowidx = nullptr, *outdeg = nullptr;
     int32_t *w = nullptr;
     float *r_own = nullptr;
+    Item *items = nullptr;
+    uint32_t nitems = 0, nslot = 0;
+    unsigned long long *acc_f = nullptr;
+    int32_t *acc_i = nullptr;
+    uint32_t *acc_cnt = nullptr;
 };
 constexpr int MAXGRAPH = 4;
 thread_local Graph graphs[MAXGRAPH];
@@ -248,163 +268,148 @@ __device__ __forceinline__ double block_sum_f64(double x, double *red)
     return t;   // valid in thread 0
 }
 
-// sum over edges [e0, e1) with stride `step` starting at `first`, 4 gathers in flight per lane
-__device__ __forceinline__ double pr_sum(const uint32_t *rowidx, const float *cin, uint32_t first, uint32_t e1,
-                                         uint32_t step, uint64_t pf, uint64_t pl)
+// Local vertex index i (0..nv_tile-1) of edge e of the tile: the last i with cp[i] <= e (cp in
+// shared memory, cp[nv_tile] = end of the tile's edges; zero-degree vertices are skipped).
+__device__ __forceinline__ uint32_t vertex_of(const uint32_t *cp, uint32_t nvt, uint32_t e)
 {
-    double s = 0.0;
-    uint32_t e = first;
-    for (; e + 3 * step < e1; e += 4 * step) {
-        const uint32_t u0 = ld_stream_u(rowidx + e, pf), u1 = ld_stream_u(rowidx + e + step, pf);
-        const uint32_t u2 = ld_stream_u(rowidx + e + 2 * step, pf), u3 = ld_stream_u(rowidx + e + 3 * step, pf);
-        const float c0 = ld_gather_f(cin + u0, pl), c1 = ld_gather_f(cin + u1, pl);
-        const float c2 = ld_gather_f(cin + u2, pl), c3 = ld_gather_f(cin + u3, pl);
-        s += (double)c0;
-        s += (double)c1;
-        s += (double)c2;
-        s += (double)c3;
+    uint32_t lo = 0, hi = nvt;
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (cp[mid] <= e) lo = mid;
+        else hi = mid;
     }
-    for (; e < e1; e += step) s += (double)ld_gather_f(cin + ld_stream_u(rowidx + e, pf), pl);
-    return s;
+    return lo;
 }
 
-// Light vertices of a tile are fetched dynamically by 8-lane groups (balances skewed degrees);
-// hubs are queued and reduced by the whole CTA afterwards.
+// Tile prologue: colptr of the tile into shared memory (+ the accumulator init by the caller).
+__device__ __forceinline__ uint32_t load_tile(const GraphDev &g, uint32_t tile, uint32_t *cp, uint32_t &lo)
+{
+    lo = g.v0 + tile * GT;
+    const uint32_t hi = min(lo + GT, g.v0 + g.nv), nvt = hi - lo;
+    for (uint32_t i = threadIdx.x; i <= nvt; i += GB) cp[i] = g.colptr[lo - g.v0 + i];
+    return nvt;
+}
+
+// Split tiles: the last item to arrive (after its global atomics) finishes the tile.
+__device__ __forceinline__ bool split_arrive(const GraphDev &g, const Item &it, uint32_t *flag)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const uint32_t old = atomicAdd(&g.acc_cnt[it.slot], 1u);
+        __threadfence();
+        *flag = old + 1 == it.nsplit;
+    }
+    __syncthreads();
+    return *flag != 0;
+}
+
+// PageRank: merge-path over the item's in-edges (RUN consecutive edges per thread, RUN gathers
+// in flight).  Per-vertex sums are accumulated EXACTLY in 2^-62 fixed point (64-bit integer
+// shared-memory atomics; every contribution is < 1 and a vertex's sum <= 1/d < 2^1, so it never
+// overflows): each term is rounded once (absolute error <= 2^-63, relative to the smallest
+// contribution ~1e-10 below 1e-9), the sum itself is exact and order independent, so results are
+// bit-reproducible for any schedule; r' = (float)((1-d)/V + d * sum) as in the oracle (R12).
+constexpr double FIX = 4611686018427387904.0;          // 2^62
+constexpr double UNFIX = 1.0 / 4611686018427387904.0;  // 2^-62
+
 __global__ void __launch_bounds__(GB, 6) pagerank_kernel(launch_ctx lc, PrParams p)
 {
     if (proact::agent_dispatch(lc)) return;
-    __shared__ uint32_t heavy[MAXHEAVY];
-    __shared__ uint32_t nheavy, next;
-    __shared__ double red[GB / 32];
+    __shared__ uint32_t acc_lo[GT], acc_hi[GT];   // 64-bit fixed point as two native 32-bit halves
+    __shared__ uint32_t cp[GT + 1];
+    __shared__ uint32_t last;
     const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
-    const uint32_t ntiles = (p.g.nv + GT - 1) / GT;
-    const uint32_t sub = threadIdx.x % GL, lead = (threadIdx.x & 31) & ~(GL - 1);
-    const uint32_t gmask = 0xFFu << lead;
-    const uint64_t pf = pol_first(), pl = pol_last();
+    const uint64_t pl = pol_last();
+    // 64-bit shared-memory atomicAdd is a CAS loop on sm_100; two 32-bit adds + carry are native
+    auto acc_add = [&](uint32_t i, unsigned long long x) {
+        const uint32_t xl = (uint32_t)x, old = atomicAdd(&acc_lo[i], xl);
+        const uint32_t carry = old + xl < old ? 1u : 0u;
+        const uint32_t xh = (uint32_t)(x >> 32) + carry;
+        if (xh) atomicAdd(&acc_hi[i], xh);
+    };
+    auto acc_get = [&](uint32_t i) { return ((unsigned long long)acc_hi[i] << 32) | acc_lo[i]; };
     bool waited = false;
-    for (uint32_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
+    for (uint32_t k = proact::producer_block(lc); k < p.g.nitems; k += proact::producer_grid(lc)) {
         if (!waited) {   // (a7) every chunk of the previous generation is in my replica
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
             waited = true;
         }
-        if (threadIdx.x == 0) {
-            nheavy = 0;
-            next = 0;
-        }
+        const Item it = p.g.items[k];
+        uint32_t lo;
+        const uint32_t nvt = load_tile(p.g, it.tile, cp, lo);
+        for (uint32_t i = threadIdx.x; i < nvt; i += GB) acc_lo[i] = acc_hi[i] = 0u;
         __syncthreads();
-        const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
-        for (;;) {   // a warp takes 4 vertices (one per 8-lane group); control flow stays converged
-            uint32_t k4 = 0;
-            if ((threadIdx.x & 31) == 0) k4 = atomicAdd(&next, 4u);
-            k4 = __shfl_sync(0xFFFFFFFFu, k4, 0);
-            if (lo + k4 >= hi) break;
-            const uint32_t v = lo + k4 + ((threadIdx.x & 31) >> 3);
-            uint32_t e0 = 0, e1 = 0;
-            if (v < hi) {
-                e0 = p.g.colptr[v - p.g.v0];
-                e1 = p.g.colptr[v - p.g.v0 + 1];
-            }
-            bool queued = false;
-            if (sub == 0 && e1 - e0 > HEAVY) {
-                const uint32_t h = atomicAdd(&nheavy, 1u);
-                if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
-            }
-            queued = __shfl_sync(0xFFFFFFFFu, queued, lead);
-            if (queued) e1 = e0;   // the hub is reduced by the whole CTA below
-            const uint32_t maxd = __reduce_max_sync(0xFFFFFFFFu, e1 - e0);
-            double s = 0.0;
-            for (uint32_t b = sub; b < maxd; b += 4 * GL) {
-                uint32_t u[4];
+        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+            const uint32_t r0 = base + threadIdx.x * RUN;
+            if (r0 < it.e1) {
+                const uint32_t r1 = min(r0 + RUN, it.e1);
+                float g[RUN];
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const uint32_t e = e0 + b + q * GL;
-                    u[q] = e < e1 ? ld_stream_u(p.g.rowidx + e, pf) : 0xFFFFFFFFu;
+                for (int q = 0; q < RUN; ++q)
+                    g[q] = r0 + q < r1 ? ld_gather_f(cin + ld_nc_u(p.g.rowidx + r0 + q), pl) : 0.f;
+                uint32_t i = vertex_of(cp, nvt, r0);
+                uint32_t nxt = cp[i + 1];
+                unsigned long long sum = 0ull;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    if (r0 + q >= r1) break;
+                    while (r0 + q >= nxt) {
+                        if (sum) acc_add(i, sum);
+                        sum = 0ull;
+                        nxt = cp[++i + 1];
+                    }
+                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
                 }
-#pragma unroll
-                for (int q = 0; q < 4; ++q)
-                    if (u[q] != 0xFFFFFFFFu) s += (double)ld_gather_f(cin + u[q], pl);
+                if (sum) acc_add(i, sum);
             }
-            for (int o = GL / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, o);
-            if (sub == 0 && v < hi && !queued) pr_finish(lc, p, v, s);
         }
         __syncthreads();
-        const uint32_t nh = min(nheavy, (uint32_t)MAXHEAVY);
-        for (uint32_t h = 0; h < nh; ++h) {   // hubs: the whole CTA, fp64 tree reduction
-            const uint32_t v = heavy[h];
-            const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
-            double s = pr_sum(p.g.rowidx, cin, e0 + threadIdx.x, e1, GB, pf, pl);
-            s = block_sum_f64(s, red);
-            if (threadIdx.x == 0) pr_finish(lc, p, v, s);
+        bool fin = true;
+        if (it.nsplit > 1) {   // hub tile: sums meet in the global accumulator
+            unsigned long long *ga = p.g.acc_f + (size_t)it.slot * GT;
+            for (uint32_t i = threadIdx.x; i < nvt; i += GB)
+                if (acc_get(i)) atomicAdd(&ga[i], acc_get(i));
+            fin = split_arrive(p.g, it, &last);
+            if (fin) {
+                for (uint32_t i = threadIdx.x; i < nvt; i += GB) {
+                    const unsigned long long v = __ldcg(&ga[i]);
+                    acc_lo[i] = (uint32_t)v;
+                    acc_hi[i] = (uint32_t)(v >> 32);
+                    ga[i] = 0ull;   // ready for the next launch
+                }
+                if (threadIdx.x == 0) p.g.acc_cnt[it.slot] = 0;
+                __syncthreads();
+            }
+        }
+        if (fin) {
+            for (uint32_t i = threadIdx.x; i < nvt; i += GB) pr_finish(lc, p, lo + i, (double)acc_get(i) * UNFIX);
+            __syncthreads();
+            if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, (uint64_t)lo * 4, (uint64_t)nvt * 4);
         }
         __syncthreads();
-        if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, (uint64_t)lo * 4, (uint64_t)(hi - lo) * 4);
     }
-}
-
-// relax edges [first, e1) stride `step` into best; sources filtered by the changed-chunk bitmap
-__device__ __forceinline__ int32_t sssp_relax(const SsspParams &p, const uint32_t *chg, uint32_t cshift,
-                                              uint32_t cdiv, const int32_t *din, uint32_t first, uint32_t e1,
-                                              uint32_t step, int32_t best, uint64_t pf, uint64_t pl)
-{
-    for (uint32_t e = first; e < e1; e += 2 * step) {
-        const bool has1 = e + step < e1;
-        const uint32_t u0 = ld_stream_u(p.g.rowidx + e, pf);
-        const uint32_t u1 = has1 ? ld_stream_u(p.g.rowidx + e + step, pf) : 0u;
-        const uint32_t g0 = cdiv ? u0 / cdiv : u0 >> cshift, g1 = cdiv ? u1 / cdiv : u1 >> cshift;
-        const bool a0 = p.first || (chg[g0 >> 5] >> (g0 & 31) & 1u);
-        const bool a1 = has1 && (p.first || (chg[g1 >> 5] >> (g1 & 31) & 1u));
-        if (a0) {
-            const int32_t du = ld_gather_i(din + u0, pl);
-            if (du != INT32_MAX) {
-                const int64_t cand = (int64_t)du + (int64_t)ld_stream_i(p.g.w + e, pf);
-                if (cand < (int64_t)best) best = (int32_t)cand;
-            }
-        }
-        if (a1) {
-            const int32_t du = ld_gather_i(din + u1, pl);
-            if (du != INT32_MAX) {
-                const int64_t cand = (int64_t)du + (int64_t)ld_stream_i(p.g.w + e + step, pf);
-                if (cand < (int64_t)best) best = (int32_t)cand;
-            }
-        }
-    }
-    return best;
-}
-
-__device__ __forceinline__ int32_t block_min_i32(int32_t x, int32_t *red)
-{
-    for (int o = 16; o > 0; o >>= 1) x = min(x, __shfl_xor_sync(0xFFFFFFFFu, x, o));
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = x;
-    __syncthreads();
-    int32_t t = INT32_MAX;
-    if (threadIdx.x < 32) {
-        t = threadIdx.x < (GB / 32) ? red[threadIdx.x] : INT32_MAX;
-        for (int o = 16; o > 0; o >>= 1) t = min(t, __shfl_xor_sync(0xFFFFFFFFu, t, o));
-    }
-    __syncthreads();
-    return t;
 }
 
 constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
 
+// SSSP: merge-path over the item's in-edges; a source is relaxed only if its chunk changed in
+// the previous round (bitmap snapshot); per-vertex minima via shared-memory atomicMin.
 __global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p)
 {
     if (proact::agent_dispatch(lc)) return;
-    __shared__ uint32_t heavy[MAXHEAVY];
-    __shared__ uint32_t nheavy, next;
-    __shared__ int32_t red[GB / 32];
+    __shared__ int32_t acc[GT];
+    __shared__ uint32_t cp[GT + 1];
     __shared__ uint32_t chg[CHG_WORDS];
+    __shared__ uint32_t last;
     const region_dev &Ri = lc.ctx->region[p.region_in];
     const int32_t *din = reinterpret_cast<const int32_t *>(Ri.base);
-    const uint32_t ntiles = (p.g.nv + GT - 1) / GT;
-    const uint32_t sub = threadIdx.x % GL, lead = (threadIdx.x & 31) & ~(GL - 1);
-    const uint32_t gmask = 0xFFu << lead;
     const uint64_t pf = pol_first(), pl = pol_last();
     // source vertex -> global chunk id: rank slices are chunk-aligned, so it is u*4/chunk_bytes
-    const uint32_t cv = Ri.chunk_bytes / 4;   // vertices per chunk
+    const uint32_t cv = Ri.chunk_bytes / 4;
     const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
     bool ready = false;
-    for (uint32_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
+    for (uint32_t k = proact::producer_block(lc); k < p.g.nitems; k += proact::producer_grid(lc)) {
         if (!ready) {   // (a7) wait for the previous generation, then snapshot its changed bits
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
             __syncthreads();
@@ -412,81 +417,99 @@ __global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p
             const bool agent = proact::uses_agent(lc);
             for (uint32_t wi = threadIdx.x; wi < CHG_WORDS && wi * 32 < Ri.n_total; wi += GB) {
                 uint32_t bits = 0;
-                for (uint32_t b = 0; b < 32; ++b) {
-                    const uint32_t g = wi * 32 + b;
+                for (uint32_t bb = 0; bb < 32; ++bb) {
+                    const uint32_t g = wi * 32 + bb;
                     if (g >= Ri.n_total) break;
                     bool c;
                     if (g >= Ri.chunk0 && g < Ri.chunk0 + Ri.n_own) c = Ri.changed_gen[g - Ri.chunk0] == gen;
                     else c = !agent || (ld_nc_u(Ri.arrive + g) & 1u);   // no flags without the agent
-                    bits |= (uint32_t)c << b;
+                    bits |= (uint32_t)c << bb;
                 }
                 chg[wi] = bits;
             }
             ready = true;
         }
-        if (threadIdx.x == 0) {
-            nheavy = 0;
-            next = 0;
+        const Item it = p.g.items[k];
+        uint32_t lo;
+        const uint32_t nvt = load_tile(p.g, it.tile, cp, lo);
+        for (uint32_t i = threadIdx.x; i < nvt; i += GB) acc[i] = INT32_MAX;
+        __syncthreads();
+        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+            const uint32_t r0 = base + threadIdx.x * RUN;
+            if (r0 < it.e1) {
+                const uint32_t r1 = min(r0 + RUN, it.e1);
+                int32_t c[RUN];
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    c[q] = INT32_MAX;
+                    if (r0 + q < r1) {
+                        const uint32_t u = ld_nc_u(p.g.rowidx + r0 + q);
+                        const uint32_t g = cdiv ? u / cdiv : u >> cshift;
+                        if (p.first || (chg[g >> 5] >> (g & 31) & 1u)) {
+                            const int32_t du = ld_gather_i(din + u, pl);
+                            if (du != INT32_MAX) {
+                                const int64_t cand = (int64_t)du + (int64_t)ld_stream_i(p.g.w + r0 + q, pf);
+                                c[q] = cand < (int64_t)INT32_MAX ? (int32_t)cand : INT32_MAX;
+                            }
+                        }
+                    }
+                }
+                uint32_t i = vertex_of(cp, nvt, r0);
+                uint32_t nxt = cp[i + 1];
+                int32_t best = INT32_MAX;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    if (r0 + q >= r1) break;
+                    while (r0 + q >= nxt) {
+                        if (best != INT32_MAX) atomicMin(&acc[i], best);
+                        best = INT32_MAX;
+                        nxt = cp[++i + 1];
+                    }
+                    best = min(best, c[q]);
+                }
+                if (best != INT32_MAX) atomicMin(&acc[i], best);
+            }
         }
         __syncthreads();
-        const uint32_t lo = p.g.v0 + t * GT, hi = min(lo + GT, p.g.v0 + p.g.nv);
-        bool changed = false;
-        for (;;) {   // a warp takes 4 vertices (one per 8-lane group); control flow stays converged
-            uint32_t k4 = 0;
-            if ((threadIdx.x & 31) == 0) k4 = atomicAdd(&next, 4u);
-            k4 = __shfl_sync(0xFFFFFFFFu, k4, 0);
-            if (lo + k4 >= hi) break;
-            const uint32_t v = lo + k4 + ((threadIdx.x & 31) >> 3);
-            uint32_t e0 = 0, e1 = 0;
-            int32_t old = INT32_MAX;
-            if (v < hi) {
-                e0 = p.g.colptr[v - p.g.v0];
-                e1 = p.g.colptr[v - p.g.v0 + 1];
-                old = din[v];
+        bool fin = true;
+        if (it.nsplit > 1) {
+            int32_t *ga = p.g.acc_i + (size_t)it.slot * GT;
+            for (uint32_t i = threadIdx.x; i < nvt; i += GB)
+                if (acc[i] != INT32_MAX) atomicMin(&ga[i], acc[i]);
+            fin = split_arrive(p.g, it, &last);
+            if (fin) {
+                for (uint32_t i = threadIdx.x; i < nvt; i += GB) {
+                    acc[i] = __ldcg(&ga[i]);
+                    ga[i] = INT32_MAX;
+                }
+                if (threadIdx.x == 0) p.g.acc_cnt[it.slot] = 0;
+                __syncthreads();
             }
-            bool queued = false;
-            if (sub == 0 && e1 - e0 > HEAVY) {
-                const uint32_t h = atomicAdd(&nheavy, 1u);
-                if (h < MAXHEAVY) { heavy[h] = v; queued = true; }
-            }
-            queued = __shfl_sync(0xFFFFFFFFu, queued, lead);
-            if (queued) e1 = e0;
-            const uint32_t maxd = __reduce_max_sync(0xFFFFFFFFu, e1 - e0);
-            int32_t best = old;
-            for (uint32_t b = sub; b < maxd; b += 2 * GL)
-                best = sssp_relax(p, chg, cshift, cdiv, din, e0 + b, min(e1, e0 + b + 2 * GL), GL, best, pf, pl);
-            for (int o = GL / 2; o > 0; o >>= 1) best = min(best, __shfl_xor_sync(0xFFFFFFFFu, best, o));
-            if (sub == 0 && v < hi && !queued) {
+        }
+        if (fin) {
+            bool changed = false;
+            for (uint32_t i = threadIdx.x; i < nvt; i += GB) {
+                const uint32_t v = lo + i;
+                const int32_t old = din[v];
+                const int32_t best = min(old, acc[i]);
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
                 changed |= best != old;
             }
-        }
-        __syncthreads();
-        const uint32_t nh = min(nheavy, (uint32_t)MAXHEAVY);
-        for (uint32_t h = 0; h < nh; ++h) {
-            const uint32_t v = heavy[h];
-            const uint32_t e0 = p.g.colptr[v - p.g.v0], e1 = p.g.colptr[v - p.g.v0 + 1];
-            const int32_t old = din[v];
-            int32_t best = sssp_relax(p, chg, cshift, cdiv, din, e0 + threadIdx.x, e1, GB, INT32_MAX, pf, pl);
-            best = min(block_min_i32(best, red), old);
+            // per-tile chunk state (SPARSE region): changed now -> flag bit + vote; push if
+            // changed now or in the previous round (the peers' ping-pong copy holds d^{k-1})
+            const int any = __syncthreads_or(changed);
             if (threadIdx.x == 0) {
-                proact::put(lc, p.region_out, (uint64_t)v * 4, best);
-                changed |= best != old;
+                const uint64_t off = (uint64_t)lo * 4;
+                const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
+                if (any) {
+                    proact::mark_changed(lc, p.region_out, off);
+                    proact::vote(lc);
+                }
+                if (any || prev) proact::mark_push(lc, p.region_out, off);
+                proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
             }
         }
-        // per-tile chunk state (SPARSE region): changed now -> flag bit + vote; push if changed
-        // now or in the previous phase (the peers' ping-pong copy holds d^{k-1}, reading R13)
-        const int any = __syncthreads_or(changed);
-        if (threadIdx.x == 0) {
-            const uint64_t off = (uint64_t)lo * 4;
-            const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
-            if (any) {
-                proact::mark_changed(lc, p.region_out, off);
-                proact::vote(lc);
-            }
-            if (any || prev) proact::mark_push(lc, p.region_out, off);
-            proact::commit_span(lc, p.region_out, off, (uint64_t)(hi - lo) * 4);
-        }
+        __syncthreads();
     }
 }
 
@@ -505,10 +528,14 @@ int graph_dev(int id, GraphDev *g)
     g->w = G.w;
     g->outdeg = G.outdeg;
     g->r_own = G.r_own;
+    g->items = G.items;
+    g->acc_f = G.acc_f;
+    g->acc_i = G.acc_i;
+    g->acc_cnt = G.acc_cnt;
     g->V = G.V;
     g->v0 = G.v0;
     g->nv = G.nv;
-    g->pad = 0;
+    g->nitems = G.nitems;
     return PROACT_OK;
 }
 
@@ -587,6 +614,43 @@ int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32
     if (E) scatter_kernel<<<1184, 256, 0, s>>>(d_src, d_dst, d_w, E, v0, v1, indeg, G.rowidx, G.w);
     GCK(cudaGetLastError());
     GCK(cudaFreeAsync(indeg, s));
+    // work items: one per 4 KiB vertex tile, tiles with more than SPLIT in-edges split
+    {
+        std::vector<uint32_t> cp((size_t)G.nv + 1);
+        GCK(cudaMemcpyAsync(cp.data(), G.colptr, 4 * cp.size(), cudaMemcpyDeviceToHost, s));
+        GCK(cudaStreamSynchronize(s));
+        const uint32_t ntiles = (G.nv + GT - 1) / GT;
+        std::vector<Item> split, whole;
+        for (uint32_t t = 0; t < ntiles; ++t) {
+            const uint32_t a = cp[(size_t)t * GT], b = cp[std::min<size_t>((size_t)(t + 1) * GT, G.nv)];
+            const uint32_t n = std::max<uint32_t>(1, (b - a + SPLIT - 1) / SPLIT);
+            for (uint32_t q = 0; q < n; ++q) {
+                Item it{};
+                it.tile = t;
+                it.e0 = a + (uint32_t)((uint64_t)(b - a) * q / n);
+                it.e1 = a + (uint32_t)((uint64_t)(b - a) * (q + 1) / n);
+                it.nsplit = n;
+                it.slot = n > 1 ? G.nslot : 0;
+                (n > 1 ? split : whole).push_back(it);
+            }
+            if (n > 1) ++G.nslot;
+        }
+        split.insert(split.end(), whole.begin(), whole.end());   // big (hub) work first
+        G.nitems = (uint32_t)split.size();
+        GCK(cudaMalloc((void **)&G.items, sizeof(Item) * std::max<size_t>(1, split.size())));
+        GCK(cudaMemcpy(G.items, split.data(), sizeof(Item) * split.size(), cudaMemcpyHostToDevice));
+        const size_t ns = std::max<uint32_t>(1, G.nslot);
+        GCK(cudaMalloc((void **)&G.acc_f, 8 * ns * GT));
+        GCK(cudaMemset(G.acc_f, 0, 8 * ns * GT));
+        GCK(cudaMalloc((void **)&G.acc_i, 4 * ns * GT));
+        GCK(cudaMemset(G.acc_i, 0x7F, 4 * ns * GT));   // 0x7F7F7F7F: re-set to INT32_MAX below
+        {
+            std::vector<int32_t> inf(ns * GT, INT32_MAX);
+            GCK(cudaMemcpy(G.acc_i, inf.data(), 4 * ns * GT, cudaMemcpyHostToDevice));
+        }
+        GCK(cudaMalloc((void **)&G.acc_cnt, 4 * ns));
+        GCK(cudaMemset(G.acc_cnt, 0, 4 * ns));
+    }
     GCK(cudaStreamSynchronize(s));
     G.used = true;
     graphs[id] = G;
@@ -602,6 +666,10 @@ int proact_graph_free(int id)
     cudaFree(G.outdeg);
     cudaFree(G.r_own);
     if (G.w) cudaFree(G.w);
+    cudaFree(G.items);
+    cudaFree(G.acc_f);
+    cudaFree(G.acc_i);
+    cudaFree(G.acc_cnt);
     G = Graph();
     return PROACT_OK;
 }
