@@ -59,6 +59,23 @@ int proact_jacobi_solve_host(const float *h_x0, float *h_out, long long N, int i
                              size_t chunk_bytes, int rows_per_tile, void *stream,
                              unsigned long long *bytes_h2d, unsigned long long *bytes_d2h);
 
+/* ---- banded-matrix Jacobi (Sec. IV-C: the paper's own Jacobi) */
+typedef struct proact_banded_params {
+    int region_in, region_out;
+    long long N, w, row0, nrows;
+    const float *a;    /* device, DIA layout (2w+1) x N: a[(o+w)*N + i] = A[i][i+o] */
+    const float *b;    /* device, N */
+} proact_banded_params;
+
+/* One Jacobi sweep of A x = b for my rows (reading R19): x'[i] = (b[i] - sum_{o != 0} A[i][i+o]
+ * x[i+o]) / A[i][i], the sum in fp32 in the order o = -w..w, each product rounded before the
+ * add, IEEE division.  region_in / region_out: two registered N-float replicas with identical
+ * whole-row slices (rank g owns rows [own_offset/4, (own_offset+own_bytes)/4)); a / b: device
+ * arrays of the full system (only my rows are read).  Waits for the peers' rows within w of my
+ * slice.  w <= 8192.  INVALID on geometry mismatch. */
+int proact_banded_phase(int region_in, int region_out, const float *a, const float *b, long long N,
+                        long long w, void *stream);
+
 /* ---- graph workloads (Sec. IV-C L265 PageRank, L267 SSSP; configs 3-4) --------- */
 
 /* Destination partition of a graph for G ranks: bounds[0..G] (host array of G+1) receive vertex

@@ -61,6 +61,8 @@ def lib():
         L.oracle_pagerank.argtypes = [i64, i64, vp, vp, i32, ctypes.c_double, vp]
         L.oracle_sssp.restype = i32
         L.oracle_sssp.argtypes = [i64, i64, vp, vp, vp, i64, i32, vp, ctypes.POINTER(i32), vp]
+        L.oracle_banded_jacobi.restype = i32
+        L.oracle_banded_jacobi.argtypes = [vp, vp, vp, i64, i64, i32]
         L.oracle_proto_run.restype = i32
         L.oracle_proto_run.argtypes = [i32, i32, i32, i32, i64, i64, i64, i32, u32, i32, u64, vp, vp]
         _lib = L
@@ -111,6 +113,17 @@ def jacobi(x0: np.ndarray, iters: int) -> np.ndarray:
     assert x.ndim == 2 and x.shape[0] == x.shape[1]
     if lib().oracle_jacobi(_p(x), x.shape[0], iters) != 0:
         raise MemoryError("oracle_jacobi")
+    return x
+
+
+def banded_jacobi(a: np.ndarray, b: np.ndarray, x0: np.ndarray, iters: int) -> np.ndarray:
+    """Banded Jacobi (NEXT-2, L271): a is the DIA array (2w+1, N), b and x0 length N."""
+    a = np.ascontiguousarray(a, dtype=np.float32)
+    b = np.ascontiguousarray(b, dtype=np.float32)
+    x = np.array(x0, dtype=np.float32, copy=True)
+    w = (a.shape[0] - 1) // 2
+    if lib().oracle_banded_jacobi(_p(a), _p(b), _p(x), x.size, w, iters) != 0:
+        raise MemoryError("oracle_banded_jacobi")
     return x
 
 

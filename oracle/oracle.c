@@ -451,3 +451,32 @@ int oracle_proto_run(int G, int P, int A, int workload, int64_t N_or_W, int64_t 
     free(S);
     return rc;
 }
+
+/* ------------------------------------------------------------------------------------------ */
+/* Banded Jacobi (Sec. IV-C: "the Jacobi solver for banded matrices ... iteratively
+ * computes the solution vector using Jacobi's method").  A in DIA layout
+ * a[(o+w)*N + i] = A[i][i+o].  Reading R19: fp32, the off-diagonal sum accumulated in the order
+ * o = -w .. w (o != 0, 0 <= i+o < N), each term a*x rounded then added (no FMA), then
+ * x'[i] = (b[i] - sum) / A[i][i] (IEEE division).  x holds x^0 on entry and x^iters on return. */
+int oracle_banded_jacobi(const float *a, const float *b, float *x, int64_t N, int64_t w, int iters)
+{
+    float *t = (float *)malloc(sizeof(float) * (size_t)(N ? N : 1));
+    if (!t) return -1;
+    float *cur = x, *nxt = t;
+    for (int k = 0; k < iters; ++k) {
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < N; ++i) {
+            float sum = 0.0f;
+            for (int64_t o = -w; o <= w; ++o) {
+                if (o == 0 || i + o < 0 || i + o >= N) continue;
+                float term = a[(o + w) * N + i] * cur[i + o];
+                sum = sum + term;
+            }
+            nxt[i] = (b[i] - sum) / a[w * N + i];
+        }
+        float *s = cur; cur = nxt; nxt = s;
+    }
+    if (cur != x) memcpy(x, cur, sizeof(float) * (size_t)N);
+    free(t);
+    return 0;
+}

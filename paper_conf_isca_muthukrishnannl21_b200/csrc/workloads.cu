@@ -362,6 +362,47 @@ __global__ void __launch_bounds__(MB, 4) micro_kernel(launch_ctx lc, proact_micr
     }
 }
 
+// ---------------------------------------------------------------- banded Jacobi (NEXT-2)
+constexpr int BB = 256;    // threads
+constexpr int BT = 1024;   // rows per tile (4 KiB of output)
+
+__device__ __forceinline__ float ld_stream_f(const float *p)
+{
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
+
+__global__ void __launch_bounds__(BB) banded_kernel(launch_ctx lc, proact_banded_params p)
+{
+    if (proact::agent_dispatch(lc)) return;
+    extern __shared__ float xs[];   // x window [i0 - w, i1 + w) of the tile
+    const float *x = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
+    const int64_t N = p.N, w = p.w, rend = p.row0 + p.nrows;
+    const int64_t ntiles = (p.nrows + BT - 1) / BT;
+    for (int64_t t = proact::producer_block(lc); t < ntiles; t += proact::producer_grid(lc)) {
+        const int64_t i0 = p.row0 + t * BT, i1 = min(i0 + (int64_t)BT, rend);
+        const int64_t lo = i0 - w > 0 ? i0 - w : 0, hi = i1 + w < N ? i1 + w : N;
+        if (threadIdx.x == 0)   // (a7) peers' rows of the previous generation within the band
+            proact::wait_range(lc, p.region_in, (uint64_t)lo * 4, (uint64_t)(hi - lo) * 4);
+        __syncthreads();
+        for (int64_t k = threadIdx.x; k < hi - lo; k += BB) xs[k] = __ldcg(x + lo + k);
+        __syncthreads();
+        for (int64_t i = i0 + threadIdx.x; i < i1; i += BB) {
+            float sum = 0.0f;
+            for (int64_t o = -w; o <= w; ++o) {
+                const int64_t j = i + o;
+                if (o == 0 || j < 0 || j >= N) continue;
+                sum = __fadd_rn(sum, __fmul_rn(ld_stream_f(p.a + (o + w) * N + i), xs[j - lo]));
+            }
+            const float v = __fdiv_rn(__fsub_rn(p.b[i], sum), p.a[w * N + i]);
+            proact::put(lc, p.region_out, (uint64_t)i * 4, v);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, (uint64_t)i0 * 4, (uint64_t)(i1 - i0) * 4);
+    }
+}
+
 }  // namespace
 
 // ================================================================ C entry points
@@ -422,6 +463,40 @@ int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int sca
 }
 
 }  // extern "C"
+
+extern "C" int proact_banded_phase(int region_in, int region_out, const float *a, const float *b, long long N,
+                                   long long w, void *stream)
+{
+    proact_region_info ri, ro;
+    int rc = proact_region_info_get(region_in, &ri);
+    if (rc) return rc;
+    rc = proact_region_info_get(region_out, &ro);
+    if (rc) return rc;
+    if (!a || !b || N < 1 || w < 0 || w > 8192 || region_in == region_out) return PROACT_ERR_INVALID;
+    if (ri.own_offset != ro.own_offset || ri.own_bytes != ro.own_bytes || ri.total_bytes != 4ull * N ||
+        ro.total_bytes != 4ull * N)
+        return PROACT_ERR_INVALID;
+    proact_banded_params p;
+    p.region_in = region_in;
+    p.region_out = region_out;
+    p.N = N;
+    p.w = w;
+    p.row0 = (long long)(ro.own_offset / 4);
+    p.nrows = (long long)(ro.own_bytes / 4);
+    p.a = a;
+    p.b = b;
+    const size_t smem = (size_t)(BT + 2 * w) * 4;
+    static size_t attr = 48 * 1024;
+    if (smem > attr) {
+        if (cudaFuncSetAttribute(banded_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+            return PROACT_ERR_CUDA;
+        attr = smem;
+    }
+    launch_ctx lc;
+    void *args[2] = {&lc, &p};
+    int regs[1] = {region_out};
+    return proact_launch(regs, 1, (const void *)banded_kernel, 0, BB, args, smem, stream);
+}
 
 // ================================================================ host-buffer Jacobi (e2e)
 namespace {

@@ -93,6 +93,41 @@ def jacobi_solve_host(x0_host, out_host, N: int, iters: int, chunk_bytes: int,
     return h2d.value, d2h.value
 
 
+# ------------------------------------------------------------------ banded Jacobi (NEXT-2)
+class Banded:
+    """The paper's Jacobi (L271): A x = b with A banded (half-bandwidth w, DIA layout), x an
+    N-float replicated vector, rows split like row_split()."""
+
+    def __init__(self, a, b, chunk_bytes: int, x0=None, device=None):
+        import numpy as np
+        G, g = rt.world(), rt.rank()
+        dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.w = (a.shape[0] - 1) // 2
+        self.N = a.shape[1]
+        self.a = torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+        self.b = torch.from_numpy(np.ascontiguousarray(b)).to(dev)
+        init = torch.zeros(self.N, dtype=torch.float32) if x0 is None else torch.from_numpy(np.asarray(x0))
+        self.bufs = [init.to(dev).clone() for _ in range(2)]
+        torch.cuda.synchronize()
+        self.r0, self.r1 = row_split(self.N, G, g)
+        # slices must be 16-byte multiples: round the split to 4 rows
+        self.r0, self.r1 = (self.r0 // 4) * 4, (self.r1 // 4) * 4 if g < G - 1 else self.N
+        self.rid = [rt.register_region(t, self.r0 * 4, (self.r1 - self.r0) * 4, chunk_bytes) for t in self.bufs]
+        self.k = 0
+
+    def step(self, stream=None, barrier: bool = False) -> None:
+        i = self.k & 1
+        check(rt.lib().proact_banded_phase(self.rid[i], self.rid[i ^ 1], ctypes.c_void_p(self.a.data_ptr()),
+                                           ctypes.c_void_p(self.b.data_ptr()), self.N, self.w, _s(stream)),
+              "banded_phase")
+        rt.phase_sync(stream, barrier=barrier)
+        self.k += 1
+
+    @property
+    def current(self) -> torch.Tensor:
+        return self.bufs[self.k & 1]
+
+
 # ------------------------------------------------------------------ microbenchmark (config 5)
 def micro_phase(rid: int, phase: int, seed: int, K: int = 1, scattered: bool = False,
                 stream=None) -> None:

@@ -25,6 +25,7 @@ RMAT_SEED = 1
 PERM_SEED = 2
 WEIGHT_SEED = 3
 MICRO_SEED = 0x5EED
+BANDED_SEED = 0xBA4D
 
 
 def build(force: bool = False) -> str:
@@ -51,6 +52,8 @@ def lib():
         L.synth_permutation.argtypes = [vp, i64, u64]
         L.synth_rmat.restype = i64
         L.synth_rmat.argtypes = [vp, vp, ctypes.c_int, i64, u64, u64]
+        L.synth_banded.restype = None
+        L.synth_banded.argtypes = [vp, vp, i64, i64, u64]
         L.synth_weights.restype = None
         L.synth_weights.argtypes = [vp, i64, u64]
         _lib = L
@@ -101,3 +104,12 @@ def weights(E: int, seed: int = WEIGHT_SEED) -> np.ndarray:
     if E:
         lib().synth_weights(_ptr(w), E, seed)
     return w
+
+
+def banded(N: int, w: int, seed: int = BANDED_SEED) -> tuple[np.ndarray, np.ndarray]:
+    """Banded system in DIA layout: a[(o+w), i] = A[i][i+o] (shape (2w+1, N)), and b (N)."""
+    a = np.empty((2 * w + 1, N), dtype=np.float32)
+    b = np.empty(N, dtype=np.float32)
+    if N:
+        lib().synth_banded(_ptr(a), _ptr(b), N, w, seed)
+    return a, b

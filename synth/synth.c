@@ -108,3 +108,26 @@ void synth_weights(int32_t *w, int64_t E, uint64_t seed)
     for (int64_t e = 0; e < E; ++e)
         w[e] = 1 + (int32_t)(synth_splitmix64(seed ^ (uint64_t)e) % 255u);
 }
+
+/* Banded system for the paper's Jacobi solver (Sec. IV-C: "Jacobi solver for
+ * banded matrices").  DIA layout: a[(o + w) * N + i] = A[i][i + o], o in [-w, w];
+ * off-diagonals -(1 + u) / (4w) with u = (splitmix64(seed ^ ((o+w)*N + i)) >> 41) * 2^-23 in
+ * [0, 1), entries outside the matrix (i + o not in [0, N)) are 0; diagonal 2 (strictly dominant:
+ * sum |off| <= 1); b[i] = 1 + (splitmix64(~seed ^ i) >> 41) * 2^-23. */
+void synth_banded(float *a, float *b, int64_t N, int64_t w, uint64_t seed)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < N; ++i) {
+        for (int64_t o = -w; o <= w; ++o) {
+            float v;
+            if (o == 0) v = 2.0f;
+            else if (i + o < 0 || i + o >= N) v = 0.0f;
+            else {
+                uint64_t m = synth_splitmix64(seed ^ (uint64_t)((o + w) * N + i)) >> 41;
+                v = -(1.0f + (float)m * (1.0f / 8388608.0f)) / (float)(4 * w);
+            }
+            a[(o + w) * N + i] = v;
+        }
+        b[i] = 1.0f + (float)(synth_splitmix64(~seed ^ (uint64_t)i) >> 41) * (1.0f / 8388608.0f);
+    }
+}
