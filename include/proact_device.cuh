@@ -93,6 +93,8 @@ struct launch_ctx {
     uint32_t armed;                            /* bit r: region r written by this launch */
     uint32_t gen[PROACT_MAX_REGIONS];          /* armed: generation produced now; else current */
     uint32_t gen_epoch[PROACT_MAX_REGIONS];    /* epoch that produced gen[r] */
+    uint8_t gen_mech[PROACT_MAX_REGIONS];      /* mechanism that produced gen[r]: decides how a
+                                                  consumer waits for it (flags / credits / none) */
     uint16_t mech;                             /* PROACT_MECH_* */
     uint16_t push;                             /* PROACT_PUSH_* */
     uint16_t agent_ctas;                       /* leading CTAs that run the agent (FUSED/ELIDE) */
@@ -328,9 +330,10 @@ __device__ __forceinline__ void vote(const launch_ctx &lc) { atomicOr(&lc.ctx->v
 /* ---------------------------------------------------------------- consumer side (a7) ------- */
 
 /* Wait (ONE thread; the caller then __syncthreads()) until every REMOTE chunk overlapping
- * [off, off + nbytes) of region r holds the region's current generation lc.gen[r].  FUSED/ELIDE
- * spin on the per-chunk arrival flags (ld.acquire.sys); INLINE/BULK on the owner's phase credit
- * (the data is complete when its producer's phase is); LOCAL returns at once.  Returns the OR of
+ * [off, off + nbytes) of region r holds the region's current generation lc.gen[r].  How depends on
+ * the mechanism that PRODUCED that generation (lc.gen_mech[r]): FUSED/ELIDE -> the per-chunk
+ * arrival flags (ld.acquire.sys); INLINE/BULK -> the owner's phase credit (the data is complete
+ * when its producer's phase is); LOCAL -> nothing (single rank, or moved by the caller).  Returns the OR of
  * the covered chunks' "changed" bits (FUSED/ELIDE only; 1 otherwise).  Generation 0 (identical
  * initial replicas, reading R16) never waits.  Must not be used on a region armed by the same
  * launch (a launch reads the previous generation of what it does not write). */
@@ -339,7 +342,9 @@ __device__ __forceinline__ uint32_t wait_range(const launch_ctx &lc, int r, uint
     const dev_ctx *C = lc.ctx;
     const region_dev &R = C->region[r];
     uint32_t gen = lc.gen[r];
-    if (gen == 0 || nbytes == 0 || lc.mech == PROACT_MECH_LOCAL) return 1u;
+    const uint32_t pm = lc.gen_mech[r];
+    if (gen == 0 || nbytes == 0 || pm == PROACT_MECH_LOCAL) return 1u;
+    const bool flags = pm == PROACT_MECH_FUSED || pm == PROACT_MECH_ELIDE;
     uint64_t hi = off + nbytes;
     uint32_t changed = 0;
     uint64_t t0 = globaltimer();
@@ -347,7 +352,7 @@ __device__ __forceinline__ uint32_t wait_range(const launch_ctx &lc, int r, uint
     for (int p = 0; p < C->world; ++p) {
         uint64_t plo = R.rank_off[p], phi = R.rank_off[p + 1];
         if (p == C->rank || phi <= off || plo >= hi || plo == phi) continue;
-        if (uses_agent(lc)) {
+        if (flags) {
             uint64_t a = (off > plo ? off : plo) - plo, b = (hi < phi ? hi : phi) - plo;
             uint32_t c0 = (uint32_t)(a / R.chunk_bytes), c1 = (uint32_t)((b - 1) / R.chunk_bytes);
             for (uint32_t c = c0; c <= c1; ++c) {
@@ -375,10 +380,12 @@ __device__ __forceinline__ void wait_all(const launch_ctx &lc, int r)
     const dev_ctx *C = lc.ctx;
     const region_dev &R = C->region[r];
     uint32_t gen = lc.gen[r];
-    if (gen == 0 || lc.mech == PROACT_MECH_LOCAL) return;
+    const uint32_t pm = lc.gen_mech[r];
+    if (gen == 0 || pm == PROACT_MECH_LOCAL) return;
+    const bool flags = pm == PROACT_MECH_FUSED || pm == PROACT_MECH_ELIDE;
     uint64_t t0 = globaltimer();
     uint32_t it = 0;
-    if (uses_agent(lc) && R.n_in != 0xFFFFFFFFu) {
+    if (flags && R.n_in != 0xFFFFFFFFu) {
         uint32_t need = gen * R.n_in;
         while (ld_acquire_sys(R.arrive_count) < need)
             if (spin_step(C, t0, it, SITE_WAIT_ALL)) return;

@@ -414,7 +414,8 @@ __global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
             __syncthreads();
             const uint32_t gen = lc.gen[p.region_in];
-            const bool agent = proact::uses_agent(lc);
+            const uint32_t pm = lc.gen_mech[p.region_in];   // how the input was produced
+            const bool agent = pm == PROACT_MECH_FUSED || pm == PROACT_MECH_ELIDE;
             for (uint32_t wi = threadIdx.x; wi < CHG_WORDS && wi * 32 < Ri.n_total; wi += GB) {
                 uint32_t bits = 0;
                 for (uint32_t bb = 0; bb < 32; ++bb) {

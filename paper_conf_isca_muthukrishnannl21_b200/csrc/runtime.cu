@@ -153,6 +153,7 @@ struct Region {
     uint32_t *d_chunk_dest = nullptr;
     uint32_t gen_done = 0;            // completed (launched) generations
     uint32_t gen_epoch = 0;           // epoch of the latest generation
+    uint8_t gen_mech = PROACT_MECH_LOCAL;   // mechanism that produced it
     int64_t last_armed_epoch = -1;
 };
 
@@ -827,15 +828,15 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         armed |= 1u << r;
     }
     lc.armed = armed;
+    // a single rank has nothing to send or receive: no tracking is needed at all, the fused
+    // launch degenerates to the plain kernel (ELIDE keeps the agent: it measures tracking).
+    if (cfg.mech == PROACT_MECH_FUSED && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
     for (int r = 0; r < c->nregions; ++r) {
         const Region &R = c->regions[r];
         lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
         lc.gen_epoch[r] = (armed >> r & 1) ? c->epoch : R.gen_epoch;
+        lc.gen_mech[r] = (armed >> r & 1) ? (uint8_t)lc.mech : R.gen_mech;
     }
-    // a single rank has nothing to send or receive: no tracking is needed at all, the fused
-    // launch degenerates to the plain kernel (ELIDE keeps the agent: it measures tracking).
-    // (Not done for G > 1 even if my masks are empty: lc.mech also drives my consumer waits.)
-    if (cfg.mech == PROACT_MECH_FUSED && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
     bool agent = (lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE) && armed;
     const bool separate = agent && cfg.agent_kernel == PROACT_AGENT_SEPARATE;
     // VEC16: agent_warps warps packed into CTAs; BULK (TMA): one agent warp per CTA, which
@@ -892,6 +893,23 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
         CK(cudaStreamWaitEvent(s, c->ev_done, 0));
     } else {
+        if (lc.mech == PROACT_MECH_INLINE && c->world > 1 && armed) {
+            // PROACT-inline stores straight into the peers' replicas: like the agent (reading
+            // R6), it may only start once every destination finished reading them (phase e-1)
+            uint32_t peers = 0;
+            for (int r = 0; r < c->nregions; ++r)
+                if (armed >> r & 1) {
+                    const Region &R = c->regions[r];
+                    if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
+                    else peers |= (uint32_t)R.dest_mask;
+                }
+            peers &= ~(1u << c->rank);
+            if (peers) {
+                credit_wait_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, peers);
+                CK(cudaGetLastError());
+                c->launches++;
+            }
+        }
         lc.agent_ctas = (uint16_t)agent_ctas;
         unsigned total = agent_ctas + (grid ? grid : cap);
         if (total > cap) total = cap;
@@ -907,6 +925,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         Region &R = c->regions[r];
         R.gen_done += 1;
         R.gen_epoch = c->epoch;
+        R.gen_mech = (uint8_t)lc.mech;
         R.last_armed_epoch = c->epoch;
     }
     c->armed_epoch_mask |= armed;
