@@ -63,8 +63,14 @@ enum {
     PROACT_MECH_BULK = 2,    /* cudaMemcpy duplication after the kernel (L245): bulk-DMA baseline */
     PROACT_MECH_LOCAL = 3,   /* no transfer by the library: uninstrumented kernel; data moved by
                                 the caller (NCCL all-gather baseline) or G = 1 reference */
-    PROACT_MECH_ELIDE = 4    /* FUSED with the remote stores elided: tracking + agent only, the
+    PROACT_MECH_ELIDE = 4,   /* FUSED with the remote stores elided: tracking + agent only, the
                                 paper's overlap methodology (Sec. V-C); output NOT valid */
+    PROACT_MECH_DMA = 5      /* "hardware PROACT" emulation (Sec. III-D; SURVEY
+                                NEXT-3): producers tally as under FUSED, but the transfer agent is
+                                the copy engines: per chunk, a stream wait on counter == expected,
+                                one DMA copy per destination, a counter reset -- prepared by the
+                                host, triggered by the counters, no SM does any transfer.
+                                Consumers wait on phase credits.  Best with large chunks. */
 };
 
 /* ---- agent push instruction (a5) -------------------------------------------------------- */

@@ -208,7 +208,7 @@ __device__ __forceinline__ bool spin_step(const dev_ctx *C, uint64_t t0, uint32_
 /* ---------------------------------------------------------------- roles ------------------- */
 __device__ __forceinline__ bool uses_agent(const launch_ctx &lc)
 {
-    return lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE;
+    return lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE || lc.mech == PROACT_MECH_DMA;
 }
 __device__ __forceinline__ uint32_t producer_block(const launch_ctx &lc) { return blockIdx.x - lc.agent_ctas; }
 __device__ __forceinline__ uint32_t producer_grid(const launch_ctx &lc) { return gridDim.x - lc.agent_ctas; }
@@ -271,7 +271,7 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
     const uint32_t ex = R.expected[c];
     if (old + b > ex) {
         raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
-    } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE) {
+    } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA) {
         const uint32_t piece = piece_size(lc, R);
         const uint32_t P = (R.chunk_bytes + piece - 1) / piece;
         const uint32_t np = pieces_of(R, c, piece);

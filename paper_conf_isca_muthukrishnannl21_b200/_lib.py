@@ -20,9 +20,9 @@ MAX_REGIONS = 8
 OK = 0
 ERR_INVALID, ERR_CUDA, ERR_NOPEER, ERR_STATE, ERR_TIMEOUT, ERR_PROTOCOL, ERR_NOMEM = range(-1, -8, -1)
 
-MECH_FUSED, MECH_INLINE, MECH_BULK, MECH_LOCAL, MECH_ELIDE = range(5)
+MECH_FUSED, MECH_INLINE, MECH_BULK, MECH_LOCAL, MECH_ELIDE, MECH_DMA = range(6)
 MECH_NAMES = {MECH_FUSED: "fused", MECH_INLINE: "inline", MECH_BULK: "bulk",
-              MECH_LOCAL: "local", MECH_ELIDE: "elide"}
+              MECH_LOCAL: "local", MECH_ELIDE: "elide", MECH_DMA: "dma"}
 PUSH_VEC16, PUSH_BULK = 0, 1
 DISCOVER_QUEUE, DISCOVER_SCAN = 0, 1
 AGENT_FUSED, AGENT_SEPARATE = 0, 1

@@ -184,6 +184,9 @@ struct RankCtx {
     int latched = 0;
     cudaStream_t side = nullptr;      // high-priority stream of the SEPARATE agent kernel
     cudaEvent_t ev_start = nullptr, ev_done = nullptr;
+    static constexpr int NDMA = 2;    // MECH_DMA: copy streams (chunks dealt round-robin)
+    cudaStream_t dma[NDMA] = {nullptr, nullptr};
+    cudaEvent_t ev_dma[NDMA] = {nullptr, nullptr};
 };
 
 thread_local RankCtx *tl = nullptr;
@@ -232,7 +235,7 @@ void apply_env(proact_config &c) {
 }
 
 int validate_config(const proact_config &c) {
-    if (c.mech < 0 || c.mech > PROACT_MECH_ELIDE) return PROACT_ERR_INVALID;
+    if (c.mech < 0 || c.mech > PROACT_MECH_DMA) return PROACT_ERR_INVALID;
     if (c.push != PROACT_PUSH_VEC16 && c.push != PROACT_PUSH_BULK) return PROACT_ERR_INVALID;
     if (c.agent_warps < 1 || c.agent_warps > 1024) return PROACT_ERR_INVALID;
     if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
@@ -295,6 +298,24 @@ int map_peer(RankCtx *c, int p, const cudaIpcMemHandle_t &h, uint64_t raw_ptr_of
 // Driver entry point resolved through the runtime, so libproact does not link libcuda.so.1 and
 // still loads (for symbol checks) on a machine without a GPU driver.
 typedef CUresult (*pfn_getrange)(CUdeviceptr *, size_t *, CUdeviceptr);
+typedef CUresult (*pfn_waitvalue)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*pfn_writevalue)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+
+pfn_waitvalue g_wait32 = nullptr;
+pfn_writevalue g_write32 = nullptr;
+
+int load_memops()
+{
+    if (g_wait32 && g_write32) return PROACT_OK;
+    void *f1 = nullptr, *f2 = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &f1, cudaEnableDefault, &q) != cudaSuccess || !f1 ||
+        cudaGetDriverEntryPoint("cuStreamWriteValue32", &f2, cudaEnableDefault, &q) != cudaSuccess || !f2)
+        return PROACT_ERR_CUDA;
+    g_wait32 = (pfn_waitvalue)f1;
+    g_write32 = (pfn_writevalue)f2;
+    return PROACT_OK;
+}
 
 int alloc_base_and_handle(void *ptr, cudaIpcMemHandle_t *h, uint64_t *off, int *ok) {
     CUdeviceptr base = 0;
@@ -578,6 +599,10 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         if (cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         if (cudaEventCreateWithFlags(&c->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         if (cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        for (int k = 0; k < RankCtx::NDMA; ++k) {
+            if (cudaStreamCreateWithPriority(&c->dma[k], cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+            if (cudaEventCreateWithFlags(&c->ev_dma[k], cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        }
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM) !=
             cudaSuccess)
             return fail(PROACT_ERR_CUDA);
@@ -797,7 +822,7 @@ int proact_launch_tallies(void)
     if (!c) return 0;
     const int m = c->cfg.mech;
     if (m == PROACT_MECH_ELIDE) return 1;
-    return m == PROACT_MECH_FUSED && c->world > 1;
+    return (m == PROACT_MECH_FUSED || m == PROACT_MECH_DMA) && c->world > 1;
 }
 
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
@@ -830,7 +855,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     lc.armed = armed;
     // a single rank has nothing to send or receive: no tracking is needed at all, the fused
     // launch degenerates to the plain kernel (ELIDE keeps the agent: it measures tracking).
-    if (cfg.mech == PROACT_MECH_FUSED && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
+    if ((cfg.mech == PROACT_MECH_FUSED || cfg.mech == PROACT_MECH_DMA) && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
     for (int r = 0; r < c->nregions; ++r) {
         const Region &R = c->regions[r];
         lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
@@ -892,6 +917,60 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         *(launch_ctx *)args[0] = lc;
         CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
         CK(cudaStreamWaitEvent(s, c->ev_done, 0));
+    } else if (lc.mech == PROACT_MECH_DMA && armed) {
+        // NEXT-3 "hardware PROACT": the copy engines are the transfer agent.  Per owned chunk,
+        // on a DMA stream: wait counter[c] == expected[c] (the producers' last tally), copy the
+        // chunk to every destination, reset the counter.  Before the first copy into peer p,
+        // wait for p's credit (it finished phase e-1, reading R6).  Prepared by the host like
+        // the paper's "descriptors for the geometry of each transfer prepared in advance" (L166).
+        int rc = load_memops();
+        if (rc) return rc;
+        lc.agent_ctas = 0;
+        *(launch_ctx *)args[0] = lc;
+        CK(cudaEventRecord(c->ev_start, s));
+        uint32_t peers = 0;
+        for (int r = 0; r < c->nregions; ++r)
+            if (armed >> r & 1) {
+                const Region &R = c->regions[r];
+                if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
+                else peers |= (uint32_t)R.dest_mask;
+            }
+        peers &= ~(1u << c->rank);
+        for (int k = 0; k < RankCtx::NDMA; ++k) {
+            cudaStream_t d = c->dma[k];
+            CK(cudaStreamWaitEvent(d, c->ev_start, 0));
+            for (int p = 0; p < c->world; ++p)
+                if (peers >> p & 1)
+                    if (g_wait32((CUstream)d, (CUdeviceptr)(c->h.done + p), c->epoch << 1, CU_STREAM_WAIT_VALUE_GEQ) !=
+                        CUDA_SUCCESS)
+                        return PROACT_ERR_CUDA;
+        }
+        uint32_t rr = 0;
+        for (int r = 0; r < c->nregions; ++r) {
+            if (!(armed >> r & 1)) continue;
+            const Region &R = c->regions[r];
+            const region_dev &D = c->h.region[r];
+            for (uint32_t k = 0; k < R.n_own; ++k) {
+                cudaStream_t d = c->dma[rr++ % RankCtx::NDMA];
+                const uint64_t lo = R.own_off + (uint64_t)k * R.chunk;
+                const uint64_t len = std::min<uint64_t>(R.chunk, R.own_bytes - (uint64_t)k * R.chunk);
+                if (g_wait32((CUstream)d, (CUdeviceptr)(D.counter + k), (cuuint32_t)len, CU_STREAM_WAIT_VALUE_EQ) !=
+                    CUDA_SUCCESS)
+                    return PROACT_ERR_CUDA;
+                const uint32_t m = R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k];
+                for (int p = 0; p < c->world; ++p)
+                    if (p != c->rank && (m >> p & 1))
+                        CK(cudaMemcpyAsync(D.peer_base[p] + lo, R.base + lo, len, cudaMemcpyDeviceToDevice, d));
+                if (g_write32((CUstream)d, (CUdeviceptr)(D.counter + k), 0, 0) != CUDA_SUCCESS) return PROACT_ERR_CUDA;
+            }
+        }
+        unsigned total = grid ? grid : cap;
+        if (total > cap) total = cap;
+        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+        for (int k = 0; k < RankCtx::NDMA; ++k) {
+            CK(cudaEventRecord(c->ev_dma[k], c->dma[k]));
+            CK(cudaStreamWaitEvent(s, c->ev_dma[k], 0));
+        }
     } else {
         if (lc.mech == PROACT_MECH_INLINE && c->world > 1 && armed) {
             // PROACT-inline stores straight into the peers' replicas: like the agent (reading
@@ -1026,6 +1105,10 @@ int proact_finalize(void)
     cudaFree(c->meta);
     cudaFreeHost(c->h_err);
     if (c->side) cudaStreamDestroy(c->side);
+    for (int k = 0; k < RankCtx::NDMA; ++k) {
+        if (c->dma[k]) cudaStreamDestroy(c->dma[k]);
+        if (c->ev_dma[k]) cudaEventDestroy(c->ev_dma[k]);
+    }
     if (c->ev_start) cudaEventDestroy(c->ev_start);
     if (c->ev_done) cudaEventDestroy(c->ev_done);
     c->shm.close(true);

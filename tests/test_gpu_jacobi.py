@@ -39,7 +39,7 @@ def _run_jacobi(r, G, N, iters, chunk, mech, halo_only=False, rpt=16, check_deli
     return J.current.cpu().numpy(), (J.r0, J.r1), deliv
 
 
-@pytest.mark.parametrize("mech", [_lib.MECH_FUSED, _lib.MECH_INLINE, _lib.MECH_BULK])
+@pytest.mark.parametrize("mech", [_lib.MECH_FUSED, _lib.MECH_INLINE, _lib.MECH_BULK, _lib.MECH_DMA])
 def test_config1_jacobi_1024_two_ranks_bit_exact(mech):
     """BASELINE.json config 1: 1024x1024 fp32, 2 row partitions, 10 iterations, full replica."""
     N, iters = 1024, 10
@@ -67,6 +67,27 @@ def test_config1_jacobi_agent_variants(cfg):
     outs = run_ranks(2, _run_jacobi, N, iters, 64 * 1024, _lib.MECH_FUSED, **cfg)
     for g, (rep, _, _) in enumerate(outs):
         assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), (g, cfg)
+
+
+def test_jacobi_mixed_mechanisms_across_phases():
+    """Consumers wait according to the mechanism that produced the generation they read."""
+    N, G = 768, 3
+    seq = [_lib.MECH_FUSED, _lib.MECH_INLINE, _lib.MECH_DMA, _lib.MECH_BULK, _lib.MECH_FUSED, _lib.MECH_DMA,
+           _lib.MECH_INLINE, _lib.MECH_FUSED]
+    want = oracle.jacobi(synth.jacobi_init(N), len(seq))
+
+    def body(r, G):
+        J = wl.Jacobi(N, 8192, x0=torch.from_numpy(synth.jacobi_init(N)).cuda())
+        s = torch.cuda.Stream()
+        for k, m in enumerate(seq):
+            rt.set_config(mech=m)
+            J.step(s, barrier=(k == len(seq) - 1))
+        s.synchronize()
+        rt.check_device()
+        return J.current.cpu().numpy()
+
+    for g, rep in enumerate(run_ranks(G, body)):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), g
 
 
 def test_jacobi_halo_only_owned_rows_and_halos():

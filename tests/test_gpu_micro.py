@@ -44,6 +44,8 @@ def _run_micro(r, G, words, chunk, mech, phases, K, scattered, piece=None, warps
     (4, 3_000_000, 1 << 20, _lib.MECH_FUSED, False, 65536),
     (3, 777_776, 12288, _lib.MECH_INLINE, True, None),
     (4, 1 << 21, 4 << 20, _lib.MECH_BULK, False, None),
+    (3, 3 << 20, 1 << 20, _lib.MECH_DMA, False, None),
+    (2, 1 << 20, 65536, _lib.MECH_DMA, True, None),
     (1, 1 << 20, 4096, _lib.MECH_FUSED, False, None),
 ])
 def test_micro_replicas_equal_closed_form(G, words, chunk, mech, scattered, piece):

@@ -32,7 +32,7 @@ from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt  # noqa: E402
 from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl  # noqa: E402
 
 MECHS = [("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE), ("fused", _lib.MECH_FUSED),
-         ("inline", _lib.MECH_INLINE), ("bulk", _lib.MECH_BULK)]
+         ("inline", _lib.MECH_INLINE), ("bulk", _lib.MECH_BULK), ("dma", _lib.MECH_DMA)]
 
 
 def body(r, G, args):
@@ -80,6 +80,7 @@ def main():
             "infinite_bw_ms": T["bulk"] - t_copy, "copy_ms": t_copy,
             "transfer_overlap": 1.0 - (T["fused"] - T["elide"]) / t_copy,
             "speedup_fused_vs_bulk": T["bulk"] / T["fused"], "speedup_fused_vs_inline": T["inline"] / T["fused"],
+            "speedup_dma_vs_bulk": T["bulk"] / T["dma"],
             "opportunity_captured": (T["bulk"] - t_copy) / T["fused"]}
     print(json.dumps(line), flush=True)
 
