@@ -33,7 +33,20 @@ namespace {
 constexpr int GB = 256;            // threads per CTA
 constexpr int GT = 1024;           // vertices per tile (4 KiB of output, the paper's L279)
 constexpr int GL = 8;              // lanes per light vertex
-constexpr int RUN = 8;             // consecutive in-edges per thread per round (merge path)
+// consecutive in-edges per thread per round (merge path) and CTAs per SM, measured on B200
+// (tools/sweep_graph.py): PageRank 4 / 8 (1.65 ms at RMAT-24; 8 / 6: 2.2 ms), SSSP 2 / 6
+#ifndef PROACT_PR_RUN
+#define PROACT_PR_RUN 4
+#endif
+#ifndef PROACT_PR_MINB
+#define PROACT_PR_MINB 8
+#endif
+#ifndef PROACT_SSSP_RUN
+#define PROACT_SSSP_RUN 2
+#endif
+#ifndef PROACT_SSSP_MINB
+#define PROACT_SSSP_MINB 6
+#endif
 constexpr uint32_t SPLIT = 32768;  // max in-edges per work item: bigger tiles are split
 
 // Work item = (vertex tile, in-edge sub-range).  Tiles whose in-edges exceed SPLIT (hubs) are
@@ -248,8 +261,12 @@ __device__ __forceinline__ uint32_t ld_nc_u(const uint32_t *p)
 __device__ __forceinline__ void pr_finish(const launch_ctx &lc, const PrParams &p, uint32_t v, double s)
 {
     const float r = (float)(p.base + p.d * s);
-    p.g.r_own[v - p.g.v0] = r;
-    const uint32_t od = p.g.outdeg[v];
+    {   // r' is only read back at the end: keep it out of the L2 working set
+        const uint64_t pf = pol_first();
+        asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" ::"l"(p.g.r_own + (v - p.g.v0)), "f"(r), "l"(pf)
+                     : "memory");
+    }
+    const uint32_t od = ld_stream_u(p.g.outdeg + v, pol_first());
     const float c = od ? __fdiv_rn(r, (float)od) : 0.f;
     proact::put(lc, p.region_out, (uint64_t)v * 4, c);
 }
@@ -286,7 +303,8 @@ __device__ __forceinline__ uint32_t load_tile(const GraphDev &g, uint32_t tile, 
 {
     lo = g.v0 + tile * GT;
     const uint32_t hi = min(lo + GT, g.v0 + g.nv), nvt = hi - lo;
-    for (uint32_t i = threadIdx.x; i <= nvt; i += GB) cp[i] = g.colptr[lo - g.v0 + i];
+    const uint64_t pf = pol_first();
+    for (uint32_t i = threadIdx.x; i <= nvt; i += GB) cp[i] = ld_stream_u(g.colptr + (lo - g.v0 + i), pf);
     return nvt;
 }
 
@@ -313,14 +331,15 @@ __device__ __forceinline__ bool split_arrive(const GraphDev &g, const Item &it, 
 constexpr double FIX = 4611686018427387904.0;          // 2^62
 constexpr double UNFIX = 1.0 / 4611686018427387904.0;  // 2^-62
 
-__global__ void __launch_bounds__(GB, 6) pagerank_kernel(launch_ctx lc, PrParams p)
+__global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx lc, PrParams p)
 {
+    constexpr int RUN = PROACT_PR_RUN;
     if (proact::agent_dispatch(lc)) return;
     __shared__ uint32_t acc_lo[GT], acc_hi[GT];   // 64-bit fixed point as two native 32-bit halves
     __shared__ uint32_t cp[GT + 1];
     __shared__ uint32_t last;
     const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
-    const uint64_t pl = pol_last();
+    const uint64_t pl = pol_last(), pf = pol_first();
     // 64-bit shared-memory atomicAdd is a CAS loop on sm_100; two 32-bit adds + carry are native
     auto acc_add = [&](uint32_t i, unsigned long long x) {
         const uint32_t xl = (uint32_t)x, old = atomicAdd(&acc_lo[i], xl);
@@ -347,7 +366,7 @@ __global__ void __launch_bounds__(GB, 6) pagerank_kernel(launch_ctx lc, PrParams
                 float g[RUN];
 #pragma unroll
                 for (int q = 0; q < RUN; ++q)
-                    g[q] = r0 + q < r1 ? ld_gather_f(cin + ld_nc_u(p.g.rowidx + r0 + q), pl) : 0.f;
+                    g[q] = r0 + q < r1 ? ld_gather_f(cin + ld_stream_u(p.g.rowidx + r0 + q, pf), pl) : 0.f;
                 uint32_t i = vertex_of(cp, nvt, r0);
                 uint32_t nxt = cp[i + 1];
                 unsigned long long sum = 0ull;
@@ -395,8 +414,9 @@ constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory 
 
 // SSSP: merge-path over the item's in-edges; a source is relaxed only if its chunk changed in
 // the previous round (bitmap snapshot); per-vertex minima via shared-memory atomicMin.
-__global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p)
+__global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx lc, SsspParams p)
 {
+    constexpr int RUN = PROACT_SSSP_RUN;
     if (proact::agent_dispatch(lc)) return;
     __shared__ int32_t acc[GT];
     __shared__ uint32_t cp[GT + 1];
@@ -444,7 +464,7 @@ __global__ void __launch_bounds__(GB, 6) sssp_kernel(launch_ctx lc, SsspParams p
                 for (int q = 0; q < RUN; ++q) {
                     c[q] = INT32_MAX;
                     if (r0 + q < r1) {
-                        const uint32_t u = ld_nc_u(p.g.rowidx + r0 + q);
+                        const uint32_t u = ld_stream_u(p.g.rowidx + r0 + q, pf);
                         const uint32_t g = cdiv ? u / cdiv : u >> cshift;
                         if (p.first || (chg[g >> 5] >> (g & 31) & 1u)) {
                             const int32_t du = ld_gather_i(din + u, pl);
