@@ -262,8 +262,10 @@ typedef double (*proact_run_fn)(const proact_config *cfg, void *user);
 /* COLLECTIVE.  Brute-force sweep (Sec. III-A): mechanism x piece/chunk x
  * agent warps, per `key`; each point's time is the max over ranks; best config returned in
  * *out and cached as JSON in $PROACT_TUNE_CACHE (default ./proact_tune.json) under `key` --
- * a cached key is returned without re-running.  `space` may be NULL (default space) or a
- * NUL-terminated list "mech=0,1;warps=4,8;piece=16384,65536". */
+ * a cached key is returned without re-running.  `space` may be NULL (default space: mechanisms
+ * FUSED/INLINE/BULK x agent warps 8..64 at the current chunk, piece, push, discovery and agent
+ * placement) or a NUL-terminated list such as
+ * "mech=0,1,2,5;chunk=65536,1048576;warps=8,32;piece=65536;push=0,1;disc=0,1;akern=0,1". */
 int proact_autotune(const char *key, const char *space, proact_run_fn fn, void *user,
                     proact_config *out);
 

@@ -1197,6 +1197,9 @@ static bool cache_lookup(const std::string &key, proact_config *out)
     out->agent_warps = (int)get("agent_warps", out->agent_warps);
     out->piece_bytes = (uint32_t)get("piece_bytes", out->piece_bytes);
     out->chunk_bytes = (uint32_t)get("chunk_bytes", out->chunk_bytes);
+    out->push = (int)get("push", out->push);
+    out->discovery = (int)get("discovery", out->discovery);
+    out->agent_kernel = (int)get("agent_kernel", out->agent_kernel);
     return true;
 }
 
@@ -1226,8 +1229,9 @@ static void cache_store(const std::string &key, const proact_config &c, double m
     while (!body.empty() && (body.back() == '\n' || body.back() == ' ' || body.back() == ',')) body.pop_back();
     char ent[512];
     snprintf(ent, sizeof ent,
-             "  \"%s\": {\"mech\":%d,\"agent_warps\":%d,\"piece_bytes\":%u,\"chunk_bytes\":%u,\"ms\":%.6f}",
-             key.c_str(), c.mech, c.agent_warps, c.piece_bytes, c.chunk_bytes, ms);
+             "  \"%s\": {\"mech\":%d,\"agent_warps\":%d,\"piece_bytes\":%u,\"chunk_bytes\":%u,"
+             "\"push\":%d,\"discovery\":%d,\"agent_kernel\":%d,\"ms\":%.6f}",
+             key.c_str(), c.mech, c.agent_warps, c.piece_bytes, c.chunk_bytes, c.push, c.discovery, c.agent_kernel, ms);
     std::string out = "{\n" + body + (body.empty() ? "" : ",\n") + ent + "\n}\n";
     std::string tmp = path + ".tmp";
     if (FILE *f = fopen(tmp.c_str(), "w")) {
@@ -1272,35 +1276,48 @@ int proact_autotune(const char *key, const char *space, proact_run_fn fn, void *
         return PROACT_OK;
     }
     std::string sp = space ? space : "";
-    // Sec. III-A: mechanism x granularity x transfer threads (Table II ranges 4kB-16MB, 32-8192)
-    auto mechs = parse_list(sp, "mech", {PROACT_MECH_FUSED, PROACT_MECH_INLINE});
+    // Sec. III-A: mechanism x granularity x transfer threads (Table II ranges 4kB-16MB, 32-8192),
+    // plus the B200 agent axes: push instruction, discovery, agent placement
+    auto mechs = parse_list(sp, "mech", {PROACT_MECH_FUSED, PROACT_MECH_INLINE, PROACT_MECH_BULK});
     auto chunks = parse_list(sp, "chunk", {(long long)c->cfg.chunk_bytes});
-    auto warps = parse_list(sp, "warps", {4, 8, 16, 32, 64});
+    auto warps = parse_list(sp, "warps", {8, 16, 32, 64});
     auto pieces = parse_list(sp, "piece", {(long long)c->cfg.piece_bytes});
+    auto pushes = parse_list(sp, "push", {(long long)c->cfg.push});
+    auto discs = parse_list(sp, "disc", {(long long)c->cfg.discovery});
+    auto akerns = parse_list(sp, "akern", {(long long)c->cfg.agent_kernel});
     proact_config base = c->cfg, best = base;
     double best_ms = 1e300;
     for (long long m : mechs)
         for (long long ch : chunks)
             for (long long w : warps)
-                for (long long pc : pieces) {
-                    bool agent = m == PROACT_MECH_FUSED || m == PROACT_MECH_ELIDE;
-                    // non-agent mechanisms ignore warps/piece: run them once
-                    if (!agent && (w != warps[0] || pc != pieces[0])) continue;
-                    proact_config t = base;
-                    t.mech = (int)m;
-                    t.chunk_bytes = (uint32_t)ch;
-                    t.agent_warps = (int)w;
-                    t.piece_bytes = (uint32_t)pc;
-                    double ms = -1.0;
-                    if (validate_config(t) == PROACT_OK && proact_set_config(&t) == PROACT_OK) ms = fn(&t, user);
-                    std::vector<double> all(c->world);
-                    rc = c->shm.allgather(c->rank, &ms, sizeof(ms), all.data());
-                    if (rc) { proact_set_config(&base); return rc; }
-                    double worst = 0;
-                    bool ok = true;
-                    for (double x : all) { if (x < 0) ok = false; worst = std::max(worst, x); }
-                    if (ok && worst < best_ms) { best_ms = worst; best = t; }
-                }
+                for (long long pc : pieces)
+                    for (long long pu : pushes)
+                        for (long long di : discs)
+                            for (long long ak : akerns) {
+                                bool agent = m == PROACT_MECH_FUSED || m == PROACT_MECH_ELIDE;
+                                // non-agent mechanisms ignore the agent axes: run them once
+                                if (!agent && (w != warps[0] || pc != pieces[0] || pu != pushes[0] ||
+                                               di != discs[0] || ak != akerns[0]))
+                                    continue;
+                                proact_config t = base;
+                                t.mech = (int)m;
+                                t.chunk_bytes = (uint32_t)ch;
+                                t.agent_warps = (int)w;
+                                t.piece_bytes = (uint32_t)pc;
+                                t.push = (int)pu;
+                                t.discovery = (int)di;
+                                t.agent_kernel = (int)ak;
+                                double ms = -1.0;
+                                if (validate_config(t) == PROACT_OK && proact_set_config(&t) == PROACT_OK)
+                                    ms = fn(&t, user);
+                                std::vector<double> all(c->world);
+                                rc = c->shm.allgather(c->rank, &ms, sizeof(ms), all.data());
+                                if (rc) { proact_set_config(&base); return rc; }
+                                double worst = 0;
+                                bool ok = true;
+                                for (double x : all) { if (x < 0) ok = false; worst = std::max(worst, x); }
+                                if (ok && worst < best_ms) { best_ms = worst; best = t; }
+                            }
     proact_set_config(&base);
     if (best_ms >= 1e300) return PROACT_ERR_INVALID;
     if (c->rank == 0) cache_store(key, best, best_ms);
