@@ -928,6 +928,12 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         lc.agent_ctas = 0;
         *(launch_ctx *)args[0] = lc;
         CK(cudaEventRecord(c->ev_start, s));
+        // the producer goes first: the DMA streams may hold more waits than a command queue
+        // can buffer, and enqueueing them must never block the launch that satisfies them
+        unsigned total = grid ? grid : cap;
+        if (total > cap) total = cap;
+        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+
         uint32_t peers = 0;
         for (int r = 0; r < c->nregions; ++r)
             if (armed >> r & 1) {
@@ -964,9 +970,6 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
                 if (g_write32((CUstream)d, (CUdeviceptr)(D.counter + k), 0, 0) != CUDA_SUCCESS) return PROACT_ERR_CUDA;
             }
         }
-        unsigned total = grid ? grid : cap;
-        if (total > cap) total = cap;
-        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
         for (int k = 0; k < RankCtx::NDMA; ++k) {
             CK(cudaEventRecord(c->ev_dma[k], c->dma[k]));
             CK(cudaStreamWaitEvent(s, c->ev_dma[k], 0));
