@@ -117,3 +117,18 @@ def test_config4_sssp_full_size():
     (rounds, d, _, _), = outs
     assert rounds == want_rounds
     assert np.array_equal(d, want)
+
+
+def test_graph_without_edges():
+    """E = 0: PageRank gives (1-d)/V everywhere, SSSP converges in one round."""
+    V = 8192
+    src = np.zeros(0, np.uint32)
+    dst = np.zeros(0, np.uint32)
+    outs = run_ranks(2, _pr_body, V, src, dst, 3, 4096, _lib.MECH_FUSED)
+    want = oracle.pagerank(V, src, dst, 3).astype(np.float64)
+    for v0, v1, r in outs:
+        assert np.allclose(r, want[v0:v1], rtol=1e-6)
+    outs = run_ranks(2, _sssp_body, V, src, dst, np.zeros(0, np.int32), 5, 4096, _lib.MECH_FUSED)
+    d_want, rounds_want, _ = oracle.sssp(V, src, dst, np.zeros(0, np.int32), 5)
+    for rounds, d, _, _ in outs:
+        assert rounds == rounds_want and np.array_equal(d, d_want)

@@ -165,3 +165,14 @@ def test_jacobi_e2e_host_buffers():
     for rows, (r0, r1), h2d, d2h in outs:
         assert np.array_equal(rows, want[r0:r1])
         assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
+
+
+@pytest.mark.parametrize("G,N,chunk", [(1, 4, 4096), (2, 8, 4096), (2, 1024, 4112), (3, 36, 4096)])
+def test_jacobi_degenerate_and_odd_chunks(G, N, chunk):
+    """All-boundary grids (N = 4: every cell copied through), ranks owning a couple of rows,
+    a chunk size that is not a multiple of the 4 KiB row segment (spans straddle chunks)."""
+    iters = 3
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(G, _run_jacobi, N, iters, chunk, _lib.MECH_FUSED)
+    for g, (rep, _, _) in enumerate(outs):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), g

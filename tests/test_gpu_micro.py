@@ -119,3 +119,14 @@ def test_watchdog_turns_a_stall_into_timeout():
 
     res = run_ranks(2, body)
     assert res[0] == _lib.ERR_TIMEOUT
+
+
+def test_micro_ranks_with_empty_slices():
+    """A region smaller than the world: some ranks own zero bytes (no chunks) but still take
+    part in every collective and phase."""
+    words, G = 8, 4   # slices of 0 / 4 / 0 / 4 words
+    outs = run_ranks(G, _run_micro, words, 4096, _lib.MECH_FUSED, 2, 1, False)
+    for p in range(2):
+        want = oracle.micro_phase(words, p, SEED, 1)
+        for g in range(G):
+            assert np.array_equal(outs[g][p], want), (p, g)
