@@ -568,7 +568,7 @@ extern "C" {
 int proact_graph_partition(const uint32_t *d_dst, unsigned long long E, unsigned V, int G, unsigned align,
                            unsigned *bounds, void *stream)
 {
-    if (!d_dst || !bounds || G < 1 || align == 0 || V == 0) return PROACT_ERR_INVALID;
+    if ((!d_dst && E) || !bounds || G < 1 || align == 0 || V == 0) return PROACT_ERR_INVALID;
     cudaStream_t s = (cudaStream_t)stream;
     uint32_t *indeg = nullptr;
     GCK(cudaMalloc((void **)&indeg, 4 * (size_t)V));
@@ -604,7 +604,7 @@ int proact_partition_bounds(const uint32_t *indeg, unsigned V, int G, unsigned a
 int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w, unsigned long long E,
                        unsigned V, unsigned v0, unsigned v1, void *stream)
 {
-    if (!d_src || !d_dst || v1 < v0 || v1 > V) return PROACT_ERR_INVALID;
+    if (((!d_src || !d_dst) && E) || v1 < v0 || v1 > V) return PROACT_ERR_INVALID;
     int id = -1;
     for (int k = 0; k < MAXGRAPH; ++k)
         if (!graphs[k].used) { id = k; break; }
@@ -754,7 +754,7 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     SsspParams p;
     int rc = graph_dev(graph, &p.g);
     if (rc) return rc;
-    if (!p.g.w) return PROACT_ERR_INVALID;
+    if (!p.g.w && graphs[graph].E_own) return PROACT_ERR_INVALID;   // built without weights
     proact_region_info ro;
     rc = proact_region_info_get(region_out, &ro);
     if (rc) return rc;
