@@ -24,15 +24,17 @@ mechs = os.environ.get("MECHS", "local,fused,elide").split(",")
 warps = [int(x) for x in os.environ.get("WARPS", "1,4,16").split(",")]
 rpts = [int(x) for x in os.environ.get("RPTS", "16,64").split(",")]
 discs = [int(x) for x in os.environ.get("DISCS", "0").split(",")]
+akerns = [int(x) for x in os.environ.get("AKERNS", "1").split(",")]   # 0 FUSED, 1 SEPARATE
 res = []
 for ch in chunks:
     if ch != rt.region_info(J.rid[0]).chunk_bytes:
         rt.rechunk(J.rid[0], ch)
         rt.rechunk(J.rid[1], ch)
-    for mech, w, rpt, disc in itertools.product(mechs, warps, rpts, discs):
-        if mech == "local" and (w != warps[0] or disc != discs[0]):
+    for mech, w, rpt, disc, ak in itertools.product(mechs, warps, rpts, discs, akerns):
+        if mech == "local" and (w != warps[0] or disc != discs[0] or ak != akerns[0]):
             continue
-        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[mech], agent_warps=w, discovery=disc)
+        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[mech], agent_warps=w, discovery=disc,
+                      agent_kernel=ak)
         J.rpt = rpt
         evs = []
         for k in range(24):
@@ -47,7 +49,7 @@ for ch in chunks:
         torch.cuda.synchronize()
         t = [a.elapsed_time(b) for a, b in evs[4:]]
         ms = statistics.median(t)
-        r = {"chunk": ch, "mech": mech, "warps": w, "rpt": rpt, "disc": disc, "ms": ms, "GBps": 8.0 * N * N / ms / 1e6}
+        r = {"chunk": ch, "mech": mech, "warps": w, "rpt": rpt, "disc": disc, "akern": ak, "ms": ms, "GBps": 8.0 * N * N / ms / 1e6}
         res.append(r)
         print(json.dumps(r), flush=True)
 rt.check_device()
