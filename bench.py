@@ -32,6 +32,10 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+# before torch touches CUDA: the agent kernel runs on its own high-priority stream, and with the
+# default 8 hardware connections its launches can queue behind the producer stream's work
+# (false dependencies: +100 us per phase measured, tools/probes/host_issue.py)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 METRIC = "strong-scaling speedup and iters/sec at 1/2/4/8 B200; NVLink GB/s vs 900 GB/s"
 N_GRID = 16384

@@ -83,6 +83,8 @@ struct dev_ctx {
     uint32_t *vote;                            /* [2] local vote words, by epoch parity */
     uint32_t *vote_host;                       /* host-mapped: (epoch+1)<<1 | global vote */
     unsigned long long *prof;                  /* PROACT_DEBUG=2: agent cycle accounting [8] */
+    uint32_t *resident;                        /* SEPARATE agent: CTAs that became resident
+                                                  (monotonic; the producer launch waits on it) */
     region_dev region[PROACT_MAX_REGIONS];
 };
 

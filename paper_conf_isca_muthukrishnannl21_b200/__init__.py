@@ -4,7 +4,14 @@ Paper: Muthukrishnan, Nellans, Lustig, Fessler, Wenisch, "Efficient Multi-GPU
 Shared Memory via Automatic Optimization of Fine-Grained Transfers", ISCA 2021.
 See DESIGN.md for the path, its boundary (include/*.h) and the readings taken.
 """
-from . import _lib
+import os as _os
+
+# The agent kernel runs on its own high-priority stream; with the default 8 hardware queues its
+# launches can wait behind the producer stream (false dependencies).  Effective only if this
+# package is imported before anything creates a CUDA context (bench.py sets it before torch).
+_os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
+from . import _lib  # noqa: E402
 from ._lib import (MECH_BULK, MECH_ELIDE, MECH_FUSED, MECH_INLINE, MECH_LOCAL, MECH_NAMES,
                    REGION_SPARSE, ProactError)
 from . import runtime

@@ -180,6 +180,8 @@ struct RankCtx {
     uint32_t bulk_mask = 0;           // regions launched with BULK in the current epoch
     int bulk_pending = 0;
     uint64_t launches = 0;
+    uint32_t resident_total = 0;      // agent CTAs launched so far (SEPARATE residency gate)
+    std::vector<const void *> carveout_set;   // producer kernels given the max smem carveout
     int last_cuda = 0;
     int latched = 0;
     cudaStream_t side = nullptr;      // high-priority stream of the SEPARATE agent kernel
@@ -492,7 +494,13 @@ __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t ma
 // staging ring: 8 x 16 KiB (+ metadata) for up to 32 agent CTAs, 8 x 8 KiB beyond (2 per SM)
 constexpr size_t AGENT_SMEM = 128 * 1024 + 1024;
 constexpr size_t AGENT_SMEM_SMALL = 64 * 1024 + 1024;
-__global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc) { proact::agent_loop(lc); }
+__global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc)
+{
+    // residency gate: the producer's stream waits until every agent CTA is resident, so the
+    // producer grid can never occupy the slots the agent needs (which would serialise them)
+    if (threadIdx.x == 0) atomicAdd(lc.ctx->resident, 1u);
+    proact::agent_loop(lc);
+}
 
 RankCtx *need_ctx() { return tl; }
 
@@ -545,7 +553,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     int coop_attr = 0;
     cudaDeviceGetAttribute(&coop_attr, cudaDevAttrCooperativeLaunch, c->device);
     // rank metadata block: done[MAXR] | err | vote[2]
-    size_t meta_bytes = 4 * MAXR + 64 + 64;
+    size_t meta_bytes = 4 * MAXR + 64 + 64 + 64;
     if (cudaMalloc((void **)&c->meta, meta_bytes) != cudaSuccess) return fail(PROACT_ERR_CUDA);
     cudaMemset(c->meta, 0, meta_bytes);
     if (cudaHostAlloc((void **)&c->h_err, 64, cudaHostAllocMapped) != cudaSuccess) return fail(PROACT_ERR_CUDA);
@@ -561,6 +569,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     c->h.done = (uint32_t *)c->meta;
     c->h.err = (uint32_t *)(c->meta + 4 * MAXR);
     c->h.vote = (uint32_t *)(c->meta + 4 * MAXR + 64);
+    c->h.resident = (uint32_t *)(c->meta + 4 * MAXR + 128);
     c->h.err_host = c->d_err_host;
     c->h.vote_host = c->d_vote_host;
     c->h.prof = nullptr;
@@ -605,6 +614,12 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         }
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM) !=
             cudaSuccess)
+            return fail(PROACT_ERR_CUDA);
+        // the L1/shared carveout is an SM-wide setting: an SM configured for a smaller carveout by
+        // the agent cannot host producer CTAs next to it (measured: 16 agent CTAs pushed 16
+        // producer CTAs into a second wave, +70% phase time).  Agent and producers use the max.
+        if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                 cudaSharedmemCarveoutMaxShared) != cudaSuccess)
             return fail(PROACT_ERR_CUDA);
     }
     rc = c->shm.barrier();
@@ -878,18 +893,35 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
     cudaStream_t s = (cudaStream_t)stream;
     if (separate) {
+        // producer kernels share SMs with the agent: same (maximal) shared-memory carveout
+        if (std::find(c->carveout_set.begin(), c->carveout_set.end(), kernel) == c->carveout_set.end()) {
+            CK(cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                    cudaSharedmemCarveoutMaxShared));
+            c->carveout_set.push_back(kernel);
+        }
         // the agent kernel first, on its own high-priority stream (ordered after my earlier
         // work), so its CTAs are resident before the producer grid fills the device; the
         // producer grid leaves one slot per agent CTA; my stream waits for the agent.
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
-        const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+        size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+        if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
+            asmem = std::min(AGENT_SMEM, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
         CK(cudaEventRecord(c->ev_start, s));
         CK(cudaStreamWaitEvent(c->side, c->ev_start, 0));
         agent_kernel<<<agent_ctas, agent_block, asmem, c->side>>>(la);
         CK(cudaGetLastError());
         CK(cudaEventRecord(c->ev_done, c->side));
         c->launches++;
+        // the producer launches only once every agent CTA is resident (wrap-safe GEQ)
+        c->resident_total += agent_ctas;
+        {
+            int mrc = load_memops();
+            if (mrc) return mrc;
+            if (g_wait32((CUstream)s, (CUdeviceptr)c->h.resident, c->resident_total, CU_STREAM_WAIT_VALUE_GEQ) !=
+                CUDA_SUCCESS)
+                return PROACT_ERR_CUDA;
+        }
         lc.agent_ctas = 0;
         // producer slots an agent CTA displaces on its SM (shared memory / registers / threads)
         unsigned lost = 1;

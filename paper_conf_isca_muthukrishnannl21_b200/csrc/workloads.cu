@@ -172,6 +172,22 @@ __global__ void __launch_bounds__(JCfg<TALLY>::threads, JCfg<TALLY>::minb)
 jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 {
     if (proact::agent_dispatch(lc)) return;
+#ifdef PROACT_TIMING_EXP
+    unsigned long long *xprof = lc.ctx->prof;
+    const unsigned long long xt0 = proact::globaltimer();
+    if (xprof && threadIdx.x == 0) atomicMax(&xprof[2], ~xt0);
+    struct XEnd {
+        unsigned long long *p, t0;
+        __device__ ~XEnd() {
+            if (p) {
+                const unsigned long long t = proact::globaltimer();
+                atomicMax(&p[3], t);
+                atomicAdd(&p[4], t - t0);
+                atomicAdd(&p[5], 1ull);
+            }
+        }
+    } xend{(xprof && threadIdx.x == 0) ? xprof : nullptr, xt0};
+#endif
     extern __shared__ __align__(128) unsigned char jsm[];
     float *ring = reinterpret_cast<float *>(jsm);
     uint64_t *full = reinterpret_cast<uint64_t *>(jsm + (size_t)JS * SLOT * 4);

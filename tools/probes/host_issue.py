@@ -2,6 +2,7 @@
 import os
 import sys
 import time
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # before torch: see bench.py
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 import torch  # noqa: E402
