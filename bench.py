@@ -74,6 +74,8 @@ class Clocks:
         self.path = f"/tmp/proact_clocks_{os.getpid()}.csv"
 
     def __enter__(self):
+        if self.index < 0:   # sampling disabled (diagnostics only)
+            return self
         try:
             self.f = open(self.path, "w")
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
@@ -244,26 +246,31 @@ def main():
         for k in range(I):
             J.step(s, barrier=(k == I - 1))
 
+    per_step: list = []   # this rank's per-step times of the last timed() call (spread check)
+
     def timed(fn, K):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(s)
-        for _ in range(K):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(K + 1)]
+        ev[0].record(s)
+        for k in range(K):
             fn()
-        e1.record(s)
+            ev[k + 1].record(s)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        return max_over_ranks(e0.elapsed_time(e1), world)
+        per_step.clear()
+        per_step.extend(ev[k].elapsed_time(ev[k + 1]) for k in range(K))
+        return max_over_ranks(ev[0].elapsed_time(ev[K]), world)
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     l0 = rt.launch_count()
-    with Clocks(dev) as clk:
+    with Clocks(dev if os.environ.get("PROACT_BENCH_NO_CLOCKS") != "1" else -1) as clk:
         ms = timed(step, args.steps)
+    step_ms = list(per_step)
     launches = rt.launch_count() - l0
     rt.check_device()
     value = args.steps * I / (ms / 1000.0)
@@ -339,7 +346,8 @@ def main():
                            "agent_warps": cfg["agent_warps"], "piece_bytes": cfg["piece_bytes"],
                            "rows_per_tile": args.rpt, "replication": "full",
                            "l2": "inputs > L2 (two 1 GiB grids), no flush",
-                           "parallelism": f"rows{world}"},
+                           "parallelism": f"rows{world}",
+                           "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)]},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead}
         print(json.dumps(line), flush=True)

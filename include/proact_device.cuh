@@ -85,6 +85,8 @@ struct dev_ctx {
     unsigned long long *prof;                  /* PROACT_DEBUG=2: agent cycle accounting [8] */
     uint32_t *resident;                        /* SEPARATE agent: CTAs that became resident
                                                   (monotonic; the producer launch waits on it) */
+    uint32_t *sched;                           /* [2] producer work counter + finished claimers:
+                                                  dynamic tile scheduling (see claim_tile) */
     region_dev region[PROACT_MAX_REGIONS];
 };
 
@@ -250,6 +252,25 @@ __device__ __forceinline__ void put(const launch_ctx &lc, int r, uint64_t off, c
             *reinterpret_cast<T *>(R.peer_base[p] + off) = v;
         }
     }
+}
+
+/* Dynamic work distribution for persistent producers: the next tile index of this launch, or
+ * a value >= ntiles when none is left.  Call from ONE thread per CTA until it returns >= ntiles;
+ * that final call also counts the CTA out, and the last CTA out re-arms the counters for the next
+ * launch on this rank (stream order makes the reset visible to it).  Balances CTAs that share SMs
+ * with agents or run slower, instead of the static round-robin's straggler tail. */
+__device__ __forceinline__ uint32_t claim_tile(const launch_ctx &lc, uint32_t ntiles)
+{
+    uint32_t *S = lc.ctx->sched;
+    const uint32_t t = atomicAdd(&S[0], 1u);
+    if (t >= ntiles) {
+        const uint32_t P = gridDim.x - lc.agent_ctas;
+        if (atomicAdd(&S[1], 1u) + 1u == P) {
+            S[0] = 0u;
+            S[1] = 0u;
+        }
+    }
+    return t;
 }
 
 /* Pieces of my chunk c under piece size `piece` (agent work units). */

@@ -570,6 +570,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     c->h.err = (uint32_t *)(c->meta + 4 * MAXR);
     c->h.vote = (uint32_t *)(c->meta + 4 * MAXR + 64);
     c->h.resident = (uint32_t *)(c->meta + 4 * MAXR + 128);
+    c->h.sched = (uint32_t *)(c->meta + 4 * MAXR + 128 + 16);
     c->h.err_host = c->d_err_host;
     c->h.vote_host = c->d_vote_host;
     c->h.prof = nullptr;
@@ -1096,9 +1097,19 @@ int proact_phase_sync(void *stream, int mode)
             }
         }
     }
-    sync_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, mode);
-    CK(cudaGetLastError());
-    c->launches++;
+    if (c->world == 1 && mode == PROACT_SYNC_SIGNAL && !env_int("PROACT_SYNC_KERNEL", 0)) {
+        // a single rank has no peer to credit: two stream memory writes (my own credit, the
+        // vote word of this epoch cleared for epoch + 2) instead of a kernel launch
+        int mrc = load_memops();
+        if (mrc) return mrc;
+        if (g_write32((CUstream)s, (CUdeviceptr)c->h.done, (c->epoch + 1u) << 1, 0) != CUDA_SUCCESS ||
+            g_write32((CUstream)s, (CUdeviceptr)(c->h.vote + (c->epoch & 1u)), 0u, 0) != CUDA_SUCCESS)
+            return PROACT_ERR_CUDA;
+    } else {
+        sync_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, mode);
+        CK(cudaGetLastError());
+        c->launches++;
+    }
     c->epoch++;
     c->armed_epoch_mask = 0;
     c->bulk_mask = 0;

@@ -87,7 +87,8 @@ constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a r
 #endif
 constexpr int JS = PROACT_JACOBI_RING;  // ring depth (rows in flight per CTA)
 constexpr int SLOT = JW + 8;            // floats per slot: columns [c0-4, c0+JW+4)
-constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8 + 4 * 8;
+constexpr int JTD = 32;                 // tile-id ring (stream warp -> compute -> committer)
+constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8 + 4 * 8 + JTD * 4;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt)
@@ -141,21 +142,33 @@ __device__ __forceinline__ JTile jtile(int t, int nstrips, int nbands, int rb, i
     return T;
 }
 
-// Producer warp (one lane): the CTA's row stream, slot by slot.
+// Producer warp (one lane): the CTA's row stream, slot by slot.  Tiles are claimed dynamically
+// (proact::claim_tile); the claimed id goes to tids[k % JTD] before the tile's first row is
+// armed, so the mbarrier arrival (release) publishes it to the compute warps.  After the last
+// tile an end marker (-1, a tx-less arrival on the next slot) lets them exit.
 __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_jacobi_params &p, float *ring,
-                                           uint64_t *full, uint64_t *empty, int t_first, int P, int ntiles,
+                                           uint64_t *full, uint64_t *empty, int *tids, int ntiles,
                                            int nstrips, int nbands)
 {
     const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows), rb = p.rows_per_tile;
     const char *in = lc.ctx->region[p.region_in].base;
     uint32_t q = 0;
-    for (int t = t_first; t < ntiles; t += P) {
-        const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+    for (uint32_t kt = 0;; ++kt) {
+        const uint32_t t = proact::claim_tile(lc, (uint32_t)ntiles);
+        const uint32_t slot0 = q % JS;
+        if (q >= JS) mbar_wait(&empty[slot0], ((q / JS) - 1) & 1u);
+        if (t >= (uint32_t)ntiles) {
+            tids[kt % JTD] = -1;
+            mbar_arrive(&full[slot0]);
+            return;
+        }
+        tids[kt % JTD] = (int)t;
+        const JTile T = jtile((int)t, nstrips, nbands, rb, row0, rend, N);
         const int lo = T.c0 >= 4 ? T.c0 - 4 : 0, hi = min(T.c0 + JW + 4, N);
         const uint32_t bytes = (uint32_t)(hi - lo) * 4;
         for (int k = T.kfirst; k <= T.klast; ++k, ++q) {
             const uint32_t slot = q % JS;
-            if (q >= JS) mbar_wait(&empty[slot], ((q / JS) - 1) & 1u);
+            if (q >= JS && k != T.kfirst) mbar_wait(&empty[slot], ((q / JS) - 1) & 1u);
             const uint64_t goff = ((uint64_t)k * N + lo) * 4;
             if (k < row0 || k >= rend) {   // (a7) halo row produced by a peer: wait, then
                 proact::wait_range(lc, p.region_in, goff, bytes);
@@ -194,6 +207,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     uint64_t *empty = full + JS;
     uint64_t *tdone = empty + JS;    // [2] compute warps finished tile k (k & 1)
     uint64_t *cdone = tdone + 2;     // [2] committer finished tile k (k & 1)
+    int *tids = reinterpret_cast<int *>(cdone + 2);   // [JTD] claimed tile ids, by sequence
 #ifndef PROACT_JACOBI_RT_TALLY
 #define PROACT_JACOBI_RT_TALLY 1
 #endif
@@ -206,8 +220,6 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     const int nstrips = (N + JW - 1) / JW;
     const int nbands = ((int)p.nrows + rb - 1) / rb;
     const int ntiles = nbands * nstrips;
-    const int P = (int)proact::producer_grid(lc);
-    const int t_first = (int)proact::producer_block(lc);
     if (tid == 0) {
         for (int s = 0; s < JS; ++s) {
             mbar_init(&full[s], 1);
@@ -221,7 +233,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     }
     __syncthreads();
     if (warp == JC) {
-        if (lane == 0) jacobi_stream(lc, p, ring, full, empty, t_first, P, ntiles, nstrips, nbands);
+        if (lane == 0) jacobi_stream(lc, p, ring, full, empty, tids, ntiles, nstrips, nbands);
         return;
     }
     if (TALLY && warp == JC + 1) {
@@ -229,10 +241,11 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
         // acquire at CTA scope), commit the tile's rows with release RMWs, merged per chunk.
         // The compute warps never stall on the commit's fence latency.
         if (!tally) return;
-        uint32_t k = 0;
-        for (int t = t_first; t < ntiles; t += P, ++k) {
-            const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+        for (uint32_t k = 0;; ++k) {
             mbar_wait(&tdone[k & 1u], (k >> 1) & 1u);
+            const int t = tids[k % JTD];   // written by the stream warp, ordered by the tile's
+            if (t < 0) return;             // row barriers and the compute warps' tdone arrival
+            const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
             for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
                 const int i = k0 + lane;
                 warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4, (uint32_t)(T.c1 - T.c0) * 4);
@@ -245,7 +258,14 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     char *outb = lc.ctx->region[p.region_out].base;
     uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
     uint32_t kt = 0;   // tiles handed to the committer
-    for (int t = t_first; t < ntiles; t += P) {
+    for (;;) {
+        // the next tile's first stream item carries its id (or the end marker)
+        mbar_wait(&full[q % JS], (q / JS) & 1u);
+        const int t = tids[kt % JTD];
+        if (t < 0) {
+            if (tally && TALLY && lane == 0) mbar_arrive(&tdone[kt & 1u]);   // release the committer
+            break;
+        }
         const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
         const int x = 4 * tid, j = T.c0 + x;
         const bool act = j < T.c1;
@@ -305,7 +325,10 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             if (lane == 0) mbar_arrive(&tdone[kt & 1u]);
             ++kt;
             if (kt >= 2) mbar_wait(&cdone[kt & 1u], ((kt - 2) >> 1) & 1u);
-        } else if (tally) {   // no committer warp: compute warps meet, warp 0 commits
+            continue;
+        }
+        ++kt;
+        if (tally) {   // no committer warp: compute warps meet, warp 0 commits
             asm volatile("bar.sync 1, %0;" ::"r"(JC * 32) : "memory");
             if (warp == 0)
                 for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
