@@ -771,4 +771,16 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     return proact_launch(regs, 1, (const void *)sssp_kernel, 0, GB, args, 0, stream);
 }
 
+// Force-load this translation unit's kernels (see proact_internal_preload_workloads).
+__attribute__((visibility("hidden"))) int proact_internal_preload_graph(void)
+{
+    cudaFuncAttributes a;
+    const void *k[] = {(const void *)count_kernel, (const void *)scan_blocks, (const void *)scan_totals,
+                       (const void *)scan_add, (const void *)scatter_kernel, (const void *)pagerank_kernel,
+                       (const void *)sssp_kernel, (const void *)pr_init_kernel};
+    for (const void *f : k)
+        if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
+    return PROACT_OK;
+}
+
 }  // extern "C"

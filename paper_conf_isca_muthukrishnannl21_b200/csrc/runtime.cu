@@ -508,6 +508,8 @@ RankCtx *need_ctx() { return tl; }
 
 // ================================================================================== C ABI
 extern "C" {
+int proact_internal_preload_workloads(void);   // workloads.cu / graph.cu: load every kernel now
+int proact_internal_preload_graph(void);
 
 const char *proact_error_string(int code)
 {
@@ -616,6 +618,15 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM) !=
             cudaSuccess)
             return fail(PROACT_ERR_CUDA);
+        // no lazy kernel loading once ranks may spin on each other (see workloads.cu)
+        {
+            cudaFuncAttributes fa;
+            const void *k[] = {(const void *)agent_kernel, (const void *)sync_kernel,
+                               (const void *)credit_wait_kernel};
+            for (const void *f : k)
+                if (cudaFuncGetAttributes(&fa, f) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+            if (proact_internal_preload_workloads() || proact_internal_preload_graph()) return fail(PROACT_ERR_CUDA);
+        }
         // the L1/shared carveout is an SM-wide setting: an SM configured for a smaller carveout by
         // the agent cannot host producer CTAs next to it (measured: 16 agent CTAs pushed 16
         // producer CTAs into a second wave, +70% phase time).  Agent and producers use the max.

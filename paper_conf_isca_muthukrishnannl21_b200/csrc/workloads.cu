@@ -501,6 +501,20 @@ int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int sca
     return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
 }
 
+// Force-load this translation unit's kernels (called by proact_init).  Under CUDA's lazy module
+// loading the first launch of a kernel loads it, and a load waits for the device's running
+// kernels -- with loopback ranks one of those can be a spin waiting for this very thread's next
+// launch (observed: smoke deadlocks until the watchdog).  Loading up front removes the hazard.
+__attribute__((visibility("hidden"))) int proact_internal_preload_workloads(void)
+{
+    cudaFuncAttributes a;
+    const void *k[] = {(const void *)jacobi_kernel<true>, (const void *)jacobi_kernel<false>,
+                       (const void *)micro_kernel, (const void *)banded_kernel};
+    for (const void *f : k)
+        if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
+    return PROACT_OK;
+}
+
 }  // extern "C"
 
 extern "C" int proact_banded_phase(int region_in, int region_out, const float *a, const float *b, long long N,
