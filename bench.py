@@ -197,6 +197,10 @@ def main():
     ap.add_argument("--grid-n", dest="n", type=int, default=N_GRID)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-baselines", action="store_true", help="N > 1: skip the bulk / inline / NCCL legs")
+    ap.add_argument("--no-overhead", action="store_true",
+                    help="skip the ELIDE tracking-overhead leg (its agent kernel must run concurrently "
+                         "with the producer, which a kernel-serialising profiler prevents)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for the timing barrier / max-over-ranks only")
     args = ap.parse_args()
@@ -229,7 +233,11 @@ def main():
     else:
         job = rt.new_job_key()
     rt.init(world, rank, job)
-    mech = {v: k for k, v in _lib.MECH_NAMES.items()}[args.mech]
+    # --mech nccl: the north star's bulk baseline -- uninstrumented kernels (LOCAL) with an NCCL
+    # all-gather of the rows between them (workloads.Jacobi.step_allgather)
+    nccl_base = args.mech == "nccl"
+    mode = {"nccl": nccl_base}
+    mech = _lib.MECH_LOCAL if nccl_base else {v: k for k, v in _lib.MECH_NAMES.items()}[args.mech]
     cfg = rt.get_config()
     chunk = args.chunk or cfg["chunk_bytes"]
     kw = {"mech": mech}
@@ -243,6 +251,10 @@ def main():
     s = torch.cuda.Stream()
 
     def step():
+        if mode["nccl"]:
+            for k in range(I):
+                J.step_allgather(s)
+            return
         for k in range(I):
             J.step(s, barrier=(k == I - 1))
 
@@ -301,7 +313,7 @@ def main():
     # ---- tracking overhead (Sec. V-C, Fig. 8): the same step with
     # instrumentation + agent but no remote stores (ELIDE) vs the uninstrumented kernel (LOCAL)
     overhead = None
-    if world == 1:
+    if world == 1 and not args.no_overhead:
         kk = max(2, args.steps // 2)
         res = {}
         for name, m in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE)):
@@ -312,6 +324,24 @@ def main():
                     "tracking_overhead_frac": res["local"] / res["elide"] - 1.0,
                     "note": "G=1: FUSED has nothing to send and runs the LOCAL kernel; ELIDE keeps "
                             "tallies + agent (paper's instrumentation-only run)"}
+        rt.set_config(mech=mech)
+
+    # ---- baselines on the same ranks (north star: beat bulk DMA / NCCL all-gather and naive
+    # P2P stores): iterations/s of the same step with each mechanism, N > 1 only (at N = 1
+    # there is nothing to move and every mechanism is the plain kernel)
+    baselines = None
+    if world > 1 and not args.no_baselines:
+        baselines = {}
+        kk = max(2, args.steps // 2)
+        legs = [("bulk_cudaMemcpyPeer", _lib.MECH_BULK, False), ("naive_p2p_inline", _lib.MECH_INLINE, False)]
+        if dist.get_backend() == "nccl":
+            legs.append(("nccl_allgather", _lib.MECH_LOCAL, True))
+        for name, m, use_nccl in legs:
+            rt.set_config(mech=m)
+            mode["nccl"] = use_nccl
+            step()
+            baselines[name] = kk * I / (timed(step, kk) / 1000.0)
+        mode["nccl"] = nccl_base
         rt.set_config(mech=mech)
 
     # ---- e2e through the C-ABI host-buffer entry point
@@ -349,7 +379,8 @@ def main():
                            "parallelism": f"rows{world}",
                            "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)]},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-                "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead}
+                "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead,
+                "baselines_iters_per_s": baselines}
         print(json.dumps(line), flush=True)
     torch.cuda.synchronize()
     rt.finalize()

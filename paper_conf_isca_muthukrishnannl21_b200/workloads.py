@@ -75,9 +75,34 @@ class Jacobi:
         rt.phase_sync(stream, barrier=barrier)
         self.k += 1
 
+    def step_allgather(self, stream=None, group=None) -> None:
+        """BASELINE (north star: "a bulk ... NCCL-allgather version between kernels"): the
+        uninstrumented phase kernel (config mech must be LOCAL), then an in-place NCCL all-gather
+        of the rows into every replica, then the phase sync.  Equal row slices required."""
+        import torch.distributed as dist
+        i = self.k & 1
+        if self.N % self.G:
+            raise ValueError("all-gather baseline needs N divisible by the world size")
+        jacobi_phase(self.rid[i], self.rid[i ^ 1], self.N, self.rpt, stream)
+        out = self.bufs[i ^ 1].view(-1)
+        mine = out[self.r0 * self.N:self.r1 * self.N]
+        if self.G > 1:
+            with torch.cuda.stream(stream) if stream is not None else _nullctx():
+                dist.all_gather_into_tensor(out, mine, group=group)
+        rt.phase_sync(stream, barrier=False)
+        self.k += 1
+
     @property
     def current(self) -> torch.Tensor:
         return self.bufs[self.k & 1]
+
+
+class _nullctx:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
 
 
 def jacobi_solve_host(x0_host, out_host, N: int, iters: int, chunk_bytes: int,

@@ -82,3 +82,6 @@ def test_bench_two_processes_json_line():
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "strong"
+    # the same ranks time the bulk-copy and naive-P2P baselines (NCCL needs distinct GPUs)
+    assert set(d["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
+    assert all(v > 0 for v in d["baselines_iters_per_s"].values())
