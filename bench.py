@@ -198,6 +198,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baselines", action="store_true", help="N > 1: skip the bulk / inline / NCCL legs")
+    ap.add_argument("--no-tune", action="store_true", help="N > 1: keep the default chunk / agent warps")
     ap.add_argument("--no-overhead", action="store_true",
                     help="skip the ELIDE tracking-overhead leg (its agent kernel must run concurrently "
                          "with the producer, which a kernel-serialising profiler prevents)")
@@ -249,6 +250,40 @@ def main():
     J = wl.Jacobi(N, chunk, x0=x0, rows_per_tile=args.rpt)
     del x0
     s = torch.cuda.Stream()
+
+    # N > 1, PROACT mechanism, no explicit --warps/--chunk: the paper's profiler (Sec. III-A,
+    # a9) picks chunk size and agent warps for this G before anything is timed -- the transfer
+    # volume grows with G - 1, so one fixed agent size cannot fit 2 and 8 GPUs.  A small space
+    # (3 warm + 5 timed phases per point, max over ranks), a fresh cache file per job.
+    tuned = None
+    if world > 1 and args.mech == "fused" and not args.warps and not args.chunk and not args.no_tune:
+        os.environ["PROACT_TUNE_CACHE"] = f"/tmp/proact_tune_{job}.json"
+
+        def run_point(c):
+            if c["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+                for rid in J.rid:
+                    rt.rechunk(rid, c["chunk_bytes"])
+            for _ in range(3):
+                J.step(s)
+            ts = []
+            for _ in range(5):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(s)
+                J.step(s, barrier=True)
+                b.record(s)
+                s.synchronize()
+                ts.append(a.elapsed_time(b))
+            return statistics.median(ts)
+
+        best = rt.autotune(f"bench_jacobi_N{N}_G{world}", run_point,
+                           "mech=0;chunk=131072,1048576;warps=16,32,64;push=1;akern=1")
+        if best["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+            for rid in J.rid:
+                rt.rechunk(rid, best["chunk_bytes"])
+        cfg = rt.set_config(mech=best["mech"], agent_warps=best["agent_warps"], push=best["push"],
+                            agent_kernel=best["agent_kernel"], chunk_bytes=best["chunk_bytes"])
+        chunk = best["chunk_bytes"]
+        tuned = "proact_autotune: chunk {128K, 1M} x agent warps {16, 32, 64}"
 
     def step():
         if mode["nccl"]:
@@ -305,6 +340,18 @@ def main():
     peaks, src = _peaks()
     peak = float(peaks.get("hbm_gbs", 6650.0))
     achieved = alg_bytes / (kms / 1000.0) / 1e9
+    # whole-phase roofline of SURVEY.md Sec. 8(d): T_roof = max(T_HBM, T_NVL) per rank, T_HBM =
+    # my rows' 8 B/cell at the HBM peak, T_NVL = the replicated ingress ((G-1)/G of the grid,
+    # full replication) at 900 GB/s per direction; frac = T_roof / measured phase time
+    NVL = 900.0
+    ingress = 4.0 * N * (N - nrows)      # bytes pushed INTO this rank per phase (max over ranks ~ equal)
+    t_phase_us = ms / (args.steps * I) * 1000.0
+    t_hbm_us = alg_bytes / (peak * 1e9) * 1e6
+    t_nvl_us = ingress / (NVL * 1e9) * 1e6
+    step_roofline = {"t_hbm_us": t_hbm_us, "t_nvl_us": t_nvl_us, "t_phase_us": t_phase_us,
+                     "frac": max(t_hbm_us, t_nvl_us) / t_phase_us,
+                     "nvlink_ingress_GBps_per_gpu": ingress / (t_phase_us * 1e-6) / 1e9, "nvlink_peak_GBps": NVL,
+                     "note": "per rank and phase; NVLink 900 GB/s/direction nominal (B200_PROFILING.md)"}
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": _traffic_from_profiles(),
                 "kernel": "jacobi_kernel", "kernel_ms": kms, "alg_bytes_per_launch": alg_bytes,
@@ -374,11 +421,11 @@ def main():
                 "config": {"workload": WORKLOAD, "N": N, "iters_per_step": I, "ranks": world,
                            "mech": args.mech, "chunk_bytes": chunk,
                            "agent_warps": cfg["agent_warps"], "piece_bytes": cfg["piece_bytes"],
-                           "rows_per_tile": args.rpt, "replication": "full",
+                           "rows_per_tile": args.rpt, "replication": "full", "tuned": tuned,
                            "l2": "inputs > L2 (two 1 GiB grids), no flush",
                            "parallelism": f"rows{world}",
                            "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)]},
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "roofline": roofline, "step_roofline": step_roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead,
                 "baselines_iters_per_s": baselines}
         print(json.dumps(line), flush=True)
