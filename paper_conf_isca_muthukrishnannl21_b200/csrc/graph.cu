@@ -57,7 +57,10 @@ constexpr uint32_t SPLIT = 32768;  // max in-edges per work item: bigger tiles a
 struct Item {
     uint32_t tile, e0, e1;   // edges [e0, e1) (local CSC indices)
     uint32_t nsplit;         // items of this tile (1 = unsplit)
-    uint32_t slot, pad[3];   // split-tile accumulator slot
+    uint32_t slot;           // split-tile accumulator slot
+    uint32_t run_pr;         // first entry of this item in runv_pr (PageRank runs of PR_RUN edges)
+    uint32_t run_ss;         // first entry of this item in runv_ss (SSSP runs of SSSP_RUN edges)
+    uint32_t pad;
 };
 
 struct GraphDev {
@@ -70,6 +73,8 @@ struct GraphDev {
     unsigned long long *acc_f;   // [nslot * GT] split-tile fixed-point sums (PageRank), zero between launches
     int32_t *acc_i;           // [nslot * GT] split-tile minima (SSSP), INT32_MAX between launches
     uint32_t *acc_cnt;        // [nslot] arrivals of a split tile's items
+    const uint16_t *runv_pr;  // per PageRank run (RUN consecutive in-edges of an item): tile-local
+    const uint16_t *runv_ss;  //   vertex of its first edge (the merge-path search, done once at build)
     uint32_t V, v0, nv, nitems;
 };
 
@@ -85,6 +90,7 @@ struct Graph {
     unsigned long long *acc_f = nullptr;
     int32_t *acc_i = nullptr;
     uint32_t *acc_cnt = nullptr;
+    uint16_t *runv_pr = nullptr, *runv_ss = nullptr;
 };
 constexpr int MAXGRAPH = 4;
 thread_local Graph graphs[MAXGRAPH];
@@ -230,6 +236,12 @@ __device__ __forceinline__ uint32_t ld_stream_u(const uint32_t *p, uint64_t pol)
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
+__device__ __forceinline__ uint32_t ld_stream_u16(const uint16_t *p, uint64_t pol)
+{
+    uint16_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
+    return v;
+}
 __device__ __forceinline__ int32_t ld_stream_i(const int32_t *p, uint64_t pol)
 {
     int32_t v;
@@ -298,6 +310,20 @@ __device__ __forceinline__ uint32_t vertex_of(const uint32_t *cp, uint32_t nvt, 
     return lo;
 }
 
+// Build-time merge-path search: for every run of RUN consecutive in-edges of every item, the
+// tile-local index of the vertex owning the run's first edge (vertex_of on the global colptr).
+// One CTA per item.  The kernels read these 2-byte entries instead of searching shared memory.
+__global__ void runv_kernel(const Item *items, const uint32_t *colptr, uint32_t nv, uint32_t RUN, int which,
+                            uint16_t *runv)
+{
+    const Item it = items[blockIdx.x];
+    const uint32_t lo = it.tile * GT, nvt = min(lo + GT, nv) - lo;
+    const uint32_t nrun = (it.e1 - it.e0 + RUN - 1) / RUN;
+    const uint32_t off = which ? it.run_ss : it.run_pr;
+    for (uint32_t j = threadIdx.x; j < nrun; j += blockDim.x)
+        runv[off + j] = (uint16_t)vertex_of(colptr + lo, nvt, it.e0 + j * RUN);
+}
+
 // Tile prologue: colptr of the tile into shared memory (+ the accumulator init by the caller).
 __device__ __forceinline__ uint32_t load_tile(const GraphDev &g, uint32_t tile, uint32_t *cp, uint32_t &lo)
 {
@@ -348,12 +374,17 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
         if (xh) atomicAdd(&acc_hi[i], xh);
     };
     auto acc_get = [&](uint32_t i) { return ((unsigned long long)acc_hi[i] << 32) | acc_lo[i]; };
+    __shared__ uint32_t kclaim;
     bool waited = false;
-    for (uint32_t k = proact::producer_block(lc); k < p.g.nitems; k += proact::producer_grid(lc)) {
-        if (!waited) {   // (a7) every chunk of the previous generation is in my replica
-            if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
-            waited = true;
+    for (;;) {
+        if (threadIdx.x == 0) {
+            if (!waited) proact::wait_all(lc, p.region_in);   // (a7) previous generation is here
+            kclaim = proact::claim_tile(lc, p.g.nitems);       // items dealt dynamically
         }
+        waited = true;
+        __syncthreads();
+        const uint32_t k = kclaim;
+        if (k >= p.g.nitems) break;
         const Item it = p.g.items[k];
         uint32_t lo;
         const uint32_t nvt = load_tile(p.g, it.tile, cp, lo);
@@ -364,10 +395,10 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
             if (r0 < it.e1) {
                 const uint32_t r1 = min(r0 + RUN, it.e1);
                 float g[RUN];
+                uint32_t i = ld_stream_u16(p.g.runv_pr + it.run_pr + (r0 - it.e0) / RUN, pf);
 #pragma unroll
                 for (int q = 0; q < RUN; ++q)
                     g[q] = r0 + q < r1 ? ld_gather_f(cin + ld_stream_u(p.g.rowidx + r0 + q, pf), pl) : 0.f;
-                uint32_t i = vertex_of(cp, nvt, r0);
                 uint32_t nxt = cp[i + 1];
                 unsigned long long sum = 0ull;
 #pragma unroll
@@ -428,8 +459,13 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
     // source vertex -> global chunk id: rank slices are chunk-aligned, so it is u*4/chunk_bytes
     const uint32_t cv = Ri.chunk_bytes / 4;
     const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
+    __shared__ uint32_t kclaim;
     bool ready = false;
-    for (uint32_t k = proact::producer_block(lc); k < p.g.nitems; k += proact::producer_grid(lc)) {
+    for (;;) {
+        if (threadIdx.x == 0) kclaim = proact::claim_tile(lc, p.g.nitems);   // items dealt dynamically
+        __syncthreads();
+        const uint32_t k = kclaim;
+        if (k >= p.g.nitems) break;
         if (!ready) {   // (a7) wait for the previous generation, then snapshot its changed bits
             if (threadIdx.x == 0) proact::wait_all(lc, p.region_in);
             __syncthreads();
@@ -475,7 +511,7 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
                         }
                     }
                 }
-                uint32_t i = vertex_of(cp, nvt, r0);
+                uint32_t i = ld_stream_u16(p.g.runv_ss + it.run_ss + (r0 - it.e0) / RUN, pf);
                 uint32_t nxt = cp[i + 1];
                 int32_t best = INT32_MAX;
 #pragma unroll
@@ -553,6 +589,8 @@ int graph_dev(int id, GraphDev *g)
     g->acc_f = G.acc_f;
     g->acc_i = G.acc_i;
     g->acc_cnt = G.acc_cnt;
+    g->runv_pr = G.runv_pr;
+    g->runv_ss = G.runv_ss;
     g->V = G.V;
     g->v0 = G.v0;
     g->nv = G.nv;
@@ -658,8 +696,23 @@ int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32
         }
         split.insert(split.end(), whole.begin(), whole.end());   // big (hub) work first
         G.nitems = (uint32_t)split.size();
+        uint64_t npr = 0, nss = 0;
+        for (Item &it : split) {
+            it.run_pr = (uint32_t)npr;
+            it.run_ss = (uint32_t)nss;
+            npr += (it.e1 - it.e0 + PROACT_PR_RUN - 1) / PROACT_PR_RUN;
+            nss += (it.e1 - it.e0 + PROACT_SSSP_RUN - 1) / PROACT_SSSP_RUN;
+        }
+        if (npr >= (1ull << 32) || nss >= (1ull << 32)) return PROACT_ERR_NOMEM;
         GCK(cudaMalloc((void **)&G.items, sizeof(Item) * std::max<size_t>(1, split.size())));
         GCK(cudaMemcpy(G.items, split.data(), sizeof(Item) * split.size(), cudaMemcpyHostToDevice));
+        GCK(cudaMalloc((void **)&G.runv_pr, 2 * std::max<uint64_t>(1, npr)));
+        GCK(cudaMalloc((void **)&G.runv_ss, 2 * std::max<uint64_t>(1, nss)));
+        if (G.nitems) {
+            runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PR_RUN, 0, G.runv_pr);
+            runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_SSSP_RUN, 1, G.runv_ss);
+            GCK(cudaGetLastError());
+        }
         const size_t ns = std::max<uint32_t>(1, G.nslot);
         GCK(cudaMalloc((void **)&G.acc_f, 8 * ns * GT));
         GCK(cudaMemset(G.acc_f, 0, 8 * ns * GT));
@@ -691,6 +744,8 @@ int proact_graph_free(int id)
     cudaFree(G.acc_f);
     cudaFree(G.acc_i);
     cudaFree(G.acc_cnt);
+    cudaFree(G.runv_pr);
+    cudaFree(G.runv_ss);
     G = Graph();
     return PROACT_OK;
 }
@@ -777,7 +832,7 @@ __attribute__((visibility("hidden"))) int proact_internal_preload_graph(void)
     cudaFuncAttributes a;
     const void *k[] = {(const void *)count_kernel, (const void *)scan_blocks, (const void *)scan_totals,
                        (const void *)scan_add, (const void *)scatter_kernel, (const void *)pagerank_kernel,
-                       (const void *)sssp_kernel, (const void *)pr_init_kernel};
+                       (const void *)sssp_kernel, (const void *)pr_init_kernel, (const void *)runv_kernel};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
     return PROACT_OK;
