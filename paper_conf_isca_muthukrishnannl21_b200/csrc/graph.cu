@@ -390,17 +390,28 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
         const uint32_t nvt = load_tile(p.g, it.tile, cp, lo);
         for (uint32_t i = threadIdx.x; i < nvt; i += GB) acc_lo[i] = acc_hi[i] = 0u;
         __syncthreads();
+        // Runs are dealt to lanes in a 4 x 8 transposed order (lane l takes run 8*(l&3)... see
+        // lrun): a warp still covers 32 consecutive runs (coalesced index loads), but lanes that
+        // issue the same atomic instruction sit RUN*8 edges apart, so light vertices rarely
+        // collide on one shared-memory address.  A warp whose 32 runs all lie inside one vertex
+        // (hub in-edges) reduces in registers and issues a single atomic.
+        const uint32_t lane = threadIdx.x & 31u;
+        const uint32_t lrun = (threadIdx.x & ~31u) + ((lane & 3u) << 3) + (lane >> 2);
         for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
-            const uint32_t r0 = base + threadIdx.x * RUN;
-            if (r0 < it.e1) {
+            const uint32_t r0 = base + lrun * RUN;
+            const bool act = r0 < it.e1;
+            uint32_t i = 0xFFFFFFFFu;
+            unsigned long long sum = 0ull;
+            bool single = false;
+            if (act) {
                 const uint32_t r1 = min(r0 + RUN, it.e1);
                 float g[RUN];
-                uint32_t i = ld_stream_u16(p.g.runv_pr + it.run_pr + (r0 - it.e0) / RUN, pf);
+                i = ld_stream_u16(p.g.runv_pr + it.run_pr + (r0 - it.e0) / RUN, pf);
 #pragma unroll
                 for (int q = 0; q < RUN; ++q)
                     g[q] = r0 + q < r1 ? ld_gather_f(cin + ld_stream_u(p.g.rowidx + r0 + q, pf), pl) : 0.f;
                 uint32_t nxt = cp[i + 1];
-                unsigned long long sum = 0ull;
+                single = r1 <= nxt;   // the whole run belongs to vertex i
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     if (r0 + q >= r1) break;
@@ -411,7 +422,15 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
                     }
                     sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
                 }
-                if (sum) acc_add(i, sum);
+            }
+            // hub fast path: every lane active, single-vertex runs, the same vertex
+            const uint32_t i0 = __shfl_sync(0xFFFFFFFFu, i, 0);
+            if (__all_sync(0xFFFFFFFFu, act && single && i == i0)) {
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xFFFFFFFFu, sum, o);
+                if (lane == 0 && sum) acc_add(i0, sum);
+            } else if (act && sum) {
+                acc_add(i, sum);
             }
         }
         __syncthreads();
@@ -491,9 +510,16 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
         const uint32_t nvt = load_tile(p.g, it.tile, cp, lo);
         for (uint32_t i = threadIdx.x; i < nvt; i += GB) acc[i] = INT32_MAX;
         __syncthreads();
+        // lane order and hub fast path as in pagerank_kernel
+        const uint32_t lane = threadIdx.x & 31u;
+        const uint32_t lrun = (threadIdx.x & ~31u) + ((lane & 3u) << 3) + (lane >> 2);
         for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
-            const uint32_t r0 = base + threadIdx.x * RUN;
-            if (r0 < it.e1) {
+            const uint32_t r0 = base + lrun * RUN;
+            const bool act = r0 < it.e1;
+            uint32_t i = 0xFFFFFFFFu;
+            int32_t best = INT32_MAX;
+            bool single = false;
+            if (act) {
                 const uint32_t r1 = min(r0 + RUN, it.e1);
                 int32_t c[RUN];
 #pragma unroll
@@ -511,9 +537,9 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
                         }
                     }
                 }
-                uint32_t i = ld_stream_u16(p.g.runv_ss + it.run_ss + (r0 - it.e0) / RUN, pf);
+                i = ld_stream_u16(p.g.runv_ss + it.run_ss + (r0 - it.e0) / RUN, pf);
                 uint32_t nxt = cp[i + 1];
-                int32_t best = INT32_MAX;
+                single = r1 <= nxt;
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     if (r0 + q >= r1) break;
@@ -524,7 +550,13 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
                     }
                     best = min(best, c[q]);
                 }
-                if (best != INT32_MAX) atomicMin(&acc[i], best);
+            }
+            const uint32_t i0 = __shfl_sync(0xFFFFFFFFu, i, 0);
+            if (__all_sync(0xFFFFFFFFu, act && single && i == i0)) {
+                best = __reduce_min_sync(0xFFFFFFFFu, best);
+                if (lane == 0 && best != INT32_MAX) atomicMin(&acc[i0], best);
+            } else if (act && best != INT32_MAX) {
+                atomicMin(&acc[i], best);
             }
         }
         __syncthreads();
