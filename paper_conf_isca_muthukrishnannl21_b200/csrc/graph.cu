@@ -30,7 +30,10 @@ using proact::region_dev;
 
 namespace {
 
-constexpr int GB = 256;            // threads per CTA
+#ifndef PROACT_GB
+#define PROACT_GB 256
+#endif
+constexpr int GB = PROACT_GB;      // threads per CTA
 constexpr int GT = 1024;           // vertices per tile (4 KiB of output, the paper's L279)
 constexpr int GL = 8;              // lanes per light vertex
 // consecutive in-edges per thread per round (merge path) and CTAs per SM, measured on B200

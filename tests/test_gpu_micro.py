@@ -130,3 +130,39 @@ def test_micro_ranks_with_empty_slices():
         want = oracle.micro_phase(words, p, SEED, 1)
         for g in range(G):
             assert np.array_equal(outs[g][p], want), (p, g)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("chunk", [4 << 20, 64 << 10])
+def test_config5_full_size_sampled(chunk):
+    """Config 5 at its largest region (R = 4 GiB, 2^30 words), two loopback ranks, in bench
+    launch configuration (default agent): every rank's replica equals the closed form on a random
+    sample of 200k words plus every slice / chunk boundary word, after each of 2 phases."""
+    W, G, K = 1 << 30, 2, 1
+    rng = np.random.default_rng(5)
+    samp = np.unique(np.concatenate([
+        rng.integers(0, W, 200_000),
+        np.array([0, 1, W // 2 - 1, W // 2, W // 2 + 1, W - 2, W - 1]),
+        np.arange(0, W, chunk // 4)[:4096], np.arange(chunk // 4 - 1, W, chunk // 4)[:4096]])).astype(np.int64)
+
+    def body(r, G_):
+        rt.set_config(mech=_lib.MECH_FUSED)
+        M = wl.Micro(W, chunk)
+        s = torch.cuda.Stream()
+        idx = torch.from_numpy(samp).cuda()
+        got = []
+        for p in range(2):
+            M.step(SEED, K, False, stream=s, barrier=True)
+            s.synchronize()
+            got.append(M.buf.index_select(0, idx).cpu().numpy().view(np.uint32).copy())
+            rt.host_barrier()
+        rt.check_device()
+        del M
+        return got
+
+    outs = run_ranks(G, body)
+    for p in range(2):
+        want = np.array([oracle.micro_word(int(k), p, SEED, K) for k in samp], dtype=np.uint32)
+        for g in range(G):
+            bad = np.nonzero(outs[g][p] != want)[0]
+            assert bad.size == 0, (p, g, samp[bad[:5]])
