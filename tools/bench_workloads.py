@@ -91,6 +91,15 @@ def pagerank(args, src, dst, V):
                          "alg_bytes_per_launch": alg, "achieved": alg / kms / 1e6, "peak": peak_hbm(),
                          "unit": "GB/s", "frac": alg / kms / 1e6 / peak_hbm(),
                          "note": "8 B/edge (index + gathered contrib) + 16 B/vertex; gathers hit L2"}}
+    # the bound that actually applies: every random 4-byte gather is one L1TEX
+    # wavefront, one per clock per SM -> t >= E_own / (SMs x SM clock)
+    prop = torch.cuda.get_device_properties(0)
+    e_max = max(r["e_own"] for r in res)
+    rate = prop.multi_processor_count * 1965e6          # gathers/s at the max SM clock
+    t_l1 = e_max / rate * 1e3
+    line["roofline_l1_gather"] = {"bound": "l1tex_wavefronts", "gathers_per_launch": e_max,
+                                  "peak_gathers_per_s": rate, "t_min_ms": t_l1, "frac": t_l1 / kms,
+                                  "note": "1 wavefront/clk/SM x SMs x 1965 MHz"}
     if not args.no_cpu:
         import oracle
         t0 = time.perf_counter()
