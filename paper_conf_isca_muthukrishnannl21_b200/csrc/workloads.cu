@@ -427,15 +427,39 @@ __global__ void __launch_bounds__(BB) banded_kernel(launch_ctx lc, proact_banded
         __syncthreads();
         for (int64_t k = threadIdx.x; k < hi - lo; k += BB) xs[k] = __ldcg(x + lo + k);
         __syncthreads();
-        for (int64_t i = i0 + threadIdx.x; i < i1; i += BB) {
-            float sum = 0.0f;
-            for (int64_t o = -w; o <= w; ++o) {
-                const int64_t j = i + o;
-                if (o == 0 || j < 0 || j >= N) continue;
-                sum = __fadd_rn(sum, __fmul_rn(ld_stream_f(p.a + (o + w) * N + i), xs[j - lo]));
+        // BR rows per thread (coalesced across the CTA); the diagonals are walked in groups of
+        // BU whose loads are all issued before the group's adds, so BR x BU streaming loads are
+        // in flight per thread while each row still sums o = -w..w in order (reading R19)
+        constexpr int BR = BT / BB, BU = 8;
+        float sum[BR];
+#pragma unroll
+        for (int r = 0; r < BR; ++r) sum[r] = 0.0f;
+        for (int64_t ob = -w; ob <= w; ob += BU) {
+            float av[BU][BR];
+#pragma unroll
+            for (int u = 0; u < BU; ++u)
+#pragma unroll
+                for (int r = 0; r < BR; ++r) {
+                    const int64_t o = ob + u, i = i0 + threadIdx.x + r * BB, j = i + o;
+                    av[u][r] = (o <= w && o != 0 && i < i1 && j >= 0 && j < N) ? ld_stream_f(p.a + (o + w) * N + i)
+                                                                                 : 0.0f;
+                }
+#pragma unroll
+            for (int u = 0; u < BU; ++u)
+#pragma unroll
+                for (int r = 0; r < BR; ++r) {
+                    const int64_t o = ob + u, i = i0 + threadIdx.x + r * BB, j = i + o;
+                    if (o <= w && o != 0 && i < i1 && j >= 0 && j < N)
+                        sum[r] = __fadd_rn(sum[r], __fmul_rn(av[u][r], xs[j - lo]));
+                }
+        }
+#pragma unroll
+        for (int r = 0; r < BR; ++r) {
+            const int64_t i = i0 + threadIdx.x + r * BB;
+            if (i < i1) {
+                const float v = __fdiv_rn(__fsub_rn(p.b[i], sum[r]), p.a[w * N + i]);
+                proact::put(lc, p.region_out, (uint64_t)i * 4, v);
             }
-            const float v = __fdiv_rn(__fsub_rn(p.b[i], sum), p.a[w * N + i]);
-            proact::put(lc, p.region_out, (uint64_t)i * 4, v);
         }
         __syncthreads();
         if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, (uint64_t)i0 * 4, (uint64_t)(i1 - i0) * 4);

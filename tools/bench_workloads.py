@@ -15,6 +15,7 @@ Roofline: the phase kernel's algorithmic bytes per launch / CUDA-event time (DES
 from __future__ import annotations
 
 import argparse
+import ctypes
 import json
 import os
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # loopback ranks: see loopback.py
@@ -173,9 +174,63 @@ def micro(args):
             "unit": "GB/s replicated (HBM loopback)", "ms_per_phase": ms / args.steps, "mech": args.mech}
 
 
+def banded(args):
+    """NEXT-2: the paper's banded-matrix Jacobi (L271), N = 2^scale rows, half-bandwidth --w;
+    step = 20 phases; roofline = (2w+1) x 4 B of A + 12 B (b, x read, x' write) per row / HBM."""
+    N, w, I = 1 << args.scale, args.w, 20
+    a, b = synth.banded(N, w)
+
+    def body(r, G):
+        rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+        B = wl.Banded(a, b, args.chunk)
+        s = torch.cuda.Stream()
+        for _ in range(2):
+            B.step(s)
+        torch.cuda.synchronize()
+        rt.host_barrier()
+        e0, e1 = ev(), ev()
+        e0.record(s)
+        for k in range(args.steps * I):
+            B.step(s, barrier=(k == args.steps * I - 1))
+        e1.record(s)
+        torch.cuda.synchronize()
+        ks = []
+        for _ in range(10):
+            x0, x1 = ev(), ev()
+            i = B.k & 1
+            x0.record(s)
+            _lib.check(rt.lib().proact_banded_phase(B.rid[i], B.rid[i ^ 1], ctypes.c_void_p(B.a.data_ptr()),
+                                                    ctypes.c_void_p(B.b.data_ptr()), B.N, B.w, wl._s(s)), "banded")
+            x1.record(s)
+            rt.phase_sync(s)
+            B.k += 1
+            ks.append((x0, x1))
+        torch.cuda.synchronize()
+        return {"ms": e0.elapsed_time(e1), "kms": statistics.median(x.elapsed_time(y) for x, y in ks),
+                "rows": B.r1 - B.r0}
+    res = run_ranks(args.ranks, body)
+    ms = max(r["ms"] for r in res)
+    kms = max(r["kms"] for r in res)
+    alg = max(((2 * w + 1) * 4 + 12) * r["rows"] for r in res)
+    line = {"workload": f"banded_jacobi N=2^{args.scale} w={w} (NEXT-2, PAPER.md L271)",
+            "value": args.steps * I / (ms / 1000.0), "unit": "iters/s", "ranks": args.ranks, "mech": args.mech,
+            "roofline": {"bound": "hbm", "kernel": "banded_kernel", "kernel_ms": kms, "alg_bytes_per_launch": alg,
+                         "achieved": alg / kms / 1e6, "peak": peak_hbm(), "unit": "GB/s",
+                         "frac": alg / kms / 1e6 / peak_hbm()}}
+    if not args.no_cpu:
+        import oracle
+        t0 = time.perf_counter()
+        oracle.banded_jacobi(a, b, np.zeros(N, dtype=np.float32), 2)
+        dt = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": 2 / dt, "unit": "iters/s", "cores": oracle.get_threads(), "kind": "oracle",
+                                "sample": "2 oracle.banded_jacobi iterations"}
+    return line
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--workload", default="pagerank", choices=["pagerank", "sssp", "micro"])
+    ap.add_argument("--workload", default="pagerank", choices=["pagerank", "sssp", "micro", "banded"])
+    ap.add_argument("--w", type=int, default=16, help="banded: half-bandwidth")
     ap.add_argument("--scale", type=int, default=24)
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
@@ -185,8 +240,8 @@ def main():
     ap.add_argument("--bytes", type=int, default=256 << 20)
     ap.add_argument("--no-cpu", action="store_true")
     args = ap.parse_args()
-    if args.workload == "micro":
-        print(json.dumps(micro(args)), flush=True)
+    if args.workload in ("micro", "banded"):
+        print(json.dumps(micro(args) if args.workload == "micro" else banded(args)), flush=True)
         return
     t0 = time.perf_counter()
     src, dst = synth.rmat(args.scale, 16)
