@@ -213,6 +213,11 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank)
         return
+    # the oracle baseline first, before this process pins host memory or touches the GPU (a
+    # later run shared the host with 2 GiB of pinned e2e buffers and measured ~3x slower)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args.n)
 
     import torch
     import torch.distributed as dist
@@ -408,10 +413,6 @@ def main():
         e2e = {"value": max(2, min(args.steps, 3)) * I / (ems / 1000.0), "unit": "iters/s",
                "h2d_bytes_per_step": nb[0], "d2h_bytes_per_step": nb[1],
                "api": "proact_jacobi_solve_host"}
-
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline(N)
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "iters/s", "n_gpus": world,

@@ -94,6 +94,15 @@ int proact_partition_bounds(const uint32_t *indeg, unsigned V, int G, unsigned a
  * exist).  The edge list may be freed afterwards.  Synchronises `stream`. */
 int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w,
                        unsigned long long E, unsigned V, unsigned v0, unsigned v1, void *stream);
+/* As proact_graph_build, plus the PageRank hot-source table: the `hot` vertices with the
+ * highest global out-degree (ties: smaller id; only vertices with out-edges; at most 45056) are
+ * staged in shared memory by every pagerank phase CTA and their in-edges read the table instead of
+ * the replica.  hot = 0: no table; hot < 0: env PROACT_GRAPH_HOT, else 8192 (two CTAs per SM).
+ * The result is bit-identical either way (exact fixed-point sums).  V < 2^31. */
+int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w,
+                          unsigned long long E, unsigned V, unsigned v0, unsigned v1, int hot, void *stream);
+/* Number of hot sources of a graph (0: none). */
+int proact_graph_hot(int graph, unsigned *nhot);
 int proact_graph_free(int graph);
 int proact_graph_info(int graph, unsigned long long *e_own, unsigned *v0, unsigned *nv);
 

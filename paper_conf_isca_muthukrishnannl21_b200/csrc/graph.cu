@@ -19,6 +19,8 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
+#include <cstring>
 #include <vector>
 
 #include "proact.h"
@@ -63,7 +65,7 @@ struct Item {
     uint32_t slot;           // split-tile accumulator slot
     uint32_t run_pr;         // first entry of this item in runv_pr (PageRank runs of PR_RUN edges)
     uint32_t run_ss;         // first entry of this item in runv_ss (SSSP runs of SSSP_RUN edges)
-    uint32_t pad;
+    uint32_t run_ph;         // first entry of this item in runv_ph (hot-kernel runs of PRH_RUN edges)
 };
 
 struct GraphDev {
@@ -78,7 +80,10 @@ struct GraphDev {
     uint32_t *acc_cnt;        // [nslot] arrivals of a split tile's items
     const uint16_t *runv_pr;  // per PageRank run (RUN consecutive in-edges of an item): tile-local
     const uint16_t *runv_ss;  //   vertex of its first edge (the merge-path search, done once at build)
-    uint32_t V, v0, nv, nitems;
+    const uint16_t *runv_ph;
+    const uint32_t *rowidx_h; // [E_own] rowidx with hot sources encoded as HOT_BIT | slot (nhot > 0)
+    const uint32_t *hot_ids;  // [nhot] the hot sources (highest out-degree), ascending ids
+    uint32_t V, v0, nv, nitems, nhot;
 };
 
 struct Graph {
@@ -93,9 +98,41 @@ struct Graph {
     unsigned long long *acc_f = nullptr;
     int32_t *acc_i = nullptr;
     uint32_t *acc_cnt = nullptr;
-    uint16_t *runv_pr = nullptr, *runv_ss = nullptr;
+    uint16_t *runv_pr = nullptr, *runv_ss = nullptr, *runv_ph = nullptr;
+    uint32_t *rowidx_h = nullptr, *hot_ids = nullptr;
+    uint32_t nhot = 0;
 };
 constexpr int MAXGRAPH = 4;
+
+// Hot-source table (pagerank_hot_kernel): the nhot sources with the highest out-degree carry
+// 23 % of RMAT-24's edges at nhot = 8192 (44 % at 45056).  Their contributions are staged once per
+// launch in shared memory, where a warp's 32 random reads cost ~3-4 bank wavefronts instead of the
+// 32 L1TEX wavefronts of a global gather (profiles/r01b_ncu_pagerank.md).  The default keeps two
+// 1024-thread CTAs per SM: one CTA with the 45056-entry table halves the warps in flight and runs
+// 2.4x slower (the gathers are latency-bound, tools/sweep_pagerank.py).
+constexpr uint32_t HOT_BIT = 0x80000000u;
+constexpr uint32_t HOT_MAX = 45056;   // 176 KiB table + 4 item groups x 12 KiB <= 227 KiB per CTA
+constexpr uint32_t HOT_DEFAULT = 8192;
+#ifndef PROACT_PRH_PG
+#define PROACT_PRH_PG 4
+#endif
+#ifndef PROACT_PRH_RUN
+#define PROACT_PRH_RUN 4
+#endif
+#ifndef PROACT_PRH_SEGRED   // warp segmented reduction instead of per-run atomics: measured slower
+#define PROACT_PRH_SEGRED 0   // (1.31 vs 1.20 ms at RMAT-24; the shared atomics are not the bound)
+#endif
+#ifndef PROACT_PRH_MINB      // hot-kernel CTAs per SM (register budget 64 / 32 per thread at 1 / 2)
+#define PROACT_PRH_MINB 1
+#endif
+#ifndef PROACT_SSH_MINB      // sssp_hot_kernel CTAs per SM
+#define PROACT_SSH_MINB 2
+#endif
+#ifndef PROACT_PRH_PIPE
+#define PROACT_PRH_PIPE 1
+#endif
+constexpr int PG = PROACT_PRH_PG;     // item groups (of GB threads) per hot-kernel CTA
+constexpr uint32_t CPS = GT + 4;      // words per group colptr window (GT + 1, padded)
 thread_local Graph graphs[MAXGRAPH];
 
 #define GCK(call)                                                                        \
@@ -206,6 +243,19 @@ __global__ void scatter_kernel(const uint32_t *src, const uint32_t *dst, const i
     }
 }
 
+__global__ void hot_slot_kernel(const uint32_t *hot_ids, uint32_t nhot, uint32_t *slot)
+{
+    for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < nhot; s += gridDim.x * blockDim.x)
+        slot[hot_ids[s]] = s;
+}
+__global__ void hot_encode_kernel(const uint32_t *rowidx, uint64_t E, const uint32_t *slot, uint32_t *out)
+{
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t u = rowidx[e], k = slot[u];
+        out[e] = k != 0xFFFFFFFFu ? (HOT_BIT | k) : u;
+    }
+}
+
 // ------------------------------------------------------------------ phase kernels
 struct PrParams {
     GraphDev g;
@@ -254,16 +304,26 @@ __device__ __forceinline__ int32_t ld_stream_i(const int32_t *p, uint64_t pol)
 // The gathered vector: written by peers' agents during the previous phase (all arrived: the CTA
 // waited with wait_all before its first load, and nothing rewrites it this phase), so the
 // read-only path is coherent here.
+#ifndef PROACT_GATHER_MODE   // 0: .nc; 1: .nc + L1::no_allocate; 2: .cg (L2 only)
+#define PROACT_GATHER_MODE 0
+#endif
+#if PROACT_GATHER_MODE == 1
+#define GATHER_OP "ld.global.nc.L1::no_allocate.L2::cache_hint"
+#elif PROACT_GATHER_MODE == 2
+#define GATHER_OP "ld.global.cg.L2::cache_hint"
+#else
+#define GATHER_OP "ld.global.nc.L2::cache_hint"
+#endif
 __device__ __forceinline__ float ld_gather_f(const float *p, uint64_t pol)
 {
     float v;
-    asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    asm volatile(GATHER_OP ".f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
     return v;
 }
 __device__ __forceinline__ int32_t ld_gather_i(const int32_t *p, uint64_t pol)
 {
     int32_t v;
-    asm volatile("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    asm volatile(GATHER_OP ".s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
 __device__ __forceinline__ uint32_t ld_nc_u(const uint32_t *p)
@@ -322,7 +382,7 @@ __global__ void runv_kernel(const Item *items, const uint32_t *colptr, uint32_t 
     const Item it = items[blockIdx.x];
     const uint32_t lo = it.tile * GT, nvt = min(lo + GT, nv) - lo;
     const uint32_t nrun = (it.e1 - it.e0 + RUN - 1) / RUN;
-    const uint32_t off = which ? it.run_ss : it.run_pr;
+    const uint32_t off = which == 2 ? it.run_ph : which ? it.run_ss : it.run_pr;
     for (uint32_t j = threadIdx.x; j < nrun; j += blockDim.x)
         runv[off + j] = (uint16_t)vertex_of(colptr + lo, nvt, it.e0 + j * RUN);
 }
@@ -460,6 +520,231 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
             if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, (uint64_t)lo * 4, (uint64_t)nvt * 4);
         }
         __syncthreads();
+    }
+}
+
+// ---- PageRank with a shared-memory hot-source table (the default when the graph has one).
+// One CTA per SM of PG independent item groups (GB threads each, own named barrier, own
+// accumulator / colptr arrays) around one table: hot[s] = contrib[hot_ids[s]], staged after the
+// arrival wait.  An in-edge whose source is hot (rowidx_h = HOT_BIT | s) reads the table; the
+// others gather from the replica as in pagerank_kernel.  Same exact fixed-point sums, so the
+// result is bit-identical to pagerank_kernel's.
+__device__ __forceinline__ void grp_bar(uint32_t grp)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(grp + 1u), "r"((uint32_t)GB) : "memory");
+}
+
+// claim_tile for PG claimers per CTA: the CTA counts out (and the last CTA re-arms the launch's
+// counters) when its last group has seen the end of the work list.
+__device__ __forceinline__ uint32_t claim_group(const launch_ctx &lc, uint32_t n, uint32_t *nout)
+{
+    uint32_t *S = lc.ctx->sched;
+    const uint32_t t = atomicAdd(&S[0], 1u);
+    if (t >= n && atomicAdd(nout, 1u) + 1u == (uint32_t)PG) {
+        const uint32_t P = gridDim.x - lc.agent_ctas;
+        if (atomicAdd(&S[1], 1u) + 1u == P) {
+            S[0] = 0u;
+            S[1] = 0u;
+        }
+    }
+    return t;
+}
+
+__global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(launch_ctx lc, PrParams p)
+{
+    constexpr int RUN = PROACT_PRH_RUN;
+    if (proact::agent_dispatch(lc)) return;
+    extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
+    __shared__ uint32_t acc_lo_a[PG][GT], acc_hi_a[PG][GT];
+    __shared__ uint32_t kclaim_a[PG], last_a[PG], nout;
+    const uint32_t grp = threadIdx.x / GB, t = threadIdx.x % GB;
+    uint32_t *acc_lo = acc_lo_a[grp], *acc_hi = acc_hi_a[grp], *cp = dyn + grp * CPS;
+    float *hot = reinterpret_cast<float *>(dyn + PG * CPS);
+    const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
+    const uint64_t pl = pol_last(), pf = pol_first();
+    auto acc_add = [&](uint32_t i, unsigned long long x) {
+        const uint32_t xl = (uint32_t)x, old = atomicAdd(&acc_lo[i], xl);
+        const uint32_t carry = old + xl < old ? 1u : 0u;
+        const uint32_t xh = (uint32_t)(x >> 32) + carry;
+        if (xh) atomicAdd(&acc_hi[i], xh);
+    };
+    auto acc_get = [&](uint32_t i) { return ((unsigned long long)acc_hi[i] << 32) | acc_lo[i]; };
+    if (threadIdx.x == 0) {
+        proact::wait_all(lc, p.region_in);   // (a7) previous generation is here
+        nout = 0u;
+    }
+    __syncthreads();
+    for (uint32_t s = threadIdx.x; s < p.g.nhot; s += blockDim.x) hot[s] = ld_gather_f(cin + __ldg(p.g.hot_ids + s), pl);
+    __syncthreads();
+    const uint32_t lane = t & 31u;
+#if PROACT_PRH_SEGRED
+    const uint32_t lrun = t;   // natural order: a warp's lanes hold 32 consecutive runs
+#else
+    const uint32_t lrun = (t & ~31u) + ((lane & 3u) << 3) + (lane >> 2);   // as in pagerank_kernel
+#endif
+    for (;;) {
+        if (t == 0) kclaim_a[grp] = claim_group(lc, p.g.nitems, &nout);
+        grp_bar(grp);
+        const uint32_t k = kclaim_a[grp];
+        if (k >= p.g.nitems) break;
+        const Item it = p.g.items[k];
+        const uint32_t lo = p.g.v0 + it.tile * GT, nvt = min(lo + GT, p.g.v0 + p.g.nv) - lo;
+        for (uint32_t i = t; i <= nvt; i += GB) cp[i] = ld_stream_u(p.g.colptr + (lo - p.g.v0 + i), pf);
+        for (uint32_t i = t; i < nvt; i += GB) acc_lo[i] = acc_hi[i] = 0u;
+        grp_bar(grp);
+        // index stream software-pipelined one round ahead (PRH_PIPE): the next round's rowidx /
+        // run entries are in flight while this round's gathers are, so a round costs one L2 round
+        // trip instead of two
+        uint32_t xn[RUN], in_ = 0;
+        auto load_idx = [&](uint32_t base) {
+            const uint32_t r0 = base + lrun * RUN;
+#pragma unroll
+            for (int q = 0; q < RUN; ++q) xn[q] = r0 + q < it.e1 ? ld_stream_u(p.g.rowidx_h + r0 + q, pf) : HOT_BIT;
+            in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - it.e0) / RUN, pf) : 0u;
+        };
+        if (PROACT_PRH_PIPE) load_idx(it.e0);
+        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+            const uint32_t r0 = base + lrun * RUN;
+            const bool act = r0 < it.e1;
+            if (!PROACT_PRH_PIPE) load_idx(base);
+            uint32_t x[RUN];
+#pragma unroll
+            for (int q = 0; q < RUN; ++q) x[q] = xn[q];
+            uint32_t i = act ? in_ : 0xFFFFFFFFu;
+            if (PROACT_PRH_PIPE && base + GB * RUN < it.e1) load_idx(base + GB * RUN);
+#if PROACT_PRH_SEGRED
+            // Per-lane segments in edge order: the first (kin, vin), the last (kout, vout); segments
+            // strictly inside the run are flushed at once.  A warp-wide segmented scan then joins
+            // the chains that cross lanes, so every vertex a warp touches costs ONE shared atomic
+            // per round (shared atomics cost ~2 cycles per active lane, B300_MICROARCH.md).
+            uint32_t kin = 0xFFFFFFFFu, kout = 0xFFFFFFFFu;
+            unsigned long long vin = 0ull, vout = 0ull;
+            bool multi = false;
+            if (act) {
+                const uint32_t r1 = min(r0 + RUN, it.e1);
+                float g[RUN];
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    const bool h = x[q] & HOT_BIT;
+                    g[q] = h ? hot[x[q] & ~HOT_BIT & 0xFFFFu] : 0.f;
+                    if (!h) g[q] = ld_gather_f(cin + x[q], pl);
+                }
+                uint32_t nxt = cp[i + 1];
+                unsigned long long sum = 0ull;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    if (r0 + q >= r1) break;
+                    while (r0 + q >= nxt) {   // vertex i closes before edge r0 + q
+                        if (!multi) {
+                            kin = i;
+                            vin = sum;
+                            multi = true;
+                        } else if (sum) {
+                            acc_add(i, sum);
+                        }
+                        sum = 0ull;
+                        nxt = cp[++i + 1];
+                    }
+                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
+                }
+                if (!multi) {
+                    kin = i;
+                    vin = sum;
+                }
+                kout = i;
+                vout = sum;
+            }
+            const uint32_t kprev = __shfl_up_sync(0xFFFFFFFFu, kout, 1);
+            const uint32_t knext = __shfl_down_sync(0xFFFFFFFFu, kin, 1);
+            // chain value ending at my last segment: inclusive segmented scan, a segment starts
+            // at every lane that does not wholly continue the previous lane's last vertex
+            unsigned long long T = vout;
+            bool st = !(lane > 0 && !multi && kin == kprev);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const unsigned long long Tu = __shfl_up_sync(0xFFFFFFFFu, T, d);
+                const bool su = __shfl_up_sync(0xFFFFFFFFu, st, d);
+                if (lane >= (uint32_t)d && !st) {
+                    T += Tu;
+                    st = su;
+                }
+            }
+            const unsigned long long Tprev = __shfl_up_sync(0xFFFFFFFFu, T, 1);
+            if (act) {
+                if (multi) {   // my first vertex, joined with the chain arriving from the left
+                    const unsigned long long hv = vin + (lane > 0 && kin == kprev ? Tprev : 0ull);
+                    if (hv) acc_add(kin, hv);
+                }
+                if ((lane == 31 || knext != kout) && T) acc_add(kout, T);   // my chain ends here
+            }
+        }
+#else
+            unsigned long long sum = 0ull;
+            bool single = false;
+            if (act) {
+                const uint32_t r1 = min(r0 + RUN, it.e1);
+                float g[RUN];
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    const bool h = x[q] & HOT_BIT;
+                    g[q] = h ? hot[x[q] & ~HOT_BIT & 0xFFFFu] : 0.f;
+                    if (!h) g[q] = ld_gather_f(cin + x[q], pl);
+                }
+                uint32_t nxt = cp[i + 1];
+                single = r1 <= nxt;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    if (r0 + q >= r1) break;
+                    while (r0 + q >= nxt) {
+                        if (sum) acc_add(i, sum);
+                        sum = 0ull;
+                        nxt = cp[++i + 1];
+                    }
+                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
+                }
+            }
+            const uint32_t i0 = __shfl_sync(0xFFFFFFFFu, i, 0);
+            if (__all_sync(0xFFFFFFFFu, act && single && i == i0)) {
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xFFFFFFFFu, sum, o);
+                if (lane == 0 && sum) acc_add(i0, sum);
+            } else if (act && sum) {
+                acc_add(i, sum);
+            }
+        }
+#endif
+        grp_bar(grp);
+        bool fin = true;
+        if (it.nsplit > 1) {   // hub tile: sums meet in the global accumulator
+            unsigned long long *ga = p.g.acc_f + (size_t)it.slot * GT;
+            for (uint32_t i = t; i < nvt; i += GB)
+                if (acc_get(i)) atomicAdd(&ga[i], acc_get(i));
+            grp_bar(grp);
+            if (t == 0) {
+                __threadfence();
+                const uint32_t old = atomicAdd(&p.g.acc_cnt[it.slot], 1u);
+                __threadfence();
+                last_a[grp] = old + 1 == it.nsplit;
+            }
+            grp_bar(grp);
+            fin = last_a[grp] != 0;
+            if (fin) {
+                for (uint32_t i = t; i < nvt; i += GB) {
+                    const unsigned long long v = __ldcg(&ga[i]);
+                    acc_lo[i] = (uint32_t)v;
+                    acc_hi[i] = (uint32_t)(v >> 32);
+                    ga[i] = 0ull;   // ready for the next launch
+                }
+                if (t == 0) p.g.acc_cnt[it.slot] = 0;
+                grp_bar(grp);
+            }
+        }
+        if (fin) {
+            for (uint32_t i = t; i < nvt; i += GB) pr_finish(lc, p, lo + i, (double)acc_get(i) * UNFIX);
+            grp_bar(grp);
+            if (t == 0) proact::commit_span(lc, p.region_out, (uint64_t)lo * 4, (uint64_t)nvt * 4);
+        }
+        grp_bar(grp);
     }
 }
 
@@ -605,6 +890,181 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
     }
 }
 
+// ---- SSSP with the hot-source table and the pipelined index stream (as pagerank_hot_kernel).
+// hot[s] = d[hot_ids[s]] if that source's chunk changed in the previous round (or first round),
+// else INT32_MAX, so a hot in-edge needs neither the bitmap test nor the global gather.
+__global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(launch_ctx lc, SsspParams p)
+{
+    constexpr int RUN = PROACT_SSSP_RUN;   // shares runv_ss with sssp_kernel
+    if (proact::agent_dispatch(lc)) return;
+    extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
+    __shared__ int32_t acc_a[PG][GT];
+    __shared__ uint32_t chg[CHG_WORDS];
+    __shared__ uint32_t kclaim_a[PG], last_a[PG], any_a[PG], nout;
+    const uint32_t grp = threadIdx.x / GB, t = threadIdx.x % GB;
+    int32_t *acc = acc_a[grp];
+    uint32_t *cp = dyn + grp * CPS;
+    int32_t *hot = reinterpret_cast<int32_t *>(dyn + PG * CPS);
+    const region_dev &Ri = lc.ctx->region[p.region_in];
+    const int32_t *din = reinterpret_cast<const int32_t *>(Ri.base);
+    const uint64_t pf = pol_first(), pl = pol_last();
+    const uint32_t cv = Ri.chunk_bytes / 4;
+    const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
+    auto changed_src = [&](uint32_t u) {
+        const uint32_t g = cdiv ? u / cdiv : u >> cshift;
+        return p.first || (chg[g >> 5] >> (g & 31) & 1u);
+    };
+    // (a7) wait for the previous generation, snapshot its changed bits, stage the hot table
+    if (threadIdx.x == 0) {
+        proact::wait_all(lc, p.region_in);
+        nout = 0u;
+    }
+    __syncthreads();
+    {
+        const uint32_t gen = lc.gen[p.region_in];
+        const uint32_t pm = lc.gen_mech[p.region_in];
+        const bool agent = pm == PROACT_MECH_FUSED || pm == PROACT_MECH_ELIDE;
+        for (uint32_t wi = threadIdx.x; wi < CHG_WORDS && wi * 32 < Ri.n_total; wi += blockDim.x) {
+            uint32_t bits = 0;
+            for (uint32_t bb = 0; bb < 32; ++bb) {
+                const uint32_t g = wi * 32 + bb;
+                if (g >= Ri.n_total) break;
+                bool c;
+                if (g >= Ri.chunk0 && g < Ri.chunk0 + Ri.n_own) c = Ri.changed_gen[g - Ri.chunk0] == gen;
+                else c = !agent || (ld_nc_u(Ri.arrive + g) & 1u);
+                bits |= (uint32_t)c << bb;
+            }
+            chg[wi] = bits;
+        }
+    }
+    __syncthreads();
+    for (uint32_t s = threadIdx.x; s < p.g.nhot; s += blockDim.x) {
+        const uint32_t u = __ldg(p.g.hot_ids + s);
+        hot[s] = changed_src(u) ? ld_gather_i(din + u, pl) : INT32_MAX;
+    }
+    __syncthreads();
+    const uint32_t lane = t & 31u;
+    const uint32_t lrun = (t & ~31u) + ((lane & 3u) << 3) + (lane >> 2);   // as in sssp_kernel
+    for (;;) {
+        if (t == 0) kclaim_a[grp] = claim_group(lc, p.g.nitems, &nout);
+        grp_bar(grp);
+        const uint32_t k = kclaim_a[grp];
+        if (k >= p.g.nitems) break;
+        const Item it = p.g.items[k];
+        const uint32_t lo = p.g.v0 + it.tile * GT, nvt = min(lo + GT, p.g.v0 + p.g.nv) - lo;
+        for (uint32_t i = t; i <= nvt; i += GB) cp[i] = ld_stream_u(p.g.colptr + (lo - p.g.v0 + i), pf);
+        for (uint32_t i = t; i < nvt; i += GB) acc[i] = INT32_MAX;
+        grp_bar(grp);
+        uint32_t xn[RUN], in_ = 0;
+        auto load_idx = [&](uint32_t base) {
+            const uint32_t r0 = base + lrun * RUN;
+#pragma unroll
+            for (int q = 0; q < RUN; ++q) xn[q] = r0 + q < it.e1 ? ld_stream_u(p.g.rowidx_h + r0 + q, pf) : HOT_BIT;
+            in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_ss + it.run_ss + (r0 - it.e0) / RUN, pf) : 0u;
+        };
+        load_idx(it.e0);
+        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+            const uint32_t r0 = base + lrun * RUN;
+            const bool act = r0 < it.e1;
+            uint32_t x[RUN];
+#pragma unroll
+            for (int q = 0; q < RUN; ++q) x[q] = xn[q];
+            uint32_t i = act ? in_ : 0xFFFFFFFFu;
+            if (base + GB * RUN < it.e1) load_idx(base + GB * RUN);
+            int32_t best = INT32_MAX;
+            bool single = false;
+            if (act) {
+                const uint32_t r1 = min(r0 + RUN, it.e1);
+                int32_t c[RUN];
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    int32_t du = INT32_MAX;
+                    if (r0 + q < r1) {
+                        if (x[q] & HOT_BIT) du = hot[x[q] & ~HOT_BIT & 0xFFFFu];
+                        else if (changed_src(x[q])) du = ld_gather_i(din + x[q], pl);
+                    }
+                    c[q] = du;
+                }
+#pragma unroll
+                for (int q = 0; q < RUN; ++q)
+                    if (c[q] != INT32_MAX) {
+                        const int64_t cand = (int64_t)c[q] + (int64_t)ld_stream_i(p.g.w + r0 + q, pf);
+                        c[q] = cand < (int64_t)INT32_MAX ? (int32_t)cand : INT32_MAX;
+                    }
+                uint32_t nxt = cp[i + 1];
+                single = r1 <= nxt;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) {
+                    if (r0 + q >= r1) break;
+                    while (r0 + q >= nxt) {
+                        if (best != INT32_MAX) atomicMin(&acc[i], best);
+                        best = INT32_MAX;
+                        nxt = cp[++i + 1];
+                    }
+                    best = min(best, c[q]);
+                }
+            }
+            const uint32_t i0 = __shfl_sync(0xFFFFFFFFu, i, 0);
+            if (__all_sync(0xFFFFFFFFu, act && single && i == i0)) {
+                best = __reduce_min_sync(0xFFFFFFFFu, best);
+                if (lane == 0 && best != INT32_MAX) atomicMin(&acc[i0], best);
+            } else if (act && best != INT32_MAX) {
+                atomicMin(&acc[i], best);
+            }
+        }
+        grp_bar(grp);
+        bool fin = true;
+        if (it.nsplit > 1) {
+            int32_t *ga = p.g.acc_i + (size_t)it.slot * GT;
+            for (uint32_t i = t; i < nvt; i += GB)
+                if (acc[i] != INT32_MAX) atomicMin(&ga[i], acc[i]);
+            grp_bar(grp);
+            if (t == 0) {
+                __threadfence();
+                const uint32_t old = atomicAdd(&p.g.acc_cnt[it.slot], 1u);
+                __threadfence();
+                last_a[grp] = old + 1 == it.nsplit;
+            }
+            grp_bar(grp);
+            fin = last_a[grp] != 0;
+            if (fin) {
+                for (uint32_t i = t; i < nvt; i += GB) {
+                    acc[i] = __ldcg(&ga[i]);
+                    ga[i] = INT32_MAX;
+                }
+                if (t == 0) p.g.acc_cnt[it.slot] = 0;
+                grp_bar(grp);
+            }
+        }
+        if (fin) {
+            if (t == 0) any_a[grp] = 0u;
+            grp_bar(grp);
+            bool changed = false;
+            for (uint32_t i = t; i < nvt; i += GB) {
+                const uint32_t v = lo + i;
+                const int32_t old = din[v];
+                const int32_t best = min(old, acc[i]);
+                proact::put(lc, p.region_out, (uint64_t)v * 4, best);
+                changed |= best != old;
+            }
+            if (__any_sync(0xFFFFFFFFu, changed) && lane == 0) any_a[grp] = 1u;
+            grp_bar(grp);   // orders the group's puts before the commit (a3)
+            if (t == 0) {   // chunk state as in sssp_kernel
+                const uint64_t off = (uint64_t)lo * 4;
+                const bool any = any_a[grp] != 0u;
+                const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
+                if (any) {
+                    proact::mark_changed(lc, p.region_out, off);
+                    proact::vote(lc);
+                }
+                if (any || prev) proact::mark_push(lc, p.region_out, off);
+                proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
+            }
+        }
+        grp_bar(grp);
+    }
+}
+
 __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t V, float r0)
 {
     for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x)
@@ -626,6 +1086,10 @@ int graph_dev(int id, GraphDev *g)
     g->acc_cnt = G.acc_cnt;
     g->runv_pr = G.runv_pr;
     g->runv_ss = G.runv_ss;
+    g->runv_ph = G.runv_ph;
+    g->rowidx_h = G.rowidx_h ? G.rowidx_h : G.rowidx;   // no table: plain ids (all < HOT_BIT)
+    g->hot_ids = G.hot_ids;
+    g->nhot = G.nhot;
     g->V = G.V;
     g->v0 = G.v0;
     g->nv = G.nv;
@@ -677,7 +1141,18 @@ int proact_partition_bounds(const uint32_t *indeg, unsigned V, int G, unsigned a
 int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w, unsigned long long E,
                        unsigned V, unsigned v0, unsigned v1, void *stream)
 {
-    if (((!d_src || !d_dst) && E) || v1 < v0 || v1 > V) return PROACT_ERR_INVALID;
+    return proact_graph_build_ex(d_src, d_dst, d_w, E, V, v0, v1, -1, stream);
+}
+
+int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w, unsigned long long E,
+                          unsigned V, unsigned v0, unsigned v1, int hot, void *stream)
+{
+    if (((!d_src || !d_dst) && E) || v1 < v0 || v1 > V || V >= HOT_BIT) return PROACT_ERR_INVALID;
+    if (hot < 0) {
+        const char *e = getenv("PROACT_GRAPH_HOT");
+        hot = e ? atoi(e) : (int)HOT_DEFAULT;
+    }
+    if ((uint32_t)hot > HOT_MAX) hot = (int)HOT_MAX;
     int id = -1;
     for (int k = 0; k < MAXGRAPH; ++k)
         if (!graphs[k].used) { id = k; break; }
@@ -731,21 +1206,25 @@ int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32
         }
         split.insert(split.end(), whole.begin(), whole.end());   // big (hub) work first
         G.nitems = (uint32_t)split.size();
-        uint64_t npr = 0, nss = 0;
+        uint64_t npr = 0, nss = 0, nph = 0;
         for (Item &it : split) {
             it.run_pr = (uint32_t)npr;
             it.run_ss = (uint32_t)nss;
+            it.run_ph = (uint32_t)nph;
             npr += (it.e1 - it.e0 + PROACT_PR_RUN - 1) / PROACT_PR_RUN;
             nss += (it.e1 - it.e0 + PROACT_SSSP_RUN - 1) / PROACT_SSSP_RUN;
+            nph += (it.e1 - it.e0 + PROACT_PRH_RUN - 1) / PROACT_PRH_RUN;
         }
-        if (npr >= (1ull << 32) || nss >= (1ull << 32)) return PROACT_ERR_NOMEM;
+        if (npr >= (1ull << 32) || nss >= (1ull << 32) || nph >= (1ull << 32)) return PROACT_ERR_NOMEM;
         GCK(cudaMalloc((void **)&G.items, sizeof(Item) * std::max<size_t>(1, split.size())));
         GCK(cudaMemcpy(G.items, split.data(), sizeof(Item) * split.size(), cudaMemcpyHostToDevice));
         GCK(cudaMalloc((void **)&G.runv_pr, 2 * std::max<uint64_t>(1, npr)));
         GCK(cudaMalloc((void **)&G.runv_ss, 2 * std::max<uint64_t>(1, nss)));
+        GCK(cudaMalloc((void **)&G.runv_ph, 2 * std::max<uint64_t>(1, nph)));
         if (G.nitems) {
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PR_RUN, 0, G.runv_pr);
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_SSSP_RUN, 1, G.runv_ss);
+            runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN, 2, G.runv_ph);
             GCK(cudaGetLastError());
         }
         const size_t ns = std::max<uint32_t>(1, G.nslot);
@@ -760,7 +1239,40 @@ int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32
         GCK(cudaMalloc((void **)&G.acc_cnt, 4 * ns));
         GCK(cudaMemset(G.acc_cnt, 0, 4 * ns));
     }
+    // hot sources: the `hot` highest out-degree vertices (ties: smaller id), ascending ids
+    if (hot > 0 && G.E_own > 0) {
+        std::vector<uint32_t> od(V);
+        GCK(cudaMemcpyAsync(od.data(), G.outdeg, 4 * (size_t)V, cudaMemcpyDeviceToHost, s));
+        GCK(cudaStreamSynchronize(s));
+        std::vector<uint32_t> ids;
+        ids.reserve(V);
+        for (uint32_t v = 0; v < V; ++v)
+            if (od[v]) ids.push_back(v);
+        const size_t H = std::min<size_t>((size_t)hot, ids.size());
+        auto hotter = [&](uint32_t a, uint32_t b) { return od[a] != od[b] ? od[a] > od[b] : a < b; };
+        if (H < ids.size()) std::nth_element(ids.begin(), ids.begin() + H, ids.end(), hotter);
+        ids.resize(H);
+        std::sort(ids.begin(), ids.end());
+        G.nhot = (uint32_t)H;
+        if (H) {
+            uint32_t *slot = nullptr;
+            GCK(cudaMalloc((void **)&G.hot_ids, 4 * H));
+            GCK(cudaMemcpy(G.hot_ids, ids.data(), 4 * H, cudaMemcpyHostToDevice));
+            GCK(cudaMalloc((void **)&slot, 4 * (size_t)V));
+            GCK(cudaMemsetAsync(slot, 0xFF, 4 * (size_t)V, s));
+            hot_slot_kernel<<<(unsigned)((H + 255) / 256), 256, 0, s>>>(G.hot_ids, (uint32_t)H, slot);
+            GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 1)));
+            hot_encode_kernel<<<1184, 256, 0, s>>>(G.rowidx, G.E_own, slot, G.rowidx_h);
+            GCK(cudaGetLastError());
+            GCK(cudaStreamSynchronize(s));
+            GCK(cudaFree(slot));
+        }
+    }
     GCK(cudaStreamSynchronize(s));
+    GCK(cudaFuncSetAttribute((const void *)pagerank_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(4 * (PG * CPS + HOT_MAX))));
+    GCK(cudaFuncSetAttribute((const void *)sssp_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(4 * (PG * CPS + HOT_MAX)) - (int)(4 * CHG_WORDS)));
     G.used = true;
     graphs[id] = G;
     return id;
@@ -781,6 +1293,9 @@ int proact_graph_free(int id)
     cudaFree(G.acc_cnt);
     cudaFree(G.runv_pr);
     cudaFree(G.runv_ss);
+    cudaFree(G.runv_ph);
+    if (G.rowidx_h) cudaFree(G.rowidx_h);
+    if (G.hot_ids) cudaFree(G.hot_ids);
     G = Graph();
     return PROACT_OK;
 }
@@ -791,6 +1306,13 @@ int proact_graph_info(int id, unsigned long long *e_own, unsigned *v0, unsigned 
     if (e_own) *e_own = graphs[id].E_own;
     if (v0) *v0 = graphs[id].v0;
     if (nv) *nv = graphs[id].nv;
+    return PROACT_OK;
+}
+
+int proact_graph_hot(int id, unsigned *nhot)
+{
+    if (id < 0 || id >= MAXGRAPH || !graphs[id].used || !nhot) return PROACT_ERR_INVALID;
+    *nhot = graphs[id].nhot;
     return PROACT_OK;
 }
 
@@ -826,6 +1348,13 @@ int proact_pagerank_phase(int graph, int region_in, int region_out, double dampi
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
+    static const int plain = [] {
+        const char *e = getenv("PROACT_PR_KERNEL");
+        return e && !strcmp(e, "plain") ? 1 : 0;
+    }();
+    if (!plain)
+        return proact_launch(regs, 1, (const void *)pagerank_hot_kernel, 0, GB * PG, args,
+                             4 * ((size_t)PG * CPS + p.g.nhot), stream);
     return proact_launch(regs, 1, (const void *)pagerank_kernel, 0, GB, args, 0, stream);
 }
 
@@ -858,6 +1387,9 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
+    if (p.g.nhot && p.g.nhot <= HOT_MAX - CHG_WORDS)   // hot table (room for the changed bitmap)
+        return proact_launch(regs, 1, (const void *)sssp_hot_kernel, 0, GB * PG, args,
+                             4 * ((size_t)PG * CPS + p.g.nhot), stream);
     return proact_launch(regs, 1, (const void *)sssp_kernel, 0, GB, args, 0, stream);
 }
 
@@ -867,7 +1399,9 @@ __attribute__((visibility("hidden"))) int proact_internal_preload_graph(void)
     cudaFuncAttributes a;
     const void *k[] = {(const void *)count_kernel, (const void *)scan_blocks, (const void *)scan_totals,
                        (const void *)scan_add, (const void *)scatter_kernel, (const void *)pagerank_kernel,
-                       (const void *)sssp_kernel, (const void *)pr_init_kernel, (const void *)runv_kernel};
+                       (const void *)sssp_kernel, (const void *)pr_init_kernel, (const void *)runv_kernel,
+                       (const void *)pagerank_hot_kernel, (const void *)hot_slot_kernel,
+                       (const void *)hot_encode_kernel, (const void *)sssp_hot_kernel};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
     return PROACT_OK;

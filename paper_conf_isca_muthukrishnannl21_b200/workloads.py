@@ -196,7 +196,7 @@ def _u32_dev(a) -> torch.Tensor:
 class _Graph:
     """Edge list -> this rank's destination partition + in-edge CSC (library-owned)."""
 
-    def __init__(self, V: int, src, dst, w, chunk_bytes: int, stream=None):
+    def __init__(self, V: int, src, dst, w, chunk_bytes: int, stream=None, hot: int = -1):
         G, g = rt.world(), rt.rank()
         self.V = V
         s = _s(stream)
@@ -208,10 +208,13 @@ class _Graph:
                                                bounds, s), "graph_partition")
         self.bounds = list(bounds)
         self.v0, self.v1 = self.bounds[g], self.bounds[g + 1]
-        self.gid = check(rt.lib().proact_graph_build(
+        self.gid = check(rt.lib().proact_graph_build_ex(
             ctypes.c_void_p(d_src.data_ptr()), ctypes.c_void_p(d_dst.data_ptr()),
-            ctypes.c_void_p(d_w.data_ptr() if d_w is not None else 0), E, V, self.v0, self.v1, s),
+            ctypes.c_void_p(d_w.data_ptr() if d_w is not None else 0), E, V, self.v0, self.v1, hot, s),
             "graph_build")
+        nh = ctypes.c_uint(0)
+        check(rt.lib().proact_graph_hot(self.gid, ctypes.byref(nh)), "graph_hot")
+        self.nhot = nh.value
         e_own = ctypes.c_ulonglong(0)
         check(rt.lib().proact_graph_info(self.gid, ctypes.byref(e_own), None, None), "graph_info")
         self.e_own = e_own.value
@@ -226,8 +229,9 @@ class _Graph:
 class PageRank(_Graph):
     """Destination-partitioned PageRank over a replicated contrib = r/out vector (config 3)."""
 
-    def __init__(self, V: int, src, dst, chunk_bytes: int, damping: float = 0.85, stream=None):
-        super().__init__(V, src, dst, None, chunk_bytes, stream)
+    def __init__(self, V: int, src, dst, chunk_bytes: int, damping: float = 0.85, stream=None, hot: int = -1):
+        """hot: size of the shared-memory hot-source table (-1 library default, 0 none)."""
+        super().__init__(V, src, dst, None, chunk_bytes, stream, hot)
         self.d = damping
         self.bufs = [torch.zeros(V, dtype=torch.float32, device="cuda") for _ in range(2)]
         torch.cuda.synchronize()
@@ -255,8 +259,9 @@ INF32 = 2**31 - 1
 class SSSP(_Graph):
     """Synchronous Bellman-Ford over a replicated int32 distance vector, SPARSE regions (config 4)."""
 
-    def __init__(self, V: int, src, dst, w, source: int, chunk_bytes: int, stream=None):
-        super().__init__(V, src, dst, w, chunk_bytes, stream)
+    def __init__(self, V: int, src, dst, w, source: int, chunk_bytes: int, stream=None, hot: int = -1):
+        """hot: size of the shared-memory hot-source table (-1 library default, 0 none)."""
+        super().__init__(V, src, dst, w, chunk_bytes, stream, hot)
         self.bufs = []
         for _ in range(2):
             b = torch.full((V,), INF32, dtype=torch.int32, device="cuda")

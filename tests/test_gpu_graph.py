@@ -18,10 +18,10 @@ from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
 pytestmark = pytest.mark.gpu
 
 
-def _pr_body(r, G, V, src, dst, iters, chunk, mech):
+def _pr_body(r, G, V, src, dst, iters, chunk, mech, hot=-1):
     rt.set_config(mech=mech)
     s = torch.cuda.Stream()
-    P = wl.PageRank(V, src, dst, chunk, stream=s)
+    P = wl.PageRank(V, src, dst, chunk, stream=s, hot=hot)
     for k in range(iters):
         P.step(s, barrier=(k == iters - 1))
     s.synchronize()
@@ -31,14 +31,21 @@ def _pr_body(r, G, V, src, dst, iters, chunk, mech):
     return P.v0, P.v1, out
 
 
-@pytest.mark.parametrize("G,scale,chunk,mech", [(1, 12, 4096, _lib.MECH_FUSED), (2, 13, 8192, _lib.MECH_FUSED),
-                                                (3, 12, 4096, _lib.MECH_FUSED), (2, 12, 16384, _lib.MECH_INLINE),
-                                                (2, 12, 4096, _lib.MECH_BULK), (4, 14, 65536, _lib.MECH_FUSED)])
-def test_pagerank_matches_oracle(G, scale, chunk, mech):
+# hot: -1 = library default (8192: nearly every source with out-edges fits the table at these
+# sizes), 0 = no table (pagerank_kernel), 97 = a partial table (both read paths in one warp)
+@pytest.mark.parametrize("G,scale,chunk,mech,hot", [(1, 12, 4096, _lib.MECH_FUSED, -1),
+                                                    (1, 12, 4096, _lib.MECH_FUSED, 0),
+                                                    (2, 13, 8192, _lib.MECH_FUSED, 97),
+                                                    (2, 13, 8192, _lib.MECH_FUSED, -1),
+                                                    (3, 12, 4096, _lib.MECH_FUSED, 0),
+                                                    (2, 12, 16384, _lib.MECH_INLINE, 97),
+                                                    (2, 12, 4096, _lib.MECH_BULK, -1),
+                                                    (4, 14, 65536, _lib.MECH_FUSED, 1000)])
+def test_pagerank_matches_oracle(G, scale, chunk, mech, hot):
     src, dst = synth.rmat(scale, 16)
     V, iters = 1 << scale, 20
     want = oracle.pagerank(V, src, dst, iters).astype(np.float64)
-    outs = run_ranks(G, _pr_body, V, src, dst, iters, chunk, mech)
+    outs = run_ranks(G, _pr_body, V, src, dst, iters, chunk, mech, hot)
     got = np.zeros(V)
     covered = 0
     for v0, v1, r in outs:
@@ -49,10 +56,20 @@ def test_pagerank_matches_oracle(G, scale, chunk, mech):
     assert rel.max() <= 1e-5, rel.max()
 
 
-def _sssp_body(r, G, V, src, dst, w, s0, chunk, mech):
+def test_pagerank_hot_table_is_bit_identical():
+    """The hot-source table changes where contributions are read, not the (exact fixed-point)
+    sums: r' is bit-identical with no table, a partial table and the default table."""
+    src, dst = synth.rmat(16, 16)
+    V = 1 << 16
+    got = [run_ranks(1, _pr_body, V, src, dst, 5, 4096, _lib.MECH_FUSED, hot)[0][2] for hot in (0, 333, -1)]
+    assert np.array_equal(got[0].view(np.uint32), got[1].view(np.uint32))
+    assert np.array_equal(got[0].view(np.uint32), got[2].view(np.uint32))
+
+
+def _sssp_body(r, G, V, src, dst, w, s0, chunk, mech, hot=-1):
     rt.set_config(mech=mech)
     st = torch.cuda.Stream()
-    S = wl.SSSP(V, src, dst, w, s0, chunk, stream=st)
+    S = wl.SSSP(V, src, dst, w, s0, chunk, stream=st, hot=hot)
     rounds = S.run(stream=st)
     rt.check_device()
     d = S.current.cpu().numpy().copy()
@@ -60,16 +77,22 @@ def _sssp_body(r, G, V, src, dst, w, s0, chunk, mech):
     return rounds, d, S.v0, S.v1
 
 
-@pytest.mark.parametrize("G,scale,chunk,mech", [(1, 12, 4096, _lib.MECH_FUSED), (2, 13, 4096, _lib.MECH_FUSED),
-                                                (3, 12, 8192, _lib.MECH_FUSED), (2, 12, 4096, _lib.MECH_INLINE),
-                                                (2, 12, 4096, _lib.MECH_BULK), (4, 14, 16384, _lib.MECH_FUSED)])
-def test_sssp_matches_oracle(G, scale, chunk, mech):
+# hot as in test_pagerank_matches_oracle (0: sssp_kernel, else sssp_hot_kernel)
+@pytest.mark.parametrize("G,scale,chunk,mech,hot", [(1, 12, 4096, _lib.MECH_FUSED, -1),
+                                                    (1, 12, 4096, _lib.MECH_FUSED, 0),
+                                                    (2, 13, 4096, _lib.MECH_FUSED, 97),
+                                                    (2, 13, 4096, _lib.MECH_FUSED, 0),
+                                                    (3, 12, 8192, _lib.MECH_FUSED, -1),
+                                                    (2, 12, 4096, _lib.MECH_INLINE, 97),
+                                                    (2, 12, 4096, _lib.MECH_BULK, -1),
+                                                    (4, 14, 16384, _lib.MECH_FUSED, 1000)])
+def test_sssp_matches_oracle(G, scale, chunk, mech, hot):
     src, dst = synth.rmat(scale, 16)
     V = 1 << scale
     w = synth.weights(src.size)
     s0 = int(np.bincount(src, minlength=V).argmax())
     want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
-    outs = run_ranks(G, _sssp_body, V, src, dst, w, s0, chunk, mech)
+    outs = run_ranks(G, _sssp_body, V, src, dst, w, s0, chunk, mech, hot)
     for rounds, d, v0, v1 in outs:
         assert rounds == want_rounds
         # owned slice always exact; full replica exact under FUSED/INLINE/BULK replication
