@@ -101,8 +101,9 @@ int proact_graph_build(const uint32_t *d_src, const uint32_t *d_dst, const int32
  * The result is bit-identical either way (exact fixed-point sums).  V < 2^31. */
 int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const int32_t *d_w,
                           unsigned long long E, unsigned V, unsigned v0, unsigned v1, int hot, void *stream);
-/* Number of hot sources of a graph (0: none). */
-int proact_graph_hot(int graph, unsigned *nhot);
+/* Number of hot sources of a graph (0: none) and of my in-edges whose source is hot (either
+ * pointer may be NULL). */
+int proact_graph_hot(int graph, unsigned *nhot, unsigned long long *e_hot);
 int proact_graph_free(int graph);
 int proact_graph_info(int graph, unsigned long long *e_own, unsigned *v0, unsigned *nv);
 

@@ -109,7 +109,7 @@ def _declare(L):
                                    ctypes.c_uint, vp]),
         "proact_graph_build_ex": (i, [vp, vp, vp, ctypes.c_ulonglong, ctypes.c_uint, ctypes.c_uint,
                                       ctypes.c_uint, i, vp]),
-        "proact_graph_hot": (i, [i, ctypes.POINTER(ctypes.c_uint)]),
+        "proact_graph_hot": (i, [i, ctypes.POINTER(ctypes.c_uint), ctypes.POINTER(ctypes.c_ulonglong)]),
         "proact_graph_free": (i, [i]),
         "proact_graph_info": (i, [i, ctypes.POINTER(ctypes.c_ulonglong), ctypes.POINTER(ctypes.c_uint),
                                   ctypes.POINTER(ctypes.c_uint)]),

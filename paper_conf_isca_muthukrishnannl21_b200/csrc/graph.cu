@@ -101,6 +101,7 @@ struct Graph {
     uint16_t *runv_pr = nullptr, *runv_ss = nullptr, *runv_ph = nullptr;
     uint32_t *rowidx_h = nullptr, *hot_ids = nullptr;
     uint32_t nhot = 0;
+    uint64_t e_hot = 0;   // my in-edges whose source is hot
 };
 constexpr int MAXGRAPH = 4;
 
@@ -122,8 +123,8 @@ constexpr uint32_t HOT_DEFAULT = 8192;
 #ifndef PROACT_PRH_SEGRED   // warp segmented reduction instead of per-run atomics: measured slower
 #define PROACT_PRH_SEGRED 0   // (1.31 vs 1.20 ms at RMAT-24; the shared atomics are not the bound)
 #endif
-#ifndef PROACT_PRH_MINB      // hot-kernel CTAs per SM (register budget 64 / 32 per thread at 1 / 2)
-#define PROACT_PRH_MINB 1
+#ifndef PROACT_PRH_MINB      // pagerank_hot_kernel CTAs per SM (64 / 32 registers per thread at 1 / 2):
+#define PROACT_PRH_MINB 2     // 1.153 ms at 2 vs 1.176 ms at 1 (RMAT-24, hot = 8192)
 #endif
 #ifndef PROACT_SSH_MINB      // sssp_hot_kernel CTAs per SM
 #define PROACT_SSH_MINB 2
@@ -248,12 +249,16 @@ __global__ void hot_slot_kernel(const uint32_t *hot_ids, uint32_t nhot, uint32_t
     for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < nhot; s += gridDim.x * blockDim.x)
         slot[hot_ids[s]] = s;
 }
-__global__ void hot_encode_kernel(const uint32_t *rowidx, uint64_t E, const uint32_t *slot, uint32_t *out)
+__global__ void hot_encode_kernel(const uint32_t *rowidx, uint64_t E, const uint32_t *slot, uint32_t *out,
+                                  unsigned long long *nhot_edges)
 {
+    uint32_t n = 0;
     for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t u = rowidx[e], k = slot[u];
         out[e] = k != 0xFFFFFFFFu ? (HOT_BIT | k) : u;
+        n += k != 0xFFFFFFFFu;
     }
+    atomicAdd(nhot_edges, (unsigned long long)n);
 }
 
 // ------------------------------------------------------------------ phase kernels
@@ -304,8 +309,8 @@ __device__ __forceinline__ int32_t ld_stream_i(const int32_t *p, uint64_t pol)
 // The gathered vector: written by peers' agents during the previous phase (all arrived: the CTA
 // waited with wait_all before its first load, and nothing rewrites it this phase), so the
 // read-only path is coherent here.
-#ifndef PROACT_GATHER_MODE   // 0: .nc; 1: .nc + L1::no_allocate; 2: .cg (L2 only)
-#define PROACT_GATHER_MODE 0
+#ifndef PROACT_GATHER_MODE   // 0: .nc; 1: .nc + L1::no_allocate; 2: .cg (L2 only).  1 and 2: -2 %
+#define PROACT_GATHER_MODE 1  // PageRank, -6 % SSSP at RMAT-24 (tools/sweep_pagerank.py, sweep_graph.py)
 #endif
 #if PROACT_GATHER_MODE == 1
 #define GATHER_OP "ld.global.nc.L1::no_allocate.L2::cache_hint"
@@ -1262,9 +1267,16 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
             GCK(cudaMemsetAsync(slot, 0xFF, 4 * (size_t)V, s));
             hot_slot_kernel<<<(unsigned)((H + 255) / 256), 256, 0, s>>>(G.hot_ids, (uint32_t)H, slot);
             GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 1)));
-            hot_encode_kernel<<<1184, 256, 0, s>>>(G.rowidx, G.E_own, slot, G.rowidx_h);
+            unsigned long long *neh = nullptr;
+            GCK(cudaMalloc((void **)&neh, 8));
+            GCK(cudaMemsetAsync(neh, 0, 8, s));
+            hot_encode_kernel<<<1184, 256, 0, s>>>(G.rowidx, G.E_own, slot, G.rowidx_h, neh);
             GCK(cudaGetLastError());
+            unsigned long long eh = 0;
+            GCK(cudaMemcpyAsync(&eh, neh, 8, cudaMemcpyDeviceToHost, s));
             GCK(cudaStreamSynchronize(s));
+            G.e_hot = eh;
+            GCK(cudaFree(neh));
             GCK(cudaFree(slot));
         }
     }
@@ -1309,10 +1321,11 @@ int proact_graph_info(int id, unsigned long long *e_own, unsigned *v0, unsigned 
     return PROACT_OK;
 }
 
-int proact_graph_hot(int id, unsigned *nhot)
+int proact_graph_hot(int id, unsigned *nhot, unsigned long long *e_hot)
 {
-    if (id < 0 || id >= MAXGRAPH || !graphs[id].used || !nhot) return PROACT_ERR_INVALID;
-    *nhot = graphs[id].nhot;
+    if (id < 0 || id >= MAXGRAPH || !graphs[id].used) return PROACT_ERR_INVALID;
+    if (nhot) *nhot = graphs[id].nhot;
+    if (e_hot) *e_hot = graphs[id].e_hot;
     return PROACT_OK;
 }
 

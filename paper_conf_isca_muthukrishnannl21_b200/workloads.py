@@ -212,9 +212,9 @@ class _Graph:
             ctypes.c_void_p(d_src.data_ptr()), ctypes.c_void_p(d_dst.data_ptr()),
             ctypes.c_void_p(d_w.data_ptr() if d_w is not None else 0), E, V, self.v0, self.v1, hot, s),
             "graph_build")
-        nh = ctypes.c_uint(0)
-        check(rt.lib().proact_graph_hot(self.gid, ctypes.byref(nh)), "graph_hot")
-        self.nhot = nh.value
+        nh, eh = ctypes.c_uint(0), ctypes.c_ulonglong(0)
+        check(rt.lib().proact_graph_hot(self.gid, ctypes.byref(nh), ctypes.byref(eh)), "graph_hot")
+        self.nhot, self.e_hot = nh.value, eh.value
         e_own = ctypes.c_ulonglong(0)
         check(rt.lib().proact_graph_info(self.gid, ctypes.byref(e_own), None, None), "graph_info")
         self.e_own = e_own.value

@@ -78,7 +78,8 @@ def pagerank(args, src, dst, V):
             ks.append((a, b))
         torch.cuda.synchronize()
         kms = statistics.median(a.elapsed_time(b) for a, b in ks)
-        out = {"ms": ms, "kms": kms, "e_own": P.e_own, "nv": P.v1 - P.v0, "iters": args.steps * I}
+        out = {"ms": ms, "kms": kms, "e_own": P.e_own, "nv": P.v1 - P.v0, "iters": args.steps * I,
+               "nhot": P.nhot, "e_hot": P.e_hot}
         P.free()
         return out
     res = run_ranks(args.ranks, body)
@@ -88,19 +89,21 @@ def pagerank(args, src, dst, V):
     line = {"workload": f"pagerank_rmat{args.scale}_ef16_20it (BASELINE.json config 3)",
             "value": res[0]["iters"] / (ms / 1000.0), "unit": "iters/s", "ranks": args.ranks,
             "mech": args.mech, "chunk_bytes": args.chunk, "edges": int(src.size),
-            "roofline": {"bound": "hbm", "kernel": "pagerank_kernel", "kernel_ms": kms,
+            "roofline": {"bound": "hbm", "kernel": "pagerank_hot_kernel" if res[0]["nhot"] else "pagerank_kernel",
+                         "kernel_ms": kms, "hot_sources": res[0]["nhot"], "hot_edge_frac": res[0]["e_hot"] / max(1, res[0]["e_own"]),
                          "alg_bytes_per_launch": alg, "achieved": alg / kms / 1e6, "peak": peak_hbm(),
                          "unit": "GB/s", "frac": alg / kms / 1e6 / peak_hbm(),
                          "note": "8 B/edge (index + gathered contrib) + 16 B/vertex; gathers hit L2"}}
-    # the bound that actually applies: every random 4-byte gather is one L1TEX
-    # wavefront, one per clock per SM -> t >= E_own / (SMs x SM clock)
+    # the bound that actually applies: every random 4-byte gather from global
+    # memory is one L1TEX wavefront / L1->L2 request, one per clock per SM -> t >= gathers /
+    # (SMs x SM clock); in-edges of hot sources read shared memory instead
     prop = torch.cuda.get_device_properties(0)
-    e_max = max(r["e_own"] for r in res)
+    e_max = max(r["e_own"] - r["e_hot"] for r in res)
     rate = prop.multi_processor_count * 1965e6          # gathers/s at the max SM clock
     t_l1 = e_max / rate * 1e3
     line["roofline_l1_gather"] = {"bound": "l1tex_wavefronts", "gathers_per_launch": e_max,
                                   "peak_gathers_per_s": rate, "t_min_ms": t_l1, "frac": t_l1 / kms,
-                                  "note": "1 wavefront/clk/SM x SMs x 1965 MHz"}
+                                  "note": "global gathers (in-edges of non-hot sources); 1 wavefront/clk/SM x SMs x 1965 MHz"}
     if not args.no_cpu:
         import oracle
         t0 = time.perf_counter()
@@ -130,7 +133,41 @@ def sssp(args, src, dst, V):
             rounds = S.run(stream=st)
             times.append(time.perf_counter() - t0)
             S.free()
-        return {"rounds": rounds, "t": sum(times[args.warmup:])}
+        # one more run, round by round: the phase kernel's CUDA-event time and its algorithmic
+        # bytes (4 B per in-edge scanned + 8 B per in-edge of a source whose
+        # chunk changed in the previous round + 12 B per vertex), the changed chunks read back
+        # from the distance vectors between rounds (outside the timed kernel)
+        S = wl.SSSP(V, src, dst, w, s0, args.chunk, stream=st)
+        cv = args.chunk // 4
+        nch = (V + cv - 1) // cv
+        prev = S.current.clone()
+        kern, algs, k = [], [], 0
+        dirty = None
+        while True:
+            a, b = ev(), ev()
+            i = S.k & 1
+            a.record(st)
+            _lib.check(rt.lib().proact_sssp_phase(S.gid, S.rid[i], S.rid[i ^ 1], int(S.k == 0), wl._s(st)), "sssp")
+            b.record(st)
+            rt.phase_sync(st, barrier=True)
+            S.k += 1
+            st.synchronize()
+            kern.append(a.elapsed_time(b))
+            de = S.e_own if dirty is None else int(epc[dirty].sum())
+            algs.append(4.0 * S.e_own + 8.0 * de + 12.0 * (S.v1 - S.v0))
+            cur = S.current
+            pad = nch * cv - V
+            diff = torch.nn.functional.pad((cur != prev).to(torch.int32), (0, pad))
+            dirty = (diff.view(nch, cv).sum(1) > 0).cpu().numpy()
+            prev = cur.clone()
+            k += 1
+            if rt.last_vote() == 0 or k >= V:
+                break
+        out = {"rounds": rounds, "t": sum(times[args.warmup:]), "kern_ms": kern, "alg": algs,
+               "nhot": S.nhot, "e_own": S.e_own}
+        S.free()
+        return out
+    epc = np.bincount(src // (args.chunk // 4), minlength=(V + args.chunk // 4 - 1) // (args.chunk // 4))
     res = run_ranks(args.ranks, body)
     t = max(r["t"] for r in res)
     rounds = res[0]["rounds"]
@@ -138,6 +175,15 @@ def sssp(args, src, dst, V):
             "value": args.steps * rounds / t, "unit": "rounds/s", "rounds": rounds, "ranks": args.ranks,
             "mech": args.mech, "chunk_bytes": args.chunk, "edges": int(src.size),
             "timing": "host wall clock per run (a BARRIER + host vote read every round)"}
+    if args.ranks == 1:
+        r0 = res[0]
+        kms, alg = sum(r0["kern_ms"]), sum(r0["alg"])
+        line["roofline"] = {"bound": "hbm", "kernel": "sssp_hot_kernel" if r0["nhot"] else "sssp_kernel",
+                            "kernel_ms_per_round": [round(x, 4) for x in r0["kern_ms"]],
+                            "alg_bytes_per_run": alg, "achieved": alg / kms / 1e6, "peak": peak_hbm(),
+                            "unit": "GB/s", "frac": alg / kms / 1e6 / peak_hbm(),
+                            "note": "4 B/in-edge scanned + 8 B/in-edge of a changed source chunk + 12 B/vertex "
+                                    "per round, summed over the run / summed kernel time"}
     if not args.no_cpu:
         import oracle
         t0 = time.perf_counter()

@@ -31,6 +31,12 @@ def one():
         src, dst = synth.rmat(scale, 16)
         np.savez(cache, src=src, dst=dst)
     V = 1 << scale
+    if os.environ.get("RELABEL"):   # experiment: ids by descending out-degree (stable)
+        od = np.bincount(src, minlength=V)
+        order = np.argsort(-od, kind="stable")
+        new = np.empty(V, np.uint32)
+        new[order] = np.arange(V, dtype=np.uint32)
+        src, dst = new[src], new[dst]
     s = torch.cuda.Stream()
     P = wl.PageRank(V, src, dst, 131072, stream=s)
     ts = []
@@ -45,7 +51,7 @@ def one():
         ts.append((a, b))
     torch.cuda.synchronize()
     pr = statistics.median(a.elapsed_time(b) for a, b in ts[3:])
-    print(f"lib={os.environ.get('PROACT_LIB', 'default')} hot={os.environ.get('PROACT_GRAPH_HOT', '-')} "
+    print(f"relabel={os.environ.get('RELABEL', '')} lib={os.environ.get('PROACT_LIB', 'default')} hot={os.environ.get('PROACT_GRAPH_HOT', '-')} "
           f"kernel={os.environ.get('PROACT_PR_KERNEL', 'hot')} nhot={P.nhot}: pagerank {pr:.4f} ms", flush=True)
     P.free()
     rt.finalize()
