@@ -347,8 +347,13 @@ __device__ __forceinline__ bool local_changed(const launch_ctx &lc, int r, uint6
     const region_dev &R = lc.ctx->region[r];
     return R.changed_gen[(off - R.own_off) / R.chunk_bytes] == lc.gen[r];
 }
-/* Phase vote (e.g. "something changed"): OR-ed over all ranks by a BARRIER phase_sync. */
-__device__ __forceinline__ void vote(const launch_ctx &lc) { atomicOr(&lc.ctx->vote[lc.epoch & 1u], 1u); }
+/* Phase vote (e.g. "something changed"): OR-ed over all ranks by a BARRIER phase_sync.  The
+ * word is tagged with the epoch (epoch + 1 marks a vote cast in `epoch`), so a slot never needs
+ * clearing: a stale tag from an earlier epoch simply does not match. */
+__device__ __forceinline__ void vote(const launch_ctx &lc)
+{
+    atomicMax(&lc.ctx->vote[lc.epoch & 1u], lc.epoch + 1u);
+}
 
 /* ---------------------------------------------------------------- consumer side (a7) ------- */
 

@@ -453,7 +453,7 @@ __global__ void sync_kernel(const dev_ctx *C, uint32_t epoch, int mode)
 {
     // (a8) credit peers "rank finished phase `epoch`" and optionally wait for everyone (L125)
     const uint32_t lane = threadIdx.x;
-    uint32_t myvote = C->vote[epoch & 1u] ? 1u : 0u;
+    uint32_t myvote = C->vote[epoch & 1u] == epoch + 1u ? 1u : 0u;   // epoch-tagged (proact::vote)
     proact::fence_acq_rel_sys();
     uint32_t val = ((epoch + 1u) << 1) | myvote;
     for (int p = lane; p < C->world; p += 32) {
@@ -474,7 +474,6 @@ __global__ void sync_kernel(const dev_ctx *C, uint32_t epoch, int mode)
         any = __any_sync(0xFFFFFFFFu, any);
         if (lane == 0) *(volatile uint32_t *)C->vote_host = ((epoch + 1u) << 1) | any;
     }
-    if (lane == 0) C->vote[epoch & 1u] = 0u;
 }
 
 __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t mask)
@@ -1108,14 +1107,17 @@ int proact_phase_sync(void *stream, int mode)
             }
         }
     }
-    if (c->world == 1 && mode == PROACT_SYNC_SIGNAL && !env_int("PROACT_SYNC_KERNEL", 0)) {
-        // a single rank has no peer to credit: two stream memory writes (my own credit, the
-        // vote word of this epoch cleared for epoch + 2) instead of a kernel launch
-        int mrc = load_memops();
-        if (mrc) return mrc;
-        if (g_write32((CUstream)s, (CUdeviceptr)c->h.done, (c->epoch + 1u) << 1, 0) != CUDA_SUCCESS ||
-            g_write32((CUstream)s, (CUdeviceptr)(c->h.vote + (c->epoch & 1u)), 0u, 0) != CUDA_SUCCESS)
-            return PROACT_ERR_CUDA;
+    static const int sync_mode = env_int("PROACT_SYNC_KERNEL", 0);   // 1: kernel, 2: memory writes
+    if (c->world == 1 && mode == PROACT_SYNC_SIGNAL && sync_mode != 1) {
+        // a single rank has no peer to credit and nobody reads its own credit before the next
+        // BARRIER sync (which writes it), and votes are epoch-tagged: nothing to enqueue.  (The
+        // two stream memory writes this used to be cost ~10 us per phase, tools/probes/phase_gaps.py.)
+        if (sync_mode == 2) {
+            int mrc = load_memops();
+            if (mrc) return mrc;
+            if (g_write32((CUstream)s, (CUdeviceptr)c->h.done, (c->epoch + 1u) << 1, 0) != CUDA_SUCCESS)
+                return PROACT_ERR_CUDA;
+        }
     } else {
         sync_kernel<<<1, 32, 0, s>>>(c->d, c->epoch, mode);
         CK(cudaGetLastError());

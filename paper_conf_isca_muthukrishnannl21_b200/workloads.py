@@ -262,14 +262,26 @@ class SSSP(_Graph):
     def __init__(self, V: int, src, dst, w, source: int, chunk_bytes: int, stream=None, hot: int = -1):
         """hot: size of the shared-memory hot-source table (-1 library default, 0 none)."""
         super().__init__(V, src, dst, w, chunk_bytes, stream, hot)
-        self.bufs = []
-        for _ in range(2):
-            b = torch.full((V,), INF32, dtype=torch.int32, device="cuda")
-            b[source] = 0
-            self.bufs.append(b)
+        self.source = source
+        self.bufs = [torch.empty(V, dtype=torch.int32, device="cuda") for _ in range(2)]
+        self._init_bufs()
         torch.cuda.synchronize()
         self.rid = [rt.register_region(b, self.v0 * 4, (self.v1 - self.v0) * 4, chunk_bytes,
                                        flags=_lib.REGION_SPARSE) for b in self.bufs]
+        self.k = 0
+
+    def _init_bufs(self):
+        for b in self.bufs:
+            b.fill_(INF32)
+            b[self.source] = 0
+
+    def reset(self) -> None:
+        """Back to round 0 (d = INF except the source) on the same graph and regions.  Every rank
+        calls it between runs, after a phase with a BARRIER sync (run() ends with one) and before
+        any rank starts the next run (the caller's host barrier)."""
+        torch.cuda.synchronize()
+        self._init_bufs()
+        torch.cuda.synchronize()
         self.k = 0
 
     def step(self, stream=None) -> bool:

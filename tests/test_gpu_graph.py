@@ -155,3 +155,65 @@ def test_graph_without_edges():
     d_want, rounds_want, _ = oracle.sssp(V, src, dst, np.zeros(0, np.int32), 5)
     for rounds, d, _, _ in outs:
         assert rounds == rounds_want and np.array_equal(d, d_want)
+
+
+def _sssp_rerun_body(r, G, V, src, dst, w, s0, chunk):
+    rt.set_config(mech=_lib.MECH_FUSED)
+    st = torch.cuda.Stream()
+    S = wl.SSSP(V, src, dst, w, s0, chunk, stream=st)
+    out = []
+    for _ in range(2):
+        S.reset()
+        rt.host_barrier()
+        rounds = S.run(stream=st)
+        out.append((rounds, S.current.cpu().numpy().copy()))
+    rt.check_device()
+    S.free()
+    return out
+
+
+def test_sssp_reset_reruns_identically():
+    """SSSP.reset() restarts on the same graph and regions (the bench reuses one build)."""
+    src, dst = synth.rmat(12, 16)
+    V = 1 << 12
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
+    for runs in run_ranks(2, _sssp_rerun_body, V, src, dst, w, s0, 4096):
+        for rounds, d in runs:
+            assert rounds == want_rounds and np.array_equal(d, want)
+
+
+def test_votes_are_epoch_tagged():
+    """A vote cast in a SIGNAL phase must not leak into a later BARRIER phase that reuses its
+    vote slot (epoch + 2): single-rank SIGNAL syncs enqueue nothing, so the slot is never
+    cleared and the epoch tag decides (proact::vote)."""
+    V = 4096
+    src = np.zeros(64, np.uint32)                    # source 0 -> vertices 1..64: one hop
+    dst = np.arange(1, 65, dtype=np.uint32)
+    w = np.ones(64, np.int32)
+
+    def body(r, G):
+        rt.set_config(mech=_lib.MECH_FUSED)
+        st = torch.cuda.Stream()
+        S = wl.SSSP(V, src, dst, w, 0, 4096, stream=st)
+        votes = []
+        for barrier in (False, False, True):   # epochs e (vote), e+1 (none), e+2 (none, BARRIER)
+            i = S.k & 1
+            _lib.check(rt.lib().proact_sssp_phase(S.gid, S.rid[i], S.rid[i ^ 1], int(S.k == 0), wl._s(st)), "sssp")
+            rt.phase_sync(st, barrier=barrier)
+            S.k += 1
+        st.synchronize()
+        votes.append(rt.last_vote())
+        S.reset()                                  # control: the voting phase itself with BARRIER
+        _lib.check(rt.lib().proact_sssp_phase(S.gid, S.rid[0], S.rid[1], 1, wl._s(st)), "sssp")
+        rt.phase_sync(st, barrier=True)
+        S.k += 1
+        st.synchronize()
+        votes.append(rt.last_vote())
+        rt.check_device()
+        S.free()
+        return votes
+
+    (votes,) = run_ranks(1, body)
+    assert votes == [0, 1]
