@@ -895,8 +895,13 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     const unsigned agent_block = separate ? 256u : block;
     unsigned wpc = cfg.push == PROACT_PUSH_BULK ? 1 : agent_block / 32;
     unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
+    // at most half of this rank's share of the SMs hosts agent CTAs: beyond that the producer
+    // starves (loopback G = 2, 96 agent warps: 7.8 ms per microbenchmark phase instead of 0.76,
+    // tools/sweep_micro.py; one rank, 128 idle agent warps: 2x the producer time)
+    const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / (2u * (unsigned)std::max(1, c->ranks_on_device)));
+    agent_ctas = std::min(agent_ctas, agent_cap);
     if (agent && !separate && cfg.push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
-    lc.agent_warps = (uint16_t)(agent ? cfg.agent_warps : 0);
+    lc.agent_warps = (uint16_t)(agent ? std::min<unsigned>(cfg.agent_warps, agent_ctas * wpc) : 0);
     int nb = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
     if (nb < 1) return PROACT_ERR_INVALID;
