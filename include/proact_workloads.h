@@ -72,7 +72,9 @@ typedef struct proact_banded_params {
  * add, IEEE division.  region_in / region_out: two registered N-float replicas with identical
  * whole-row slices (rank g owns rows [own_offset/4, (own_offset+own_bytes)/4)); a / b: device
  * arrays of the full system (only my rows are read).  Waits for the peers' rows within w of my
- * slice.  w <= 8192.  INVALID on geometry mismatch. */
+ * slice.  w <= 8192.  INVALID on geometry mismatch.  With w <= 4096 and 16-byte aligned a / b
+ * the TMA-fed banded_tma_kernel runs (bulk copies of contiguous diagonal slices), otherwise
+ * banded_kernel; both give the same bits. */
 int proact_banded_phase(int region_in, int region_out, const float *a, const float *b, long long N,
                         long long w, void *stream);
 

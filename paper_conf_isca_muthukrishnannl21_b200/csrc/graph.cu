@@ -1076,6 +1076,20 @@ __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t 
         contrib[u] = outdeg[u] ? __fdiv_rn(r0, (float)outdeg[u]) : 0.f;
 }
 
+}  // namespace
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_l2_window(const void *base, size_t bytes);
+namespace {
+
+// PROACT_L2_WINDOW=1: mark the gathered replica persisting in L2 for the phase launch
+int l2_window_on()
+{
+    static const int on = [] {
+        const char *e = getenv("PROACT_L2_WINDOW");
+        return e ? atoi(e) : 0;
+    }();
+    return on;
+}
+
 int graph_dev(int id, GraphDev *g)
 {
     if (id < 0 || id >= MAXGRAPH || !graphs[id].used) return PROACT_ERR_INVALID;
@@ -1365,6 +1379,11 @@ int proact_pagerank_phase(int graph, int region_in, int region_out, double dampi
         const char *e = getenv("PROACT_PR_KERNEL");
         return e && !strcmp(e, "plain") ? 1 : 0;
     }();
+    if (l2_window_on()) {
+        proact_region_info ri;
+        if (proact_region_info_get(region_in, &ri) == PROACT_OK)
+            proact_internal_l2_window(ri.replica_base, ri.total_bytes);
+    }
     if (!plain)
         return proact_launch(regs, 1, (const void *)pagerank_hot_kernel, 0, GB * PG, args,
                              4 * ((size_t)PG * CPS + p.g.nhot), stream);
@@ -1400,6 +1419,11 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
+    if (l2_window_on()) {
+        proact_region_info ri;
+        if (proact_region_info_get(region_in, &ri) == PROACT_OK)
+            proact_internal_l2_window(ri.replica_base, ri.total_bytes);
+    }
     if (p.g.nhot && p.g.nhot <= HOT_MAX - CHG_WORDS)   // hot table (room for the changed bitmap)
         return proact_launch(regs, 1, (const void *)sssp_hot_kernel, 0, GB * PG, args,
                              4 * ((size_t)PG * CPS + p.g.nhot), stream);

@@ -851,9 +851,59 @@ int proact_launch_tallies(void)
     return (m == PROACT_MECH_FUSED || m == PROACT_MECH_DMA) && c->world > 1;
 }
 
+// Optional L2 access-policy window for the NEXT producer launch of this thread (set by a
+// workload entry point right before proact_launch, consumed by it): the gathered replica of the
+// graph kernels is marked persisting so the streamed CSC arrays cannot evict it.
+namespace {
+thread_local const void *g_l2_base = nullptr;
+thread_local size_t g_l2_bytes = 0;
+
+cudaError_t launch_producer(const void *kernel, unsigned total, unsigned block, void **args, size_t smem,
+                            cudaStream_t s, int device, const void *l2_base, size_t l2_bytes)
+{
+    if (!l2_base || !l2_bytes) return cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s);
+    static thread_local int limit_dev = -1;
+    static thread_local size_t limit = 0;
+    if (limit_dev != device) {   // reserve the persisting L2 set-aside once per device
+        cudaDeviceProp prop;
+        if (cudaGetDeviceProperties(&prop, device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
+            limit = (size_t)prop.persistingL2CacheMaxSize;
+            if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, limit) != cudaSuccess) limit = 0;
+        }
+        limit_dev = device;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(total);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    at[0].val.accessPolicyWindow.base_ptr = const_cast<void *>(l2_base);
+    at[0].val.accessPolicyWindow.num_bytes = l2_bytes;
+    at[0].val.accessPolicyWindow.hitRatio =
+        limit ? (float)std::min(1.0, (double)limit / (double)l2_bytes) : 0.f;
+    at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    cfg.attrs = at;
+    cfg.numAttrs = limit ? 1 : 0;
+    return cudaLaunchKernelExC(&cfg, kernel, args);
+}
+}  // namespace
+
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_l2_window(const void *base, size_t bytes)
+{
+    g_l2_base = base;
+    g_l2_bytes = bytes;
+}
+
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
                   void **args, size_t smem, void *stream)
 {
+    const void *l2b = g_l2_base;   // this launch's L2 window hint (proact_internal_l2_window)
+    const size_t l2n = g_l2_bytes;
+    g_l2_base = nullptr;
+    g_l2_bytes = 0;
     RankCtx *c = need_ctx();
     if (!c) return PROACT_ERR_STATE;
     if (!kernel || !args || !args[0] || nregions < 0 || (nregions && !regions)) return PROACT_ERR_INVALID;
@@ -963,7 +1013,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         const unsigned reserve = std::min(cap - 1, agent_ctas * lost);
         if (total + reserve > cap) total = cap - reserve;
         *(launch_ctx *)args[0] = lc;
-        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
         CK(cudaStreamWaitEvent(s, c->ev_done, 0));
     } else if (lc.mech == PROACT_MECH_DMA && armed) {
         // NEXT-3 "hardware PROACT": the copy engines are the transfer agent.  Per owned chunk,
@@ -980,7 +1030,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         // can buffer, and enqueueing them must never block the launch that satisfies them
         unsigned total = grid ? grid : cap;
         if (total > cap) total = cap;
-        CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
 
         uint32_t peers = 0;
         for (int r = 0; r < c->nregions; ++r)
@@ -1048,7 +1098,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         if (c->coop && agent)
             CK(cudaLaunchCooperativeKernel(kernel, dim3(total), dim3(block), args, smem, s));
         else
-            CK(cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s));
+            CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
     }
     for (int r = 0; r < c->nregions; ++r) {
         if (!(armed >> r & 1)) continue;

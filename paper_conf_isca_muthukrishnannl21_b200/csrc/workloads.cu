@@ -11,6 +11,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "proact.h"
 #include "proact_device.cuh"
 #include "proact_workloads.h"
@@ -525,21 +527,172 @@ int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int sca
     return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
 }
 
-// Force-load this translation unit's kernels (called by proact_init).  Under CUDA's lazy module
-// loading the first launch of a kernel loads it, and a load waits for the device's running
-// kernels -- with loopback ranks one of those can be a spin waiting for this very thread's next
-// launch (observed: smoke deadlocks until the watchdog).  Loading up front removes the hazard.
-__attribute__((visibility("hidden"))) int proact_internal_preload_workloads(void)
-{
-    cudaFuncAttributes a;
-    const void *k[] = {(const void *)jacobi_kernel<true>, (const void *)jacobi_kernel<false>,
-                       (const void *)micro_kernel, (const void *)banded_kernel};
-    for (const void *f : k)
-        if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
-    return PROACT_OK;
-}
-
 }  // extern "C"
+
+// ---- banded Jacobi, TMA-fed (default when N % 4 == 0 and w <= BW_MAX): the first kernel was
+// latency bound (one CTA iteration = 7 serialised global round trips; 2.0 TB/s).  Here one
+// producer warp streams, per BT2-row tile, the x window + b + diagonal slices (tile slots, double
+// buffered) and then the tile's off-diagonals in groups of BDG through a BNS-deep shared-memory
+// ring (cp.async.bulk, 8 KiB per diagonal slice, contiguous in the DIA layout); eight compute
+// warps sum each row over o = -w..w (o != 0) in order from shared memory (reading R19).
+namespace {
+// measured at N = 2^24, w = 16 (tools/bench_workloads.py --workload banded, one variant per
+// build): 2048 rows x 2 diagonals x 4 stages, 2 CTAs/SM: 0.414 ms (0.89 of HBM); 512 x 8 x 6:
+// 0.634 ms; 1024 x 4 x 5: 0.482 ms; 4096 x 1 x 3 (1 CTA/SM): 0.617 ms -- 8 KiB bulk copies beat
+// 2 KiB ones (TMA issue cost), two CTAs per SM beat one (latency hiding)
+#ifndef PROACT_BANDED_BT
+#define PROACT_BANDED_BT 2048
+#endif
+#ifndef PROACT_BANDED_DG
+#define PROACT_BANDED_DG 2
+#endif
+#ifndef PROACT_BANDED_RING
+#define PROACT_BANDED_RING 4
+#endif
+#ifndef PROACT_BANDED_MINB
+#define PROACT_BANDED_MINB 2
+#endif
+constexpr int BT2 = PROACT_BANDED_BT;    // rows per tile
+constexpr int BCW = 8;                   // compute warps
+constexpr int BRT = BT2 / (BCW * 32);    // rows per compute thread
+constexpr int BDG = PROACT_BANDED_DG;    // diagonals per ring stage
+constexpr int BNS = PROACT_BANDED_RING;  // ring stages
+constexpr int BW_MAX = 4096;             // larger bands use banded_kernel
+
+__host__ __device__ __forceinline__ int banded_xw(long long w) { return (int)((BT2 + 2 * w + 8 + 3) & ~3LL); }
+__host__ __device__ __forceinline__ size_t banded_smem(long long w)
+{
+    return (size_t)BNS * BDG * BT2 * 4 + 2 * ((size_t)banded_xw(w) + 2 * BT2) * 4 + (2 * BNS + 4) * 8 + 16;
+}
+// i-th off-diagonal of the band in the summation order o = -w..-1, 1..w
+__device__ __forceinline__ int64_t band_o(int64_t idx, int64_t w) { return idx < w ? idx - w : idx - w + 1; }
+
+__device__ __noinline__ void banded_stream(const launch_ctx &lc, const proact_banded_params &p, float *ring,
+                                           float *slots, int xw, uint64_t *full, uint64_t *empty, uint64_t *tfull,
+                                           uint64_t *tempty, int *tids, int64_t ntiles)
+{
+    const int64_t N = p.N, w = p.w, rend = p.row0 + p.nrows, ngroups = (2 * w + BDG - 1) / BDG;
+    const float *x = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
+    uint32_t q = 0;
+    for (uint32_t kt = 0;; ++kt) {
+        const uint32_t t = proact::claim_tile(lc, (uint32_t)ntiles);
+        const uint32_t slot = kt & 1u;
+        if (kt >= 2) mbar_wait(&tempty[slot], ((kt >> 1) - 1) & 1u);
+        if (t >= (uint32_t)ntiles) {
+            tids[slot] = -1;
+            mbar_arrive(&tfull[slot]);
+            return;
+        }
+        tids[slot] = (int)t;
+        const int64_t i0 = p.row0 + (int64_t)t * BT2, i1 = min(i0 + (int64_t)BT2, rend), nr = i1 - i0;
+        const int64_t lo = i0 - w > 0 ? i0 - w : 0, hi = i1 + w < N ? i1 + w : N;
+        const int64_t lo4 = lo & ~(int64_t)3, hi4 = min(N, (int64_t)((hi + 3) & ~(int64_t)3));
+        // (a7) peers' rows of the previous generation within the band, then generic -> async proxy
+        proact::wait_range(lc, p.region_in, (uint64_t)lo * 4, (uint64_t)(hi - lo) * 4);
+        asm volatile("fence.proxy.async;" ::: "memory");
+        float *xs = slots + slot * (xw + 2 * BT2);
+        mbar_expect_tx(&tfull[slot], (uint32_t)((hi4 - lo4) + 2 * nr) * 4);
+        bulk_g2s(xs, x + lo4, (uint32_t)(hi4 - lo4) * 4, &tfull[slot]);
+        bulk_g2s(xs + xw, p.b + i0, (uint32_t)nr * 4, &tfull[slot]);
+        bulk_g2s(xs + xw + BT2, p.a + w * N + i0, (uint32_t)nr * 4, &tfull[slot]);
+        for (int64_t g = 0; g < ngroups; ++g, ++q) {
+            const uint32_t st = q % BNS;
+            if (q >= BNS) mbar_wait(&empty[st], ((q / BNS) - 1) & 1u);
+            const int64_t nd = min((int64_t)BDG, 2 * w - g * BDG);
+            mbar_expect_tx(&full[st], (uint32_t)(nd * nr) * 4);
+            for (int64_t k = 0; k < nd; ++k) {
+                const int64_t o = band_o(g * BDG + k, w);
+                bulk_g2s(ring + ((size_t)st * BDG + k) * BT2, p.a + (o + w) * N + i0, (uint32_t)nr * 4, &full[st]);
+            }
+        }
+    }
+}
+}  // namespace
+
+__global__ void __launch_bounds__((BCW + 1) * 32, PROACT_BANDED_MINB) banded_tma_kernel(launch_ctx lc, proact_banded_params p)
+{
+    if (proact::agent_dispatch(lc)) return;
+    extern __shared__ __align__(128) unsigned char bsm[];
+    const int64_t N = p.N, w = p.w, rend = p.row0 + p.nrows, ngroups = (2 * w + BDG - 1) / BDG;
+    const int xw = banded_xw(w);
+    float *ring = reinterpret_cast<float *>(bsm);
+    float *slots = ring + (size_t)BNS * BDG * BT2;
+    uint64_t *full = reinterpret_cast<uint64_t *>(slots + 2 * (xw + 2 * BT2));
+    uint64_t *empty = full + BNS, *tfull = empty + BNS, *tempty = tfull + 2;
+    int *tids = reinterpret_cast<int *>(tempty + 2);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t ntiles = (p.nrows + BT2 - 1) / BT2;
+    if (tid == 0) {
+        for (int s = 0; s < BNS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], BCW);
+        }
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(&tfull[s], 1);
+            mbar_init(&tempty[s], BCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (warp == BCW) {
+        if (lane == 0) banded_stream(lc, p, ring, slots, xw, full, empty, tfull, tempty, tids, ntiles);
+        return;
+    }
+    uint32_t q = 0;
+    for (uint32_t kt = 0;; ++kt) {
+        const uint32_t slot = kt & 1u;
+        mbar_wait(&tfull[slot], (kt >> 1) & 1u);
+        const int t = tids[slot];
+        if (t < 0) break;
+        const int64_t i0 = p.row0 + (int64_t)t * BT2, i1 = min(i0 + (int64_t)BT2, rend), nr = i1 - i0;
+        const int64_t lo = i0 - w > 0 ? i0 - w : 0, lo4 = lo & ~(int64_t)3;
+        const float *xs = slots + slot * (xw + 2 * BT2);
+        const bool clean = nr == BT2 && i0 - w >= 0 && i1 + w <= N;
+        float sum[BRT];
+#pragma unroll
+        for (int r = 0; r < BRT; ++r) sum[r] = 0.0f;
+        for (int64_t g = 0; g < ngroups; ++g, ++q) {
+            const uint32_t st = q % BNS;
+            mbar_wait(&full[st], (q / BNS) & 1u);
+            const float *sa = ring + (size_t)st * BDG * BT2;
+            const int64_t nd = min((int64_t)BDG, 2 * w - g * BDG);
+            if (clean) {   // full tile, band inside [0, N): no per-element bounds tests
+                for (int k = 0; k < (int)nd; ++k) {
+                    const int o = (int)band_o(g * BDG + k, w);
+                    const float *ao = sa + k * BT2 + tid;
+                    const float *xo = xs + (int)(i0 - lo4) + o + tid;
+#pragma unroll
+                    for (int r = 0; r < BRT; ++r)
+                        sum[r] = __fadd_rn(sum[r], __fmul_rn(ao[r * (BCW * 32)], xo[r * (BCW * 32)]));
+                }
+            } else {
+                for (int64_t k = 0; k < nd; ++k) {
+                    const int64_t o = band_o(g * BDG + k, w);
+#pragma unroll
+                    for (int r = 0; r < BRT; ++r) {
+                        const int64_t ii = tid + r * (BCW * 32), i = i0 + ii, j = i + o;
+                        if (ii < nr && j >= 0 && j < N)
+                            sum[r] = __fadd_rn(sum[r], __fmul_rn(sa[k * BT2 + ii], xs[j - lo4]));
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[st]);
+        }
+#pragma unroll
+        for (int r = 0; r < BRT; ++r) {
+            const int64_t ii = tid + r * (BCW * 32);
+            if (ii < nr) {
+                const float v = __fdiv_rn(__fsub_rn(xs[xw + ii], sum[r]), xs[xw + BT2 + ii]);
+                proact::put(lc, p.region_out, (uint64_t)(i0 + ii) * 4, v);
+            }
+        }
+        asm volatile("bar.sync 1, %0;" ::"r"(BCW * 32) : "memory");   // the compute warps' stores
+        if (tid == 0) proact::commit_span(lc, p.region_out, (uint64_t)i0 * 4, (uint64_t)nr * 4);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[slot]);
+    }
+}
 
 extern "C" int proact_banded_phase(int region_in, int region_out, const float *a, const float *b, long long N,
                                    long long w, void *stream)
@@ -562,6 +715,24 @@ extern "C" int proact_banded_phase(int region_in, int region_out, const float *a
     p.nrows = (long long)(ro.own_bytes / 4);
     p.a = a;
     p.b = b;
+    launch_ctx lc;
+    void *args[2] = {&lc, &p};
+    int regs[1] = {region_out};
+    static const int tma_off = [] {
+        const char *e = getenv("PROACT_BANDED_PLAIN");
+        return e && atoi(e) ? 1 : 0;
+    }();
+    if (!tma_off && N % 4 == 0 && w <= BW_MAX && (uintptr_t)a % 16 == 0 && (uintptr_t)b % 16 == 0) {
+        const size_t tsmem = banded_smem(w);
+        static size_t tattr = 48 * 1024;
+        if (tsmem > tattr) {
+            if (cudaFuncSetAttribute(banded_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tsmem) !=
+                cudaSuccess)
+                return PROACT_ERR_CUDA;
+            tattr = tsmem;
+        }
+        return proact_launch(regs, 1, (const void *)banded_tma_kernel, 0, (BCW + 1) * 32, args, tsmem, stream);
+    }
     const size_t smem = (size_t)(BT + 2 * w) * 4;
     static size_t attr = 48 * 1024;
     if (smem > attr) {
@@ -569,9 +740,6 @@ extern "C" int proact_banded_phase(int region_in, int region_out, const float *a
             return PROACT_ERR_CUDA;
         attr = smem;
     }
-    launch_ctx lc;
-    void *args[2] = {&lc, &p};
-    int regs[1] = {region_out};
     return proact_launch(regs, 1, (const void *)banded_kernel, 0, BB, args, smem, stream);
 }
 
@@ -629,3 +797,21 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
     if (bytes_d2h) *bytes_d2h = (unsigned long long)((r1 - r0) * rowb);
     return PROACT_OK;
 }
+
+extern "C" {
+// Force-load this translation unit's kernels (called by proact_init).  Under CUDA's lazy module
+// loading the first launch of a kernel loads it, and a load waits for the device's running
+// kernels -- with loopback ranks one of those can be a spin waiting for this very thread's next
+// launch (observed: smoke deadlocks until the watchdog).  Loading up front removes the hazard.
+__attribute__((visibility("hidden"))) int proact_internal_preload_workloads(void)
+{
+    cudaFuncAttributes a;
+    const void *k[] = {(const void *)jacobi_kernel<true>, (const void *)jacobi_kernel<false>,
+                       (const void *)micro_kernel, (const void *)banded_kernel,
+                       (const void *)banded_tma_kernel};
+    for (const void *f : k)
+        if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
+    return PROACT_OK;
+}
+
+}  // extern "C"
