@@ -129,6 +129,9 @@ constexpr uint32_t HOT_DEFAULT = 8192;
 #ifndef PROACT_SSH_MINB      // sssp_hot_kernel CTAs per SM
 #define PROACT_SSH_MINB 2
 #endif
+#ifndef PROACT_PRH_VEC       // pagerank_hot_kernel: 16-byte index loads from a 4-edge-aligned base
+#define PROACT_PRH_VEC 1
+#endif
 #ifndef PROACT_PRH_PIPE
 #define PROACT_PRH_PIPE 1
 #endif
@@ -386,10 +389,12 @@ __global__ void runv_kernel(const Item *items, const uint32_t *colptr, uint32_t 
 {
     const Item it = items[blockIdx.x];
     const uint32_t lo = it.tile * GT, nvt = min(lo + GT, nv) - lo;
-    const uint32_t nrun = (it.e1 - it.e0 + RUN - 1) / RUN;
+    // hot-kernel runs (which == 2, PRH_VEC) start at the 4-edge-aligned base below e0
+    const uint32_t b0 = which == 2 && PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0;
+    const uint32_t nrun = (it.e1 - b0 + RUN - 1) / RUN;
     const uint32_t off = which == 2 ? it.run_ph : which ? it.run_ss : it.run_pr;
     for (uint32_t j = threadIdx.x; j < nrun; j += blockDim.x)
-        runv[off + j] = (uint16_t)vertex_of(colptr + lo, nvt, it.e0 + j * RUN);
+        runv[off + j] = (uint16_t)vertex_of(colptr + lo, nvt, max(it.e0, b0 + j * RUN));
 }
 
 // Tile prologue: colptr of the tile into shared memory (+ the accumulator init by the caller).
@@ -601,14 +606,40 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         // run entries are in flight while this round's gathers are, so a round costs one L2 round
         // trip instead of two
         uint32_t xn[RUN], in_ = 0;
+#if PROACT_PRH_VEC
+        static_assert(PROACT_PRH_RUN == 4, "PRH_VEC loads one run of 4 edges as 16 bytes");
+        const uint32_t abase = it.e0 & ~3u;   // runs start 16-byte aligned; edges < e0 are masked
+        auto load_idx = [&](uint32_t base) {
+            const uint32_t r0 = base + lrun * RUN;
+            if (r0 < it.e1) {
+                uint32_t v0, v1, v2, v3;
+                asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                             : "=r"(v0), "=r"(v1), "=r"(v2), "=r"(v3) : "l"(p.g.rowidx_h + r0), "l"(pf));
+                xn[0] = v0;
+                xn[1] = v1;
+                xn[2] = v2;
+                xn[3] = v3;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q)
+                    if (r0 + q >= it.e1 || r0 + q < it.e0) xn[q] = HOT_BIT;   // not this item's edge
+                in_ = ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - abase) / RUN, pf);
+            } else {
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) xn[q] = HOT_BIT;
+                in_ = 0u;
+            }
+        };
+#else
+        const uint32_t abase = it.e0;
         auto load_idx = [&](uint32_t base) {
             const uint32_t r0 = base + lrun * RUN;
 #pragma unroll
             for (int q = 0; q < RUN; ++q) xn[q] = r0 + q < it.e1 ? ld_stream_u(p.g.rowidx_h + r0 + q, pf) : HOT_BIT;
             in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - it.e0) / RUN, pf) : 0u;
         };
-        if (PROACT_PRH_PIPE) load_idx(it.e0);
-        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+#endif
+        if (PROACT_PRH_PIPE) load_idx(abase);
+        for (uint32_t base = abase; base < it.e1; base += GB * RUN) {
             const uint32_t r0 = base + lrun * RUN;
             const bool act = r0 < it.e1;
             if (!PROACT_PRH_PIPE) load_idx(base);
@@ -639,6 +670,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     if (r0 + q >= r1) break;
+                    if (r0 + q < it.e0) continue;   // PRH_VEC: the aligned run starts before the item
                     while (r0 + q >= nxt) {   // vertex i closes before edge r0 + q
                         if (!multi) {
                             kin = i;
@@ -700,6 +732,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     if (r0 + q >= r1) break;
+                    if (r0 + q < it.e0) continue;   // PRH_VEC: the aligned run starts before the item
                     while (r0 + q >= nxt) {
                         if (sum) acc_add(i, sum);
                         sum = 0ull;
@@ -1196,7 +1229,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
     GCK(cudaMemcpyAsync(&e_own, G.colptr + G.nv, 4, cudaMemcpyDeviceToHost, s));
     GCK(cudaStreamSynchronize(s));
     G.E_own = e_own;
-    GCK(cudaMalloc((void **)&G.rowidx, 4 * ((size_t)e_own + 1)));
+    GCK(cudaMalloc((void **)&G.rowidx, 4 * ((size_t)e_own + 4)));   // +4: 16-byte index loads
     if (d_w) GCK(cudaMalloc((void **)&G.w, 4 * ((size_t)e_own + 1)));
     GCK(cudaMemcpyAsync(indeg, G.colptr, 4 * ((size_t)G.nv + 1), cudaMemcpyDeviceToDevice, s));   // cursors
     if (E) scatter_kernel<<<1184, 256, 0, s>>>(d_src, d_dst, d_w, E, v0, v1, indeg, G.rowidx, G.w);
@@ -1232,7 +1265,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
             it.run_ph = (uint32_t)nph;
             npr += (it.e1 - it.e0 + PROACT_PR_RUN - 1) / PROACT_PR_RUN;
             nss += (it.e1 - it.e0 + PROACT_SSSP_RUN - 1) / PROACT_SSSP_RUN;
-            nph += (it.e1 - it.e0 + PROACT_PRH_RUN - 1) / PROACT_PRH_RUN;
+            nph += (it.e1 - (PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0) + PROACT_PRH_RUN - 1) / PROACT_PRH_RUN;
         }
         if (npr >= (1ull << 32) || nss >= (1ull << 32) || nph >= (1ull << 32)) return PROACT_ERR_NOMEM;
         GCK(cudaMalloc((void **)&G.items, sizeof(Item) * std::max<size_t>(1, split.size())));
@@ -1280,7 +1313,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
             GCK(cudaMalloc((void **)&slot, 4 * (size_t)V));
             GCK(cudaMemsetAsync(slot, 0xFF, 4 * (size_t)V, s));
             hot_slot_kernel<<<(unsigned)((H + 255) / 256), 256, 0, s>>>(G.hot_ids, (uint32_t)H, slot);
-            GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 1)));
+            GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 4)));
             unsigned long long *neh = nullptr;
             GCK(cudaMalloc((void **)&neh, 8));
             GCK(cudaMemsetAsync(neh, 0, 8, s));

@@ -490,9 +490,12 @@ __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t ma
 }
 
 // PROACT_AGENT_SEPARATE: the transfer agent as its own kernel (own registers, TMA staging ring)
-// staging ring: 8 x 16 KiB (+ metadata) for up to 32 agent CTAs, 8 x 8 KiB beyond (2 per SM)
-constexpr size_t AGENT_SMEM = 128 * 1024 + 1024;
+// staging ring of a BULK agent CTA: 8 x 24 KiB for up to 32 agent CTAs (one per SM; loopback G = 2
+// microbenchmark, 16 agent CTAs: 1.02 ms per phase vs 1.23 ms with 8 x 16 KiB; Jacobi 32 CTAs:
+// 0.767 vs 0.845 ms), 8 x 8 KiB beyond
+constexpr size_t AGENT_SMEM = 200 * 1024 + 1024;
 constexpr size_t AGENT_SMEM_SMALL = 64 * 1024 + 1024;
+constexpr size_t AGENT_SMEM_MAX = 224 * 1024 + 1024;   // PROACT_AGENT_SMEM_KB upper bound
 __global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc)
 {
     // residency gate: the producer's stream waits until every agent CTA is resident, so the
@@ -614,7 +617,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
             if (cudaStreamCreateWithPriority(&c->dma[k], cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
             if (cudaEventCreateWithFlags(&c->ev_dma[k], cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         }
-        if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM) !=
+        if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM_MAX) !=
             cudaSuccess)
             return fail(PROACT_ERR_CUDA);
         // no lazy kernel loading once ranks may spin on each other (see workloads.cu)
@@ -972,7 +975,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         la.agent_ctas = (uint16_t)agent_ctas;
         size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
-            asmem = std::min(AGENT_SMEM, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
+            asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
         CK(cudaEventRecord(c->ev_start, s));
         CK(cudaStreamWaitEvent(c->side, c->ev_start, 0));
         agent_kernel<<<agent_ctas, agent_block, asmem, c->side>>>(la);
