@@ -132,6 +132,9 @@ constexpr uint32_t HOT_DEFAULT = 8192;
 #ifndef PROACT_PRH_VEC       // pagerank_hot_kernel: 16-byte index loads from a 4-edge-aligned base
 #define PROACT_PRH_VEC 1
 #endif
+#ifndef PROACT_SSH_VEC       // sssp_hot_kernel: runs of 4 edges, 16-byte index / weight loads (runv_ph)
+#define PROACT_SSH_VEC 1
+#endif
 #ifndef PROACT_PRH_PIPE
 #define PROACT_PRH_PIPE 1
 #endif
@@ -933,7 +936,12 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
 // else INT32_MAX, so a hot in-edge needs neither the bitmap test nor the global gather.
 __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(launch_ctx lc, SsspParams p)
 {
+#if PROACT_SSH_VEC
+    static_assert(PROACT_PRH_VEC && PROACT_PRH_RUN == 4, "SSH_VEC shares the aligned 4-edge runs of runv_ph");
+    constexpr int RUN = 4;
+#else
     constexpr int RUN = PROACT_SSSP_RUN;   // shares runv_ss with sssp_kernel
+#endif
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
     __shared__ int32_t acc_a[PG][GT];
@@ -994,14 +1002,34 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         for (uint32_t i = t; i < nvt; i += GB) acc[i] = INT32_MAX;
         grp_bar(grp);
         uint32_t xn[RUN], in_ = 0;
+#if PROACT_SSH_VEC
+        const uint32_t abase = it.e0 & ~3u;   // as in pagerank_hot_kernel (PRH_VEC)
+        auto load_idx = [&](uint32_t base) {
+            const uint32_t r0 = base + lrun * RUN;
+            if (r0 < it.e1) {
+                uint32_t v0, v1, v2, v3;
+                asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                             : "=r"(v0), "=r"(v1), "=r"(v2), "=r"(v3) : "l"(p.g.rowidx_h + r0), "l"(pf));
+                xn[0] = v0;
+                xn[1] = v1;
+                xn[2] = v2;
+                xn[3] = v3;
+                in_ = ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - abase) / RUN, pf);
+            } else {
+                in_ = 0u;
+            }
+        };
+#else
+        const uint32_t abase = it.e0;
         auto load_idx = [&](uint32_t base) {
             const uint32_t r0 = base + lrun * RUN;
 #pragma unroll
             for (int q = 0; q < RUN; ++q) xn[q] = r0 + q < it.e1 ? ld_stream_u(p.g.rowidx_h + r0 + q, pf) : HOT_BIT;
             in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_ss + it.run_ss + (r0 - it.e0) / RUN, pf) : 0u;
         };
-        load_idx(it.e0);
-        for (uint32_t base = it.e0; base < it.e1; base += GB * RUN) {
+#endif
+        load_idx(abase);
+        for (uint32_t base = abase; base < it.e1; base += GB * RUN) {
             const uint32_t r0 = base + lrun * RUN;
             const bool act = r0 < it.e1;
             uint32_t x[RUN];
@@ -1017,23 +1045,41 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     int32_t du = INT32_MAX;
-                    if (r0 + q < r1) {
+                    if (r0 + q < r1 && r0 + q >= it.e0) {
                         if (x[q] & HOT_BIT) du = hot[x[q] & ~HOT_BIT & 0xFFFFu];
                         else if (changed_src(x[q])) du = ld_gather_i(din + x[q], pl);
                     }
                     c[q] = du;
                 }
+#if PROACT_SSH_VEC
+                bool anyc = false;
+#pragma unroll
+                for (int q = 0; q < RUN; ++q) anyc |= c[q] != INT32_MAX;
+                if (anyc) {   // one 16-byte weight load for the run
+                    int32_t wv[4];
+                    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+                                 : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3]) : "l"(p.g.w + r0), "l"(pf));
+#pragma unroll
+                    for (int q = 0; q < RUN; ++q)
+                        if (c[q] != INT32_MAX) {
+                            const int64_t cand = (int64_t)c[q] + (int64_t)wv[q];
+                            c[q] = cand < (int64_t)INT32_MAX ? (int32_t)cand : INT32_MAX;
+                        }
+                }
+#else
 #pragma unroll
                 for (int q = 0; q < RUN; ++q)
                     if (c[q] != INT32_MAX) {
                         const int64_t cand = (int64_t)c[q] + (int64_t)ld_stream_i(p.g.w + r0 + q, pf);
                         c[q] = cand < (int64_t)INT32_MAX ? (int32_t)cand : INT32_MAX;
                     }
+#endif
                 uint32_t nxt = cp[i + 1];
                 single = r1 <= nxt;
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     if (r0 + q >= r1) break;
+                    if (r0 + q < it.e0) continue;   // SSH_VEC: the aligned run starts before the item
                     while (r0 + q >= nxt) {
                         if (best != INT32_MAX) atomicMin(&acc[i], best);
                         best = INT32_MAX;
@@ -1230,7 +1276,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
     GCK(cudaStreamSynchronize(s));
     G.E_own = e_own;
     GCK(cudaMalloc((void **)&G.rowidx, 4 * ((size_t)e_own + 4)));   // +4: 16-byte index loads
-    if (d_w) GCK(cudaMalloc((void **)&G.w, 4 * ((size_t)e_own + 1)));
+    if (d_w) GCK(cudaMalloc((void **)&G.w, 4 * ((size_t)e_own + 4)));   // +4: 16-byte loads
     GCK(cudaMemcpyAsync(indeg, G.colptr, 4 * ((size_t)G.nv + 1), cudaMemcpyDeviceToDevice, s));   // cursors
     if (E) scatter_kernel<<<1184, 256, 0, s>>>(d_src, d_dst, d_w, E, v0, v1, indeg, G.rowidx, G.w);
     GCK(cudaGetLastError());
