@@ -80,6 +80,20 @@ def pagerank(args, src, dst, V):
         kms = statistics.median(a.elapsed_time(b) for a, b in ks)
         out = {"ms": ms, "kms": kms, "e_own": P.e_own, "nv": P.v1 - P.v0, "iters": args.steps * I,
                "nhot": P.nhot, "e_hot": P.e_hot}
+        if G == 1:   # tracking overhead (Fig. 8 methodology): tallies + agent, pushes elided, vs LOCAL
+            def phase_ms(mech, n=10):
+                rt.set_config(mech=mech)
+                torch.cuda.synchronize()
+                a, b = ev(), ev()
+                a.record(s)
+                for _ in range(n):
+                    P.step(s)
+                b.record(s)
+                torch.cuda.synchronize()
+                return a.elapsed_time(b) / n
+            phase_ms(_lib.MECH_ELIDE, 2)
+            out["overhead"] = {"local_ms": phase_ms(_lib.MECH_LOCAL), "elide_ms": phase_ms(_lib.MECH_ELIDE)}
+            rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
         P.free()
         return out
     res = run_ranks(args.ranks, body)
@@ -104,6 +118,11 @@ def pagerank(args, src, dst, V):
     line["roofline_l1_gather"] = {"bound": "l1tex_wavefronts", "gathers_per_launch": e_max,
                                   "peak_gathers_per_s": rate, "t_min_ms": t_l1, "frac": t_l1 / kms,
                                   "note": "global gathers (in-edges of non-hot sources); 1 wavefront/clk/SM x SMs x 1965 MHz"}
+    if "overhead" in res[0]:
+        o = res[0]["overhead"]
+        line["overhead"] = {"local_ms_per_phase": o["local_ms"], "elide_ms_per_phase": o["elide_ms"],
+                            "tracking_overhead_frac": o["elide_ms"] / o["local_ms"] - 1.0,
+                            "note": "G=1: ELIDE keeps tallies + agent with remote stores skipped (Fig. 8 methodology)"}
     if not args.no_cpu:
         import oracle
         t0 = time.perf_counter()
@@ -166,6 +185,16 @@ def sssp(args, src, dst, V):
                 break
         out = {"rounds": rounds, "t": sum(times[args.warmup:]), "kern_ms": kern, "alg": algs,
                "nhot": S.nhot, "e_own": S.e_own}
+        if G == 1:   # tracking overhead: a whole run under ELIDE vs LOCAL
+            oh = {}
+            for name, mech in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE), ("local", _lib.MECH_LOCAL)):
+                rt.set_config(mech=mech)
+                S.reset()
+                t0 = time.perf_counter()
+                S.run(stream=st)
+                oh[name] = time.perf_counter() - t0
+            out["overhead"] = oh
+            rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
         S.free()
         return out
     epc = np.bincount(src // (args.chunk // 4), minlength=(V + args.chunk // 4 - 1) // (args.chunk // 4))
@@ -176,6 +205,11 @@ def sssp(args, src, dst, V):
             "value": args.steps * rounds / t, "unit": "rounds/s", "rounds": rounds, "ranks": args.ranks,
             "mech": args.mech, "chunk_bytes": args.chunk, "edges": int(src.size),
             "timing": "host wall clock per run (a BARRIER + host vote read every round)"}
+    if "overhead" in res[0]:
+        o = res[0]["overhead"]
+        line["overhead"] = {"local_s_per_run": o["local"], "elide_s_per_run": o["elide"],
+                            "tracking_overhead_frac": o["elide"] / o["local"] - 1.0,
+                            "note": "G=1: ELIDE keeps tallies + agent with remote stores skipped (Fig. 8 methodology)"}
     if args.ranks == 1:
         r0 = res[0]
         kms, alg = sum(r0["kern_ms"]), sum(r0["alg"])
