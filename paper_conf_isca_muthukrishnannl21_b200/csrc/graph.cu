@@ -1157,6 +1157,7 @@ __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t 
 
 }  // namespace
 extern "C" __attribute__((visibility("hidden"))) void proact_internal_l2_window(const void *base, size_t bytes);
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_keep_l1(const void *kernel);
 namespace {
 
 // PROACT_L2_WINDOW=1: mark the gathered replica persisting in L2 for the phase launch
@@ -1376,6 +1377,9 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
     GCK(cudaStreamSynchronize(s));
     GCK(cudaFuncSetAttribute((const void *)pagerank_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)(4 * (PG * CPS + HOT_MAX))));
+    for (const void *k : {(const void *)pagerank_hot_kernel, (const void *)pagerank_kernel,
+                          (const void *)sssp_hot_kernel, (const void *)sssp_kernel})
+        proact_internal_keep_l1(k);
     GCK(cudaFuncSetAttribute((const void *)sssp_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)(4 * (PG * CPS + HOT_MAX)) - (int)(4 * CHG_WORDS)));
     G.used = true;

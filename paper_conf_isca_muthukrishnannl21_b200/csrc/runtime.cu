@@ -854,6 +854,26 @@ int proact_launch_tallies(void)
     return (m == PROACT_MECH_FUSED || m == PROACT_MECH_DMA) && c->world > 1;
 }
 
+// Producer kernels that must keep the driver's default shared-memory carve-out even next to a
+// separate agent (registered by their entry points): the graph kernels' random gathers need the
+// L1 left over as landing space -- at the maximal carve-out PageRank / SSSP phases ran 2.2x slower
+// (a carve-out attribute persists for every later launch of the kernel, in every mechanism).
+namespace {
+std::mutex g_l1_mu;
+std::vector<const void *> g_l1_kernels;
+bool keeps_l1(const void *k)
+{
+    std::lock_guard<std::mutex> g(g_l1_mu);
+    return std::find(g_l1_kernels.begin(), g_l1_kernels.end(), k) != g_l1_kernels.end();
+}
+}  // namespace
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_keep_l1(const void *kernel)
+{
+    std::lock_guard<std::mutex> g(g_l1_mu);
+    if (std::find(g_l1_kernels.begin(), g_l1_kernels.end(), kernel) == g_l1_kernels.end())
+        g_l1_kernels.push_back(kernel);
+}
+
 // Optional L2 access-policy window for the NEXT producer launch of this thread (set by a
 // workload entry point right before proact_launch, consumed by it): the gathered replica of the
 // graph kernels is marked persisting so the streamed CSC arrays cannot evict it.
@@ -963,7 +983,8 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     cudaStream_t s = (cudaStream_t)stream;
     if (separate) {
         // producer kernels share SMs with the agent: same (maximal) shared-memory carveout
-        if (std::find(c->carveout_set.begin(), c->carveout_set.end(), kernel) == c->carveout_set.end()) {
+        if (std::find(c->carveout_set.begin(), c->carveout_set.end(), kernel) == c->carveout_set.end() &&
+            !keeps_l1(kernel)) {
             CK(cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
                                     cudaSharedmemCarveoutMaxShared));
             c->carveout_set.push_back(kernel);

@@ -247,9 +247,14 @@ class PageRank(_Graph):
         self.k += 1
 
     def ranks(self, stream=None) -> torch.Tensor:
+        """My r' (nv floats), copied on `stream` after its phases; the current torch stream is made
+        to wait for that copy, so the tensor can be used (e.g. .cpu()) on it directly."""
         out = torch.empty(self.v1 - self.v0, dtype=torch.float32, device="cuda")
         check(rt.lib().proact_pagerank_ranks(self.gid, ctypes.c_void_p(out.data_ptr()), _s(stream)),
               "pagerank_ranks")
+        if stream is not None and stream != torch.cuda.current_stream():
+            out.record_stream(stream)
+            torch.cuda.current_stream().wait_stream(stream)
         return out
 
 

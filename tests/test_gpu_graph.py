@@ -217,3 +217,26 @@ def test_votes_are_epoch_tagged():
 
     (votes,) = run_ranks(1, body)
     assert votes == [0, 1]
+
+
+def test_pagerank_ranks_is_stream_ordered():
+    """PageRank.ranks(s) right after the phases (no host sync): the returned tensor must be
+    readable on the current stream.  Before the fix .cpu() could run ahead of the copy on `s`
+    and return recycled memory (seen as r ~ 3e-42 on the second run in one process)."""
+    src, dst = synth.rmat(12, 16)
+    V = 1 << 12
+    want = oracle.pagerank(V, src, dst, 2).astype(np.float64)
+
+    def body(r, G):
+        rt.set_config(mech=_lib.MECH_FUSED)
+        s = torch.cuda.Stream()
+        P = wl.PageRank(V, src, dst, 4096, stream=s, hot=0)
+        for k in range(2):
+            P.step(s, barrier=(k == 1))
+        out = (P.v0, P.v1, P.ranks(s).cpu().numpy())
+        P.free()
+        return out
+
+    for _ in range(4):
+        for v0, v1, r in run_ranks(2, body):
+            assert np.max(np.abs(r - want[v0:v1]) / want[v0:v1]) <= 1e-5
