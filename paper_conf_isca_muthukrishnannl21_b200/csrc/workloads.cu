@@ -84,6 +84,9 @@ template <bool TALLY> struct JCfg {
     static constexpr int minb = TALLY ? 3 : 4;
 };
 constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
+#ifndef PROACT_JACOBI_OUT_EVICT_LAST   // G > 1: output rows evict-last until the agent has read them
+#define PROACT_JACOBI_OUT_EVICT_LAST 0
+#endif
 #ifndef PROACT_JACOBI_RING
 #define PROACT_JACOBI_RING 16
 #endif
@@ -258,6 +261,8 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
         return;
     }
     char *outb = lc.ctx->region[p.region_out].base;
+    uint64_t pol_out = 0;
+    if (PROACT_JACOBI_OUT_EVICT_LAST) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_out));
     uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
     uint32_t kt = 0;   // tiles handed to the committer
     for (;;) {
@@ -310,8 +315,15 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     if (j + 3 == N - 1) o.w = cur.w;
                 }
                 const uint64_t off = ((uint64_t)i * N + j) * 4;
-                if (lc.mech == PROACT_MECH_INLINE) proact::put(lc, p.region_out, off, o);
-                else *reinterpret_cast<float4 *>(outb + off) = o;
+                if (lc.mech == PROACT_MECH_INLINE) {
+                    proact::put(lc, p.region_out, off, o);
+                } else if (PROACT_JACOBI_OUT_EVICT_LAST && tally) {
+                    // the agent pushes this chunk within microseconds: keep it in L2 for that read
+                    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                                 ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
+                } else {
+                    *reinterpret_cast<float4 *>(outb + off) = o;
+                }
             }
             __syncwarp();
             if (lane == 0) {
