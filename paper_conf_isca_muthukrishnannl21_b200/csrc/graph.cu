@@ -36,7 +36,10 @@ namespace {
 #define PROACT_GB 256
 #endif
 constexpr int GB = PROACT_GB;      // threads per CTA
-constexpr int GT = 1024;           // vertices per tile (4 KiB of output, the paper's L279)
+#ifndef PROACT_GT   // 512: PageRank 1.035 vs 1.065 ms at 1024 (smaller per-group accumulators leave
+#define PROACT_GT 512 // more L1 as landing space for the gathers), SSSP unchanged
+#endif
+constexpr int GT = PROACT_GT;      // vertices per tile (2 KiB of output)
 constexpr int GL = 8;              // lanes per light vertex
 // consecutive in-edges per thread per round (merge path) and CTAs per SM, measured on B200
 // (tools/sweep_graph.py): PageRank 4 / 8 (1.65 ms at RMAT-24; 8 / 6: 2.2 ms), SSSP 2 / 6
