@@ -281,14 +281,14 @@ def main():
             return statistics.median(ts)
 
         best = rt.autotune(f"bench_jacobi_N{N}_G{world}", run_point,
-                           "mech=0;chunk=131072,1048576;warps=16,32,64;push=1;akern=1")
+                           "mech=0;chunk=131072,1048576;warps=8,16,32;push=1;akern=1")
         if best["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
             for rid in J.rid:
                 rt.rechunk(rid, best["chunk_bytes"])
         cfg = rt.set_config(mech=best["mech"], agent_warps=best["agent_warps"], push=best["push"],
                             agent_kernel=best["agent_kernel"], chunk_bytes=best["chunk_bytes"])
         chunk = best["chunk_bytes"]
-        tuned = "proact_autotune: chunk {128K, 1M} x agent warps {16, 32, 64}"
+        tuned = "proact_autotune: chunk {128K, 1M} x agent warps {8, 16, 32}"
 
     def step():
         if mode["nccl"]:
