@@ -186,7 +186,7 @@ def run_reference(args, dist_rank: int) -> None:
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)   # >= 3 nvidia-smi samples (100 ms) in the timed region
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="proact", choices=["proact", "reference"])
     ap.add_argument("--mech", default="fused")
