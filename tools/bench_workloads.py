@@ -91,9 +91,14 @@ def pagerank(args, src, dst, V):
                 b.record(s)
                 torch.cuda.synchronize()
                 return a.elapsed_time(b) / n
+            w0 = rt.get_config()["agent_warps"]
             phase_ms(_lib.MECH_ELIDE, 2)
-            out["overhead"] = {"local_ms": phase_ms(_lib.MECH_LOCAL), "elide_ms": phase_ms(_lib.MECH_ELIDE)}
-            rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+            out["overhead"] = {"local_ms": phase_ms(_lib.MECH_LOCAL), "elide_ms": phase_ms(_lib.MECH_ELIDE),
+                               "agent_warps": w0}
+            rt.set_config(agent_warps=4)   # PageRank pushes 4 B/vertex: a few agent CTAs suffice
+            phase_ms(_lib.MECH_ELIDE, 2)
+            out["overhead"]["elide4_ms"] = phase_ms(_lib.MECH_ELIDE)
+            rt.set_config(agent_warps=w0, mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
         P.free()
         return out
     res = run_ranks(args.ranks, body)
@@ -122,6 +127,8 @@ def pagerank(args, src, dst, V):
         o = res[0]["overhead"]
         line["overhead"] = {"local_ms_per_phase": o["local_ms"], "elide_ms_per_phase": o["elide_ms"],
                             "tracking_overhead_frac": o["elide_ms"] / o["local_ms"] - 1.0,
+                            "agent_warps": o["agent_warps"],
+                            "tracking_overhead_frac_4_agent_warps": o["elide4_ms"] / o["local_ms"] - 1.0,
                             "note": "G=1: ELIDE keeps tallies + agent with remote stores skipped (Fig. 8 methodology)"}
     if not args.no_cpu:
         import oracle
@@ -187,14 +194,17 @@ def sssp(args, src, dst, V):
                "nhot": S.nhot, "e_own": S.e_own}
         if G == 1:   # tracking overhead: a whole run under ELIDE vs LOCAL
             oh = {}
-            for name, mech in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE), ("local", _lib.MECH_LOCAL)):
-                rt.set_config(mech=mech)
+            w0 = rt.get_config()["agent_warps"]
+            for name, mech, aw in (("local", _lib.MECH_LOCAL, w0), ("elide", _lib.MECH_ELIDE, w0),
+                                   ("local", _lib.MECH_LOCAL, w0), ("elide4", _lib.MECH_ELIDE, 4)):
+                rt.set_config(mech=mech, agent_warps=aw)
                 S.reset()
                 t0 = time.perf_counter()
                 S.run(stream=st)
                 oh[name] = time.perf_counter() - t0
+            oh["agent_warps"] = w0
             out["overhead"] = oh
-            rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
+            rt.set_config(agent_warps=w0, mech={v: k for k, v in _lib.MECH_NAMES.items()}[args.mech])
         S.free()
         return out
     epc = np.bincount(src // (args.chunk // 4), minlength=(V + args.chunk // 4 - 1) // (args.chunk // 4))
@@ -209,6 +219,8 @@ def sssp(args, src, dst, V):
         o = res[0]["overhead"]
         line["overhead"] = {"local_s_per_run": o["local"], "elide_s_per_run": o["elide"],
                             "tracking_overhead_frac": o["elide"] / o["local"] - 1.0,
+                            "agent_warps": o["agent_warps"],
+                            "tracking_overhead_frac_4_agent_warps": o["elide4"] / o["local"] - 1.0,
                             "note": "G=1: ELIDE keeps tallies + agent with remote stores skipped (Fig. 8 methodology)"}
     if args.ranks == 1:
         r0 = res[0]
