@@ -103,6 +103,9 @@ def _declare(L):
         "proact_jacobi_solve_host": (i, [vp, vp, ctypes.c_longlong, i, sz, i, vp,
                                          ctypes.POINTER(ctypes.c_ulonglong),
                                          ctypes.POINTER(ctypes.c_ulonglong)]),
+        "proact_jacobi_solve_host_pipelined": (i, [vp, vp, i, ctypes.c_longlong, i, sz, i, vp,
+                                                   ctypes.POINTER(ctypes.c_ulonglong),
+                                                   ctypes.POINTER(ctypes.c_ulonglong)]),
         "proact_graph_partition": (i, [vp, ctypes.c_ulonglong, ctypes.c_uint, i, ctypes.c_uint,
                                        ctypes.POINTER(ctypes.c_uint), vp]),
         "proact_graph_build": (i, [vp, vp, vp, ctypes.c_ulonglong, ctypes.c_uint, ctypes.c_uint,

@@ -810,6 +810,103 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
     return PROACT_OK;
 }
 
+// Pipelined host-buffer solves: nsolve independent solves, each with its own H2D of the input
+// and D2H of its result, over two device buffer sets so that solve k's phases overlap the H2D of
+// solve k+1 and the D2H of solve k-1 (PCIe is full duplex; both copies run on the copy engines
+// while the SMs compute).  Streams: `stream` computes, two library streams copy.
+namespace {
+struct JacobiPipe {
+    long long N = 0;
+    size_t chunk = 0;
+    float *buf[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};
+    int rid[2][2] = {{-1, -1}, {-1, -1}};
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_done[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
+};
+thread_local JacobiPipe jp;
+}  // namespace
+
+extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *const *h_outs, int nsolve,
+                                                  long long N, int iters, size_t chunk_bytes, int rows_per_tile,
+                                                  void *stream, unsigned long long *bytes_h2d,
+                                                  unsigned long long *bytes_d2h)
+{
+    const int G = proact_world(), g = proact_rank();
+    if (G <= 0) return PROACT_ERR_STATE;
+    if (!h_x0 || !h_outs || nsolve < 1 || N < 4 || N % 4 || iters < 0) return PROACT_ERR_INVALID;
+    for (int k = 0; k < nsolve; ++k)
+        if (!h_outs[k]) return PROACT_ERR_INVALID;
+    const long long r0 = N * g / G, r1 = N * (g + 1) / G;
+    const size_t rowb = (size_t)N * 4;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (jp.N && jp.N != N) return PROACT_ERR_STATE;   // regions cannot be unregistered
+    if (!jp.N) {
+        const uint64_t all = G >= 64 ? ~0ull : ((1ull << G) - 1);
+        for (int b = 0; b < 2; ++b)
+            for (int h = 0; h < 2; ++h) {
+                if (cudaMalloc((void **)&jp.buf[b][h], rowb * N) != cudaSuccess) return PROACT_ERR_NOMEM;
+                jp.rid[b][h] = proact_register_region((char *)jp.buf[b][h] + r0 * rowb, (r1 - r0) * rowb,
+                                                      chunk_bytes, all);
+                if (jp.rid[b][h] < 0) return jp.rid[b][h];
+            }
+        if (cudaStreamCreateWithFlags(&jp.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamCreateWithFlags(&jp.d2h, cudaStreamNonBlocking) != cudaSuccess)
+            return PROACT_ERR_CUDA;
+        for (int b = 0; b < 2; ++b)
+            if (cudaEventCreateWithFlags(&jp.ev_in[b], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&jp.ev_done[b], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&jp.ev_out[b], cudaEventDisableTiming) != cudaSuccess)
+                return PROACT_ERR_CUDA;
+        jp.N = N;
+        jp.chunk = chunk_bytes;
+    } else if (jp.chunk != chunk_bytes) {
+        for (int b = 0; b < 2; ++b)
+            for (int h = 0; h < 2; ++h) {
+                int rc = proact_region_rechunk(jp.rid[b][h], chunk_bytes);
+                if (rc) return rc;
+            }
+        jp.chunk = chunk_bytes;
+    }
+    // the copy streams start after everything already on `stream`
+    if (cudaEventRecord(jp.ev_out[0], s) != cudaSuccess || cudaEventRecord(jp.ev_out[1], s) != cudaSuccess)
+        return PROACT_ERR_CUDA;
+    auto h2d = [&](int k) -> int {   // input of solve k into set k & 1, once that set's last D2H read it
+        const int b = k & 1;
+        if (cudaStreamWaitEvent(jp.h2d, jp.ev_out[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
+        if (cudaMemcpyAsync(jp.buf[b][0], h_x0, rowb * N, cudaMemcpyHostToDevice, jp.h2d) != cudaSuccess)
+            return PROACT_ERR_CUDA;
+        return cudaEventRecord(jp.ev_in[b], jp.h2d) == cudaSuccess ? PROACT_OK : PROACT_ERR_CUDA;
+    };
+    int rc = h2d(0);
+    if (rc) return rc;
+    for (int k = 0; k < nsolve; ++k) {
+        const int b = k & 1;
+        if (k + 1 < nsolve && (rc = h2d(k + 1))) return rc;   // overlaps this solve's phases
+        if (cudaStreamWaitEvent(s, jp.ev_in[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
+        for (int it = 0; it < iters; ++it) {
+            const int in = jp.rid[b][it & 1], out = jp.rid[b][(it & 1) ^ 1];
+            if ((rc = proact_jacobi_phase(in, out, N, rows_per_tile, stream))) return rc;
+            if ((rc = proact_phase_sync(stream, it == iters - 1 ? PROACT_SYNC_BARRIER : PROACT_SYNC_SIGNAL)))
+                return rc;
+        }
+        if (cudaEventRecord(jp.ev_done[b], s) != cudaSuccess) return PROACT_ERR_CUDA;
+        if (cudaStreamWaitEvent(jp.d2h, jp.ev_done[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
+        const float *res = jp.buf[b][iters & 1];
+        if (cudaMemcpyAsync(h_outs[k] + r0 * N, res + r0 * N, (r1 - r0) * rowb, cudaMemcpyDeviceToHost, jp.d2h) !=
+            cudaSuccess)
+            return PROACT_ERR_CUDA;
+        // the next solve of set b (k + 2) overwrites these buffers only after its H2D, which waits
+        // for this event: no wait on `stream` here, so solve k + 1 computes during this D2H
+        if (cudaEventRecord(jp.ev_out[b], jp.d2h) != cudaSuccess) return PROACT_ERR_CUDA;
+    }
+    // completion on `stream`: the last D2H
+    for (int b = 0; b < 2; ++b)
+        if (cudaStreamWaitEvent(s, jp.ev_out[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
+    if (bytes_h2d) *bytes_h2d = (unsigned long long)(rowb * N);
+    if (bytes_d2h) *bytes_d2h = (unsigned long long)((r1 - r0) * rowb);
+    return PROACT_OK;
+}
+
 extern "C" {
 // Force-load this translation unit's kernels (called by proact_init).  Under CUDA's lazy module
 // loading the first launch of a kernel loads it, and a load waits for the device's running

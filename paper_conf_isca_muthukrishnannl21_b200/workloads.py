@@ -118,6 +118,22 @@ def jacobi_solve_host(x0_host, out_host, N: int, iters: int, chunk_bytes: int,
     return h2d.value, d2h.value
 
 
+def jacobi_solve_host_pipelined(x0_host, outs_host, N: int, iters: int, chunk_bytes: int,
+                                rows_per_tile: int = 16, stream=None) -> tuple[int, int]:
+    """proact_jacobi_solve_host_pipelined: len(outs_host) solves of x0_host, pipelined; complete
+    when `stream` is.  Returns the per-solve H2D / D2H byte counts."""
+    assert x0_host.dtype == torch.float32 and x0_host.is_contiguous()
+    for o in outs_host:
+        assert o.dtype == torch.float32 and o.is_contiguous()
+    ptrs = (ctypes.c_void_p * len(outs_host))(*[o.data_ptr() for o in outs_host])
+    h2d, d2h = ctypes.c_ulonglong(0), ctypes.c_ulonglong(0)
+    check(rt.lib().proact_jacobi_solve_host_pipelined(ctypes.c_void_p(x0_host.data_ptr()), ptrs, len(outs_host),
+                                                      N, iters, chunk_bytes, rows_per_tile, _s(stream),
+                                                      ctypes.byref(h2d), ctypes.byref(d2h)),
+          "jacobi_solve_host_pipelined")
+    return h2d.value, d2h.value
+
+
 # ------------------------------------------------------------------ banded Jacobi (NEXT-2)
 class Banded:
     """The paper's Jacobi (L271): A x = b with A banded (half-bandwidth w, DIA layout), x an

@@ -167,6 +167,33 @@ def test_jacobi_e2e_host_buffers():
         assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
 
 
+@pytest.mark.parametrize("G,iters", [(1, 7), (2, 6), (2, 0)])
+def test_jacobi_e2e_pipelined_host_buffers(G, iters):
+    """proact_jacobi_solve_host_pipelined: every one of the nsolve outputs (two device buffer
+    sets reused in turn, copies on library streams) equals the oracle, over two calls."""
+    N = 512
+    x0 = synth.jacobi_init(N)
+    want = oracle.jacobi(x0, iters) if iters else x0
+
+    def body(r, G_):
+        xh = torch.from_numpy(x0).pin_memory()
+        s = torch.cuda.Stream()
+        got = []
+        for nsolve in (5, 2):
+            outs = [torch.full((N, N), -1.0, dtype=torch.float32).pin_memory() for _ in range(nsolve)]
+            h2d, d2h = wl.jacobi_solve_host_pipelined(xh, outs, N, iters, 16384, stream=s)
+            s.synchronize()
+            r0, r1 = wl.row_split(N, G_, r)
+            got.append(([o.numpy()[r0:r1].copy() for o in outs], (r0, r1), h2d, d2h))
+        return got
+
+    for per_rank in run_ranks(G, body):
+        for rows_list, (r0, r1), h2d, d2h in per_rank:
+            for rows in rows_list:
+                assert np.array_equal(rows.view(np.uint32), want[r0:r1].view(np.uint32))
+            assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
+
+
 @pytest.mark.parametrize("G,N,chunk", [(1, 4, 4096), (2, 8, 4096), (2, 1024, 4112), (3, 36, 4096)])
 def test_jacobi_degenerate_and_odd_chunks(G, N, chunk):
     """All-boundary grids (N = 4: every cell copied through), ranks owning a couple of rows,
