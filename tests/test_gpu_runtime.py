@@ -75,13 +75,16 @@ def test_bench_two_processes_json_line():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--steps", "1", "--warmup", "3", "--grid-n", "1024", "--iters", "4", "--backend", "gloo",
-           "--no-cpu", "--no-e2e"]
+           "--no-cpu"]
     r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout + r.stderr
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "strong"
+    # e2e through both host-buffer entry points (sequential and pipelined), two processes
+    assert d["e2e"]["value"] > 0 and d["e2e"]["sequential_value"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] == 1024 * 1024 * 4
     # the same ranks time the bulk-copy and naive-P2P baselines (NCCL needs distinct GPUs)
     assert set(d["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
     assert all(v > 0 for v in d["baselines_iters_per_s"].values())
