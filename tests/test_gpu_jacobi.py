@@ -167,7 +167,7 @@ def test_jacobi_e2e_host_buffers():
         assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
 
 
-@pytest.mark.parametrize("G,iters", [(1, 7), (2, 6), (2, 0)])
+@pytest.mark.parametrize("G,iters", [(1, 7), (2, 6), (2, 0), (3, 5)])
 def test_jacobi_e2e_pipelined_host_buffers(G, iters):
     """proact_jacobi_solve_host_pipelined: every one of the nsolve outputs (two device buffer
     sets reused in turn, copies on library streams) equals the oracle, over two calls."""
