@@ -51,6 +51,36 @@ def _peaks():
         return {"hbm_gbs": 6650.0}, "fallback"
 
 
+def _sustained_copy_gbs(stream, seconds: float) -> dict:
+    """torch copy_ of 1 Gi bf16 elements (MEASURED_PEAKS.json's recipe: read + write bytes) back to
+    back for `seconds`, per-launch CUDA events; the median of the second half is the sustained
+    copy bandwidth.  Calibration only: outside the timed region, not one of our kernels."""
+    import torch
+    n = 1 << 30
+    a = torch.empty(n, dtype=torch.bfloat16, device="cuda")
+    b = torch.empty_like(a)
+    a.fill_(1.0)
+    with torch.cuda.stream(stream):
+        b.copy_(a)
+        torch.cuda.synchronize()
+        per = 4.0 * n / 6.4e12                     # rough seconds per copy, sizes the run
+        reps = max(8, int(seconds / per))
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+        for e0, e1 in ev:
+            e0.record(stream)
+            b.copy_(a)
+            e1.record(stream)
+        torch.cuda.synchronize()
+    t = [e0.elapsed_time(e1) for e0, e1 in ev]
+    burst = min(t)
+    late = statistics.median(t[reps // 2:])
+    del a, b
+    torch.cuda.empty_cache()
+    return {"gbs": 4.0 * n / (late * 1e-3) / 1e9, "burst_gbs": 4.0 * n / (burst * 1e-3) / 1e9,
+            "launches": reps, "note": "median of the second half of back-to-back 1 Gi bf16 copies, "
+                                      "same recipe as MEASURED_PEAKS.json hbm_gbs; context, not the peak"}
+
+
 def _traffic_from_profiles():
     """dram bytes per launch of jacobi_kernel from the committed ncu --set full summary."""
     p = os.path.join(ROOT, "profiles", "ncu_jacobi_summary.json")
@@ -192,7 +222,7 @@ def main():
     ap.add_argument("--mech", default="fused")
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--warps", type=int, default=0)
-    ap.add_argument("--rpt", type=int, default=16)
+    ap.add_argument("--rpt", type=int, default=32)   # sustained-load sweep r01v: 32 > 64 > 16 > 8
     ap.add_argument("--iters", type=int, default=ITERS)
     ap.add_argument("--grid-n", dest="n", type=int, default=N_GRID)
     ap.add_argument("--no-cpu", action="store_true")
@@ -360,7 +390,10 @@ def main():
         evs.append((a, b))
     torch.cuda.synchronize()
     kms_isolated = statistics.mean(a.elapsed_time(b) for a, b in evs)
-    kms = statistics.mean(a.elapsed_time(b) for a, b in live_ev) if live_ev else kms_isolated
+    live_t = [a.elapsed_time(b) for a, b in live_ev]
+    kms = statistics.mean(live_t) if live_t else kms_isolated
+    live_trend = ([statistics.median(live_t[:max(1, len(live_t) // 10)]),
+                   statistics.median(live_t[len(live_t) // 2:])] if live_t else None)
     nrows = J.r1 - J.r0
     alg_bytes = 8.0 * N * nrows          # read x^k + write x^{k+1} of my rows
     peaks, src = _peaks()
@@ -378,12 +411,20 @@ def main():
                      "frac": max(t_hbm_us, t_nvl_us) / t_phase_us,
                      "nvlink_ingress_GBps_per_gpu": ingress / (t_phase_us * 1e-6) / 1e9, "nvlink_peak_GBps": NVL,
                      "note": "per rank and phase; NVLink 900 GB/s/direction nominal (B200_PROFILING.md)"}
+    # context for the live fraction: the MEASURED_PEAKS.json copy recipe (1 Gi bf16 elements,
+    # read + write bytes) run back to back for about as long as the timed region, on this box, now
+    sustained = None
+    if os.environ.get("PROACT_BENCH_NO_SUSTAINED") != "1":
+        sustained = _sustained_copy_gbs(s, max(0.1, ms / 1000.0))
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": _traffic_from_profiles(),
                 "kernel": "jacobi_kernel", "kernel_ms": kms, "alg_bytes_per_launch": alg_bytes,
                 "kernel_ms_source": ("mean of %d launches timed live in the timed region" % len(live_ev)
                                      if live_ev else "isolated 20-launch run"),
                 "kernel_ms_isolated": kms_isolated,
+                "kernel_ms_live_first10pct_last50pct": live_trend,
+                "sustained_copy": sustained,
+                "frac_of_sustained_copy": (achieved / sustained["gbs"]) if sustained else None,
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({src})"}
 
     # ---- tracking overhead (Sec. V-C, Fig. 8): the same step with

@@ -136,10 +136,11 @@ def test_config2_full_size_sampled():
     """Config 2 size (16384^2, 100 iterations) in bench.py's launch configuration (G=1, FUSED),
     checked on sampled cells computed one by one by the oracle."""
     N, iters = 16384, 100
-    (rep, _, _), = run_ranks(1, _run_jacobi, N, iters, 128 * 1024, _lib.MECH_FUSED)
+    (rep, _, _), = run_ranks(1, _run_jacobi, N, iters, 128 * 1024, _lib.MECH_FUSED, rpt=32)
     rng = np.random.default_rng(0)
     pts = [(int(a), int(b)) for a, b in rng.integers(iters + 1, N - iters - 2, size=(12, 2))]
-    pts += [(iters + 1, iters + 1), (N - iters - 2, N - iters - 2), (8192, 1023), (8191, 1024)]
+    pts += [(iters + 1, iters + 1), (N - iters - 2, N - iters - 2), (8192, 1023), (8191, 1024),
+            (8223, 2047), (8224, 2048)]   # tile-band and strip boundaries at rows_per_tile = 32
     for i, j in pts:
         assert rep[i, j] == _window_oracle(N, iters, i, j), (i, j)
     # boundary rows/cols are copied through (Dirichlet)
