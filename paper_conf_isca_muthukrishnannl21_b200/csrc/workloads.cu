@@ -75,7 +75,14 @@ __device__ __forceinline__ float ld_f(const float *p)
 // shared memory) and release slots on per-slot "empty" mbarriers.  The row stream runs across
 // the CTA's tiles without draining.  Every input row is read from HBM once per tile (+2 halo
 // rows per tile, L2 hits); outputs are 16-byte stores.
-constexpr int JC = 8;                   // compute warps
+#ifndef PROACT_JACOBI_JC
+#define PROACT_JACOBI_JC 8
+#endif
+#ifndef PROACT_JACOBI_JV
+#define PROACT_JACOBI_JV 1
+#endif
+constexpr int JC = PROACT_JACOBI_JC;    // compute warps
+constexpr int JV = PROACT_JACOBI_JV;    // float4 column groups per compute thread (JC * JV = 8)
 // Two instantiations: TALLY = false (no remote destinations this launch: LOCAL / INLINE / BULK /
 // G = 1) has 8 compute + 1 TMA warp and the register budget of 4 CTAs/SM; TALLY = true adds a
 // committer warp that publishes the tile tallies so the compute warps never wait on a release.
@@ -83,7 +90,7 @@ template <bool TALLY> struct JCfg {
     static constexpr int threads = (JC + 1 + (TALLY ? 1 : 0)) * 32;
     static constexpr int minb = TALLY ? 3 : 4;
 };
-constexpr int JW = JC * 32 * 4;         // strip width in columns = 4 KiB of a row
+constexpr int JW = JC * 32 * 4 * JV;    // strip width in columns = 4 KiB of a row
 #ifndef PROACT_JACOBI_OUT_EVICT_LAST   // G > 1: output rows evict-last until the agent has read them
 #define PROACT_JACOBI_OUT_EVICT_LAST 0
 #endif
@@ -274,45 +281,61 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             break;
         }
         const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
-        const int x = 4 * tid, j = T.c0 + x;
-        const bool act = j < T.c1;
-        const float *ringf = ring + 4 + x;
-        float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur, dn = up;
+        // group g of this thread: columns [c0 + 4*tid + g*GW, +4), GW = the compute warps' width
+        constexpr int GW = JC * 32 * 4;
+        const float *ringf = ring + 4 + 4 * tid;
+        float4 up[JV], cur[JV], dn[JV];
+        bool act[JV];
+#pragma unroll
+        for (int g = 0; g < JV; ++g) {
+            act[g] = T.c0 + 4 * tid + g * GW < T.c1;
+            up[g] = make_float4(0.f, 0.f, 0.f, 0.f);
+            dn[g] = up[g];
+        }
         if (T.i0 > 0) {   // top halo / previous row: registers only, release at once
             mbar_wait(&full[q % JS], (q / JS) & 1u);
-            if (act) up = lds128(ringf + (q % JS) * SLOT);
+#pragma unroll
+            for (int g = 0; g < JV; ++g)
+                if (act[g]) up[g] = lds128(ringf + (q % JS) * SLOT + g * GW);
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[q % JS]);
             ++q;
         }
         uint32_t qcur = q;
         mbar_wait(&full[q % JS], (q / JS) & 1u);
-        cur = act ? lds128(ringf + (q % JS) * SLOT) : up;
+#pragma unroll
+        for (int g = 0; g < JV; ++g) cur[g] = act[g] ? lds128(ringf + (q % JS) * SLOT + g * GW) : up[g];
         ++q;
         for (int i = T.i0; i < T.i1; ++i) {
             const uint32_t qdn = q;
             const bool has_dn = i + 1 <= T.klast;
             if (has_dn) {
                 mbar_wait(&full[q % JS], (q / JS) & 1u);
-                if (act) dn = lds128(ringf + (q % JS) * SLOT);
+#pragma unroll
+                for (int g = 0; g < JV; ++g)
+                    if (act[g]) dn[g] = lds128(ringf + (q % JS) * SLOT + g * GW);
                 ++q;
             }
-            const float *cs = ringf + (qcur % JS) * SLOT;
-            float lft = __shfl_up_sync(0xFFFFFFFFu, cur.w, 1);
-            float rgt = __shfl_down_sync(0xFFFFFFFFu, cur.x, 1);
+#pragma unroll
+            for (int g = 0; g < JV; ++g) {
+            const int j = T.c0 + 4 * tid + g * GW;
+            const float *cs = ringf + (qcur % JS) * SLOT + g * GW;
+            float lft = __shfl_up_sync(0xFFFFFFFFu, cur[g].w, 1);
+            float rgt = __shfl_down_sync(0xFFFFFFFFu, cur[g].x, 1);
             if (lane == 0) lft = cs[-1];
             if (lane == 31) rgt = cs[4];
-            if (act) {
+            if (act[g]) {
+                const float4 c = cur[g], u = up[g], d = dn[g];
                 float4 o;
                 if (i == 0 || i == N - 1) {
-                    o = cur;
+                    o = c;
                 } else {
-                    o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.x, dn.x), __fadd_rn(lft, cur.y)));
-                    o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.y, dn.y), __fadd_rn(cur.x, cur.z)));
-                    o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.z, dn.z), __fadd_rn(cur.y, cur.w)));
-                    o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up.w, dn.w), __fadd_rn(cur.z, rgt)));
-                    if (j == 0) o.x = cur.x;
-                    if (j + 3 == N - 1) o.w = cur.w;
+                    o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.x, d.x), __fadd_rn(lft, c.y)));
+                    o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.y, d.y), __fadd_rn(c.x, c.z)));
+                    o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.z, d.z), __fadd_rn(c.y, c.w)));
+                    o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.w, d.w), __fadd_rn(c.z, rgt)));
+                    if (j == 0) o.x = c.x;
+                    if (j + 3 == N - 1) o.w = c.w;
                 }
                 const uint64_t off = ((uint64_t)i * N + j) * 4;
                 if (lc.mech == PROACT_MECH_INLINE) {
@@ -325,13 +348,17 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     *reinterpret_cast<float4 *>(outb + off) = o;
                 }
             }
+            }
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&empty[qcur % JS]);                    // row i: done
                 if (has_dn && i + 1 == T.i1) mbar_arrive(&empty[qdn % JS]);   // bottom halo row
             }
-            up = cur;
-            cur = dn;
+#pragma unroll
+            for (int g = 0; g < JV; ++g) {
+                up[g] = cur[g];
+                cur[g] = dn[g];
+            }
             qcur = qdn;
         }
         if (tally && TALLY) {   // hand the tile to the committer warp; never run > 2 tiles ahead
