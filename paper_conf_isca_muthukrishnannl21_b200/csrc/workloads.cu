@@ -12,6 +12,7 @@
 #include <stdint.h>
 
 #include <cstdlib>
+#include <type_traits>
 
 #include "proact.h"
 #include "proact_device.cuh"
@@ -306,61 +307,72 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 #pragma unroll
         for (int g = 0; g < JV; ++g) cur[g] = act[g] ? lds128(ringf + (q % JS) * SLOT + g * GW) : up[g];
         ++q;
-        for (int i = T.i0; i < T.i1; ++i) {
-            const uint32_t qdn = q;
-            const bool has_dn = i + 1 <= T.klast;
-            if (has_dn) {
-                mbar_wait(&full[q % JS], (q / JS) & 1u);
-#pragma unroll
-                for (int g = 0; g < JV; ++g)
-                    if (act[g]) dn[g] = lds128(ringf + (q % JS) * SLOT + g * GW);
-                ++q;
-            }
-#pragma unroll
-            for (int g = 0; g < JV; ++g) {
-            const int j = T.c0 + 4 * tid + g * GW;
-            const float *cs = ringf + (qcur % JS) * SLOT + g * GW;
-            float lft = __shfl_up_sync(0xFFFFFFFFu, cur[g].w, 1);
-            float rgt = __shfl_down_sync(0xFFFFFFFFu, cur[g].x, 1);
-            if (lane == 0) lft = cs[-1];
-            if (lane == 31) rgt = cs[4];
-            if (act[g]) {
-                const float4 c = cur[g], u = up[g], d = dn[g];
-                float4 o;
-                if (i == 0 || i == N - 1) {
-                    o = c;
-                } else {
-                    o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.x, d.x), __fadd_rn(lft, c.y)));
-                    o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.y, d.y), __fadd_rn(c.x, c.z)));
-                    o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.z, d.z), __fadd_rn(c.y, c.w)));
-                    o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.w, d.w), __fadd_rn(c.z, rgt)));
-                    if (j == 0) o.x = c.x;
-                    if (j + 3 == N - 1) o.w = c.w;
+        // interior tiles (no Dirichlet row or column, full strip, plain stores) run a copy of the
+        // row loop with those checks compiled out
+        const bool fast = T.i0 > 0 && T.i1 < N && T.c0 > 0 && T.c0 + JW < N &&
+                          lc.mech != PROACT_MECH_INLINE && !(PROACT_JACOBI_OUT_EVICT_LAST && tally);
+        auto rows = [&](auto fast_tag) {
+            constexpr bool FAST = decltype(fast_tag)::value;
+            for (int i = T.i0; i < T.i1; ++i) {
+                const uint32_t qdn = q;
+                const bool has_dn = i + 1 <= T.klast;
+                if (has_dn) {
+                    mbar_wait(&full[q % JS], (q / JS) & 1u);
+    #pragma unroll
+                    for (int g = 0; g < JV; ++g)
+                        if (act[g]) dn[g] = lds128(ringf + (q % JS) * SLOT + g * GW);
+                    ++q;
                 }
-                const uint64_t off = ((uint64_t)i * N + j) * 4;
-                if (lc.mech == PROACT_MECH_INLINE) {
-                    proact::put(lc, p.region_out, off, o);
-                } else if (PROACT_JACOBI_OUT_EVICT_LAST && tally) {
-                    // the agent pushes this chunk within microseconds: keep it in L2 for that read
-                    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
-                                 ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
-                } else {
-                    *reinterpret_cast<float4 *>(outb + off) = o;
+    #pragma unroll
+                for (int g = 0; g < JV; ++g) {
+                const int j = T.c0 + 4 * tid + g * GW;
+                const float *cs = ringf + (qcur % JS) * SLOT + g * GW;
+                float lft = __shfl_up_sync(0xFFFFFFFFu, cur[g].w, 1);
+                float rgt = __shfl_down_sync(0xFFFFFFFFu, cur[g].x, 1);
+                if (lane == 0) lft = cs[-1];
+                if (lane == 31) rgt = cs[4];
+                if (FAST || act[g]) {
+                    const float4 c = cur[g], u = up[g], d = dn[g];
+                    float4 o;
+                    if (!FAST && (i == 0 || i == N - 1)) {
+                        o = c;
+                    } else {
+                        o.x = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.x, d.x), __fadd_rn(lft, c.y)));
+                        o.y = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.y, d.y), __fadd_rn(c.x, c.z)));
+                        o.z = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.z, d.z), __fadd_rn(c.y, c.w)));
+                        o.w = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(u.w, d.w), __fadd_rn(c.z, rgt)));
+                        if (!FAST && j == 0) o.x = c.x;
+                        if (!FAST && j + 3 == N - 1) o.w = c.w;
+                    }
+                    const uint64_t off = ((uint64_t)i * N + j) * 4;
+                    if (!FAST && lc.mech == PROACT_MECH_INLINE) {
+                        proact::put(lc, p.region_out, off, o);
+                    } else if (!FAST && PROACT_JACOBI_OUT_EVICT_LAST && tally) {
+                        // the agent pushes this chunk within microseconds: keep it in L2 for that read
+                        asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                                     ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
+                    } else {
+                        *reinterpret_cast<float4 *>(outb + off) = o;
+                    }
                 }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    mbar_arrive(&empty[qcur % JS]);                    // row i: done
+                    if (has_dn && i + 1 == T.i1) mbar_arrive(&empty[qdn % JS]);   // bottom halo row
+                }
+    #pragma unroll
+                for (int g = 0; g < JV; ++g) {
+                    up[g] = cur[g];
+                    cur[g] = dn[g];
+                }
+                qcur = qdn;
             }
-            }
-            __syncwarp();
-            if (lane == 0) {
-                mbar_arrive(&empty[qcur % JS]);                    // row i: done
-                if (has_dn && i + 1 == T.i1) mbar_arrive(&empty[qdn % JS]);   // bottom halo row
-            }
-#pragma unroll
-            for (int g = 0; g < JV; ++g) {
-                up[g] = cur[g];
-                cur[g] = dn[g];
-            }
-            qcur = qdn;
-        }
+        };
+        if (fast)
+            rows(std::true_type{});
+        else
+            rows(std::false_type{});
         if (tally && TALLY) {   // hand the tile to the committer warp; never run > 2 tiles ahead
             __syncwarp();
             if (lane == 0) mbar_arrive(&tdone[kt & 1u]);
