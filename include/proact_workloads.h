@@ -63,8 +63,9 @@ int proact_jacobi_solve_host(const float *h_x0, float *h_out, long long N, int i
  * path): each solve copies h_x0 in (full grid), runs `iters` phases (BARRIER on the last) and
  * copies this rank's rows of its result out to h_outs[k] (nsolve host pointers, pinned), like
  * proact_jacobi_solve_host.  Two library-owned device buffer sets (4 registered regions on the
- * first call) and two library copy streams let solve k's phases overlap the H2D of solve k+1 and
- * the D2H of solve k-1.  Asynchronous: everything is complete when `stream` is.  COLLECTIVE.
+ * first call), an unregistered H2D staging buffer (moved into the set by a device copy at the
+ * start of each solve) and two library copy streams let solve k's phases overlap the H2D of
+ * solve k+1 and the D2H of solve k-1, the two copies running at the same time.  Asynchronous: everything is complete when `stream` is.  COLLECTIVE.
  * *bytes_h2d / *bytes_d2h get the per-solve counts. */
 int proact_jacobi_solve_host_pipelined(const float *h_x0, float *const *h_outs, int nsolve, long long N,
                                        int iters, size_t chunk_bytes, int rows_per_tile, void *stream,

@@ -861,6 +861,8 @@ struct JacobiPipe {
     int rid[2][2] = {{-1, -1}, {-1, -1}};
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t ev_in[2] = {nullptr, nullptr}, ev_done[2] = {nullptr, nullptr}, ev_out[2] = {nullptr, nullptr};
+    float *stage = nullptr;                 // H2D landing buffer (not a region)
+    cudaEvent_t ev_staged = nullptr, ev_stage_free = nullptr;
 };
 thread_local JacobiPipe jp;
 }  // namespace
@@ -896,6 +898,10 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
                 cudaEventCreateWithFlags(&jp.ev_done[b], cudaEventDisableTiming) != cudaSuccess ||
                 cudaEventCreateWithFlags(&jp.ev_out[b], cudaEventDisableTiming) != cudaSuccess)
                 return PROACT_ERR_CUDA;
+        if (cudaMalloc((void **)&jp.stage, rowb * N) != cudaSuccess) return PROACT_ERR_NOMEM;
+        if (cudaEventCreateWithFlags(&jp.ev_staged, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&jp.ev_stage_free, cudaEventDisableTiming) != cudaSuccess)
+            return PROACT_ERR_CUDA;
         jp.N = N;
         jp.chunk = chunk_bytes;
     } else if (jp.chunk != chunk_bytes) {
@@ -907,21 +913,30 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
         jp.chunk = chunk_bytes;
     }
     // the copy streams start after everything already on `stream`
-    if (cudaEventRecord(jp.ev_out[0], s) != cudaSuccess || cudaEventRecord(jp.ev_out[1], s) != cudaSuccess)
+    if (cudaEventRecord(jp.ev_out[0], s) != cudaSuccess || cudaEventRecord(jp.ev_out[1], s) != cudaSuccess ||
+        cudaEventRecord(jp.ev_stage_free, s) != cudaSuccess)
         return PROACT_ERR_CUDA;
-    auto h2d = [&](int k) -> int {   // input of solve k into set k & 1, once that set's last D2H read it
-        const int b = k & 1;
-        if (cudaStreamWaitEvent(jp.h2d, jp.ev_out[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
-        if (cudaMemcpyAsync(jp.buf[b][0], h_x0, rowb * N, cudaMemcpyHostToDevice, jp.h2d) != cudaSuccess)
+    // H2D of solve k lands in the staging buffer (it waits only for the previous solve's device
+    // copy out of it), so it never queues behind the D2H of solve k - 2 that reads set k & 1:
+    // H2D and D2H run at the same time on the full-duplex link, both under the phases
+    auto h2d = [&](int k) -> int {
+        (void)k;
+        if (cudaStreamWaitEvent(jp.h2d, jp.ev_stage_free, 0) != cudaSuccess) return PROACT_ERR_CUDA;
+        if (cudaMemcpyAsync(jp.stage, h_x0, rowb * N, cudaMemcpyHostToDevice, jp.h2d) != cudaSuccess)
             return PROACT_ERR_CUDA;
-        return cudaEventRecord(jp.ev_in[b], jp.h2d) == cudaSuccess ? PROACT_OK : PROACT_ERR_CUDA;
+        return cudaEventRecord(jp.ev_staged, jp.h2d) == cudaSuccess ? PROACT_OK : PROACT_ERR_CUDA;
     };
     int rc = h2d(0);
     if (rc) return rc;
     for (int k = 0; k < nsolve; ++k) {
         const int b = k & 1;
+        // set b is free once solve k - 2's D2H read it; the input moves in by a device copy
+        if (cudaStreamWaitEvent(s, jp.ev_staged, 0) != cudaSuccess ||
+            cudaStreamWaitEvent(s, jp.ev_out[b], 0) != cudaSuccess ||
+            cudaMemcpyAsync(jp.buf[b][0], jp.stage, rowb * N, cudaMemcpyDeviceToDevice, s) != cudaSuccess ||
+            cudaEventRecord(jp.ev_stage_free, s) != cudaSuccess)
+            return PROACT_ERR_CUDA;
         if (k + 1 < nsolve && (rc = h2d(k + 1))) return rc;   // overlaps this solve's phases
-        if (cudaStreamWaitEvent(s, jp.ev_in[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
         for (int it = 0; it < iters; ++it) {
             const int in = jp.rid[b][it & 1], out = jp.rid[b][(it & 1) ^ 1];
             if ((rc = proact_jacobi_phase(in, out, N, rows_per_tile, stream))) return rc;
