@@ -93,10 +93,26 @@ enum {
 enum {
     PROACT_AGENT_FUSED = 0,    /* leading CTAs of the producer's own grid (cooperative launch on a
                                   dedicated GPU: co-residency guaranteed); shares its registers */
-    PROACT_AGENT_SEPARATE = 1  /* its own small kernel, launched first on a high-priority stream
+    PROACT_AGENT_SEPARATE = 1, /* its own small kernel, launched first on a high-priority stream
                                   (the paper's "independently launched long-lived kernel", L137),
-                                  with its own registers and a 128 KiB TMA staging ring; the
+                                  with its own registers and a 200 KiB TMA staging ring; the
                                   producer grid leaves room for it */
+    PROACT_AGENT_PRODUCER = 2  /* a transfer warp inside every producer CTA: the compute warps
+                                  stage each finished output row/tile in shared memory, the
+                                  transfer warp bulk-stores it (TMA, cp.async.bulk smem->global)
+                                  to the local replica and to every destination mirror, and once
+                                  the stores completed counts the chunk's DELIVERED bytes; the
+                                  last contributor publishes the chunk's arrival flags.  No
+                                  read-back of the produced bytes, no agent SMs (B200 re-design
+                                  of L137's specialised transfer warps).  Only for kernels
+                                  launched with PROACT_LAUNCH_TILE_PUSH; other launches fall back
+                                  to PROACT_AGENT_SEPARATE. */
+};
+
+/* ---- proact_launch_ex flags ------------------------------------------------------------- */
+enum {
+    PROACT_LAUNCH_TILE_PUSH = 1  /* the kernel implements proact::tile_pusher (a transfer warp that
+                                    pushes its own tiles) and may run under PROACT_AGENT_PRODUCER */
 };
 
 /* ---- phase synchronisation modes (a8) ----------------------------------------------------- */
@@ -209,10 +225,19 @@ int proact_region_rechunk(int region, size_t chunk_bytes);
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid,
                   unsigned block, void **args, size_t smem, void *stream);
 
+/* As proact_launch; `flags` = PROACT_LAUNCH_* capabilities of `kernel`. */
+int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsigned grid,
+                     unsigned block, void **args, size_t smem, void *stream, unsigned flags);
+
 /* 1 if the next proact_launch of this rank will run tallies and the agent (FUSED with G > 1, or
  * ELIDE), 0 if not (LOCAL / INLINE / BULK, or FUSED on a single rank): lets a workload pick a
  * kernel instantiation without the tally machinery. */
 int proact_launch_tallies(void);
+/* What the next launch of a kernel that supports PROACT_LAUNCH_TILE_PUSH should instantiate:
+ * 0 = plain stores (no tallies), 1 = tallies for a polling agent (FUSED / SEPARATE / ELIDE / DMA),
+ * 2 = tile push (PROACT_AGENT_PRODUCER: the kernel's transfer warp pushes its own tiles; launch
+ * it with PROACT_LAUNCH_TILE_PUSH). */
+int proact_launch_mode(void);
 
 /* Close phase e on `stream` (a8): peers get the credit "rank finished phase e" (write-after-read
  * guard for ping-pong replicas, reading R6), a BULK launch's copies are issued first, and in

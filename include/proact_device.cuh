@@ -87,6 +87,8 @@ struct dev_ctx {
                                                   (monotonic; the producer launch waits on it) */
     uint32_t *sched;                           /* [2] producer work counter + finished claimers:
                                                   dynamic tile scheduling (see claim_tile) */
+    uint32_t *started;                         /* epoch + 1 once the producer grid of that epoch
+                                                  started (SEPARATE agent start-up deadline) */
     region_dev region[PROACT_MAX_REGIONS];
 };
 
@@ -105,12 +107,21 @@ struct launch_ctx {
     uint16_t agent_warps;                      /* warps of those CTAs that poll/push */
     uint32_t piece_bytes;                      /* agent work unit */
     uint16_t discovery;                        /* PROACT_DISCOVER_* */
-    uint16_t flags;                            /* reserved */
+    uint16_t flags;                            /* LCF_* */
+};
+
+/* launch_ctx::flags */
+enum { LCF_SEPARATE = 1,   /* this is the SEPARATE agent kernel's copy (start-up deadline armed) */
+       LCF_TILE_PUSH = 2   /* PROACT_AGENT_PRODUCER: every producer CTA's transfer warp pushes its
+                              own tiles (proact::tile_pusher); counters count DELIVERED bytes and
+                              the last contributor of a chunk publishes its arrival flags */
 };
 
 /* error word encoding: (site << 8) | (-PROACT_ERR_*) */
 enum { SITE_AGENT_POLL = 1, SITE_AGENT_CREDIT = 2, SITE_WAIT_RANGE = 3, SITE_WAIT_ALL = 4,
-       SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7, SITE_AGENT_PUSH = 8 };
+       SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7, SITE_AGENT_PUSH = 8,
+       SITE_AGENT_START = 9,   /* SEPARATE agent: its producer grid never started (serialised?) */
+       SITE_TILE_PUSH = 10 };  /* tile pusher: credit wait / store completion */
 
 #ifdef __CUDACC__
 
@@ -287,6 +298,32 @@ __device__ __forceinline__ uint32_t piece_size(const launch_ctx &lc, const regio
  * this CTA's stores; acquire lets the LAST committer (old + b == expected, decided from the
  * returned value, reading R2) hand the chunk to the agent with everything ordered before it:
  * under QUEUE discovery it enqueues the chunk's pieces with release stores. */
+/* PROACT_AGENT_PRODUCER (LCF_TILE_PUSH): my chunk c of region r has been DELIVERED to every
+ * destination (its last contributor calls this, after acquiring every contributor's release):
+ * raise its arrival flag (gen << 1 | changed) on every destination and bump their arrival
+ * counters (a6), set my own flag, reset the counter for the next generation (reading R4).  The
+ * contributors each executed fence.acq_rel.sys after their bulk stores completed, so the
+ * release-store of the flag is ordered after every byte of the chunk at system scope. */
+__device__ __forceinline__ void publish_chunk(const launch_ctx &lc, int r, uint32_t c)
+{
+    const dev_ctx *C = lc.ctx;
+    const region_dev &R = C->region[r];
+    const uint32_t gen = lc.gen[r];
+    const uint32_t changed = (R.flags & PROACT_REGION_SPARSE) ? (R.changed_gen[c] == gen ? 1u : 0u) : 1u;
+    const uint32_t flag = (gen << 1) | changed;
+    const uint32_t g = R.chunk0 + c;
+    uint32_t m = dests_of(lc, R, c);
+    while (m) {
+        const int p = __ffs(m) - 1;
+        m &= m - 1;
+        st_release_sys(R.peer_arrive[p] + g, flag);
+        red_add_relaxed_sys(R.peer_arrive_count[p], 1u);
+        if (R.deliv) atomicAdd(&R.deliv[(uint64_t)c * C->world + p], 1u);
+    }
+    R.arrive[g] = flag;
+    R.counter[c] = 0u;
+}
+
 __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32_t c, uint32_t b)
 {
     const region_dev &R = lc.ctx->region[r];
@@ -294,6 +331,8 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
     const uint32_t ex = R.expected[c];
     if (old + b > ex) {
         raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
+    } else if (old + b == ex && (lc.flags & LCF_TILE_PUSH)) {
+        publish_chunk(lc, r, c);
     } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA) {
         const uint32_t piece = piece_size(lc, R);
         const uint32_t P = (R.chunk_bytes + piece - 1) / piece;
@@ -326,6 +365,26 @@ __device__ __forceinline__ void commit_span(const launch_ctx &lc, int r, uint64_
         commit_chunk(lc, r, c, b);
         rel += b;
         nbytes -= b;
+    }
+}
+
+/* Commit `nb` bytes at region offset `off` for each lane of the calling warp that has a span
+ * (has = true; whole warp, converged); lanes whose spans fall in the same chunk are merged into
+ * one release atomic (a3). */
+__device__ __forceinline__ void warp_commit(const launch_ctx &lc, int r, bool has, uint64_t off, uint32_t nb)
+{
+    if (!uses_agent(lc)) return;
+    const region_dev &R = lc.ctx->region[r];
+    uint64_t rel = off - R.own_off;
+    uint32_t c = has ? (uint32_t)(rel / R.chunk_bytes) : 0xFFFFFFFFu;
+    bool single = has && (uint32_t)((rel + nb - 1) / R.chunk_bytes) == c;
+    uint32_t key = single ? c : 0xFFFFFFFFu;
+    uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
+    const uint32_t tot = __reduce_add_sync(grp, single ? nb : 0u);   // spans may differ in size
+    if (single) {
+        if ((__ffs(grp) - 1) == (int)(threadIdx.x & 31)) commit_chunk(lc, r, c, tot);
+    } else if (has) {
+        commit_span(lc, r, off, nb);
     }
 }
 
@@ -439,12 +498,17 @@ __device__ __forceinline__ uint32_t chunk_flag(const launch_ctx &lc, int r, uint
 
 #ifdef __CUDACC__
 #include "proact_agent.cuh"
+#include "proact_tile.cuh"
 namespace proact {
 /* Agent CTAs (the first lc.agent_ctas blocks of a FUSED/ELIDE launch) run the polling agent and
  * return true; producer CTAs get false.  Call first thing in a producer kernel. */
 __device__ __forceinline__ bool agent_dispatch(const launch_ctx &lc)
 {
-    if (blockIdx.x >= lc.agent_ctas) return false;
+    if (blockIdx.x >= lc.agent_ctas) {
+        // the producer grid of this epoch has started (a separate agent's start-up deadline)
+        if (blockIdx.x == lc.agent_ctas && threadIdx.x == 0) *(volatile uint32_t *)lc.ctx->started = lc.epoch + 1u;
+        return false;
+    }
     agent_loop(lc);
     return true;
 }

@@ -25,7 +25,8 @@ MECH_NAMES = {MECH_FUSED: "fused", MECH_INLINE: "inline", MECH_BULK: "bulk",
               MECH_LOCAL: "local", MECH_ELIDE: "elide", MECH_DMA: "dma"}
 PUSH_VEC16, PUSH_BULK = 0, 1
 DISCOVER_QUEUE, DISCOVER_SCAN = 0, 1
-AGENT_FUSED, AGENT_SEPARATE = 0, 1
+AGENT_FUSED, AGENT_SEPARATE, AGENT_PRODUCER = 0, 1, 2
+LAUNCH_TILE_PUSH = 1
 SYNC_SIGNAL, SYNC_BARRIER = 0, 1
 REGION_SPARSE = 1
 
@@ -86,6 +87,9 @@ def _declare(L):
                               ctypes.POINTER(vp), sz, vp]),
         "proact_phase_sync": (i, [vp, i]),
         "proact_launch_tallies": (i, []),
+        "proact_launch_mode": (i, []),
+        "proact_launch_ex": (i, [ctypes.POINTER(ctypes.c_int), i, vp, ctypes.c_uint, ctypes.c_uint,
+                                 ctypes.POINTER(vp), sz, vp, ctypes.c_uint]),
         "proact_last_vote": (i, []),
         "proact_check": (i, []),
         "proact_host_barrier": (i, []),

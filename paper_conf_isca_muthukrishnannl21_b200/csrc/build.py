@@ -16,7 +16,7 @@ INC = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libproact.so")
 SOURCES = ["runtime.cu", "workloads.cu", "graph.cu"]
 DEPS = SOURCES
-HEADERS = ["proact.h", "proact_device.cuh", "proact_agent.cuh", "proact_workloads.h"]
+HEADERS = sorted(f for f in os.listdir(INC) if f.endswith((".h", ".cuh")))   # every public header
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC,-O2", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
@@ -43,7 +43,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
         return OUT
     objs = []
     for s in SOURCES:
-        obj = os.path.join(HERE, s.replace(".cu", ".o"))
+        obj = os.path.join(HERE, s.replace(".cu", f".{os.getpid()}.o"))   # parallel variant builds
         cmd = [NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-I", INC, "-c", os.path.join(HERE, s), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:

@@ -189,6 +189,7 @@ struct RankCtx {
     static constexpr int NDMA = 2;    // MECH_DMA: copy streams (chunks dealt round-robin)
     cudaStream_t dma[NDMA] = {nullptr, nullptr};
     cudaEvent_t ev_dma[NDMA] = {nullptr, nullptr};
+    std::vector<void (*)(void)> on_finalize;   // library state tied to this context (host solves)
 };
 
 thread_local RankCtx *tl = nullptr;
@@ -243,7 +244,7 @@ int validate_config(const proact_config &c) {
     if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
     if (c.piece_bytes < 4096 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
     if (c.discovery != PROACT_DISCOVER_QUEUE && c.discovery != PROACT_DISCOVER_SCAN) return PROACT_ERR_INVALID;
-    if (c.agent_kernel != PROACT_AGENT_FUSED && c.agent_kernel != PROACT_AGENT_SEPARATE) return PROACT_ERR_INVALID;
+    if (c.agent_kernel < PROACT_AGENT_FUSED || c.agent_kernel > PROACT_AGENT_PRODUCER) return PROACT_ERR_INVALID;
     if (c.watchdog_ms < 1) return PROACT_ERR_INVALID;
     if (c.chunk_bytes < 4096 || c.chunk_bytes % 16) return PROACT_ERR_INVALID;
     return PROACT_OK;
@@ -575,6 +576,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     c->h.vote = (uint32_t *)(c->meta + 4 * MAXR + 64);
     c->h.resident = (uint32_t *)(c->meta + 4 * MAXR + 128);
     c->h.sched = (uint32_t *)(c->meta + 4 * MAXR + 128 + 16);
+    c->h.started = (uint32_t *)(c->meta + 4 * MAXR + 128 + 32);
     c->h.err_host = c->d_err_host;
     c->h.vote_host = c->d_vote_host;
     c->h.prof = nullptr;
@@ -854,6 +856,14 @@ int proact_launch_tallies(void)
     return (m == PROACT_MECH_FUSED || m == PROACT_MECH_DMA) && c->world > 1;
 }
 
+int proact_launch_mode(void)
+{
+    RankCtx *c = need_ctx();
+    if (!c || !proact_launch_tallies()) return 0;
+    const int m = c->cfg.mech;
+    return (m == PROACT_MECH_FUSED || m == PROACT_MECH_ELIDE) && c->cfg.agent_kernel == PROACT_AGENT_PRODUCER ? 2 : 1;
+}
+
 // Producer kernels that must keep the driver's default shared-memory carve-out even next to a
 // separate agent (registered by their entry points): the graph kernels' random gathers need the
 // L1 left over as landing space -- at the maximal carve-out PageRank / SSSP phases ran 2.2x slower
@@ -872,6 +882,35 @@ extern "C" __attribute__((visibility("hidden"))) void proact_internal_keep_l1(co
     std::lock_guard<std::mutex> g(g_l1_mu);
     if (std::find(g_l1_kernels.begin(), g_l1_kernels.end(), kernel) == g_l1_kernels.end())
         g_l1_kernels.push_back(kernel);
+}
+
+// cudaFuncAttributeMaxDynamicSharedMemorySize is a per-device attribute: set it once per
+// (device, kernel), never lowering an earlier, larger opt-in.  Thread-safe (rank threads).
+namespace {
+std::mutex g_attr_mu;
+std::map<std::pair<int, const void *>, size_t> g_attr;
+}  // namespace
+extern "C" __attribute__((visibility("hidden"))) int proact_internal_smem_attr(const void *kernel, size_t bytes)
+{
+    if (bytes <= 48 * 1024) return 0;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return (int)e;
+    std::lock_guard<std::mutex> g(g_attr_mu);
+    size_t &have = g_attr[{dev, kernel}];
+    if (have >= bytes) return 0;
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e != cudaSuccess) return (int)e;
+    have = bytes;
+    return 0;
+}
+
+// Library state owned by the calling thread's rank context (e.g. the host-solve buffers of
+// workloads.cu): `fn` runs on this thread in proact_finalize, after every rank stopped using the
+// context's memory, before the context is destroyed.
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_on_finalize(void (*fn)(void))
+{
+    if (tl) tl->on_finalize.push_back(fn);
 }
 
 // Optional L2 access-policy window for the NEXT producer launch of this thread (set by a
@@ -923,6 +962,12 @@ extern "C" __attribute__((visibility("hidden"))) void proact_internal_l2_window(
 int proact_launch(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
                   void **args, size_t smem, void *stream)
 {
+    return proact_launch_ex(regions, nregions, kernel, grid, block, args, smem, stream, 0u);
+}
+
+int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsigned grid, unsigned block,
+                     void **args, size_t smem, void *stream, unsigned flags)
+{
     const void *l2b = g_l2_base;   // this launch's L2 window hint (proact_internal_l2_window)
     const size_t l2n = g_l2_bytes;
     g_l2_base = nullptr;
@@ -962,7 +1007,19 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         lc.gen_mech[r] = (armed >> r & 1) ? (uint8_t)lc.mech : R.gen_mech;
     }
     bool agent = (lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE) && armed;
-    const bool separate = agent && cfg.agent_kernel == PROACT_AGENT_SEPARATE;
+    // PROACT_AGENT_PRODUCER: the kernel's own transfer warps push its tiles (no agent CTAs);
+    // a kernel without that capability gets the separate agent instead
+    const bool tile_push = agent && cfg.agent_kernel == PROACT_AGENT_PRODUCER && (flags & PROACT_LAUNCH_TILE_PUSH);
+    if (tile_push) {
+        agent = false;
+        lc.flags |= proact::LCF_TILE_PUSH;
+    }
+    const bool separate = agent && cfg.agent_kernel != PROACT_AGENT_FUSED;
+    // PROACT_AGENT_AFTER=1 (single rank only): the separate agent runs AFTER the producer on the
+    // same stream and drains the completed chunks -- no co-residency needed, so it survives
+    // kernel serialisation (profilers); tracking-overhead runs only, nothing overlaps
+    static const bool after_env = env_int("PROACT_AGENT_AFTER", 0) != 0;
+    const bool after = separate && after_env && c->world == 1;
     // VEC16: agent_warps warps packed into CTAs; BULK (TMA): one agent warp per CTA, which
     // uses the CTA's whole dynamic shared memory as its staging ring (>= PROACT_BULK_SMEM)
     const unsigned agent_block = separate ? 256u : block;
@@ -981,7 +1038,20 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
     unsigned cap = (unsigned)std::max(1, nb * c->nsm / std::max(1, c->ranks_on_device));
     if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
     cudaStream_t s = (cudaStream_t)stream;
-    if (separate) {
+    if (after) {
+        lc.agent_ctas = 0;
+        unsigned total = grid ? grid : cap;
+        if (total > cap) total = cap;
+        *(launch_ctx *)args[0] = lc;
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
+        launch_ctx la = lc;
+        la.agent_ctas = (uint16_t)agent_ctas;
+        const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+        agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
+        CK(cudaGetLastError());
+        c->resident_total += agent_ctas;   // its CTAs count themselves resident too
+        c->launches++;
+    } else if (separate) {
         // producer kernels share SMs with the agent: same (maximal) shared-memory carveout
         if (std::find(c->carveout_set.begin(), c->carveout_set.end(), kernel) == c->carveout_set.end() &&
             !keeps_l1(kernel)) {
@@ -994,6 +1064,7 @@ int proact_launch(const int *regions, int nregions, const void *kernel, unsigned
         // producer grid leaves one slot per agent CTA; my stream waits for the agent.
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
+        la.flags |= proact::LCF_SEPARATE;
         size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
             asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
@@ -1239,6 +1310,7 @@ int proact_finalize(void)
     }
     for (void *p : c->opened) cudaIpcCloseMemHandle(p);
     int rc2 = c->shm.barrier();  // nobody uses our memory any more
+    for (auto it = c->on_finalize.rbegin(); it != c->on_finalize.rend(); ++it) (*it)();
     cudaFree(c->d);
     cudaFree(c->meta);
     cudaFreeHost(c->h_err);

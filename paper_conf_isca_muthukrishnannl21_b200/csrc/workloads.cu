@@ -21,26 +21,13 @@
 using proact::launch_ctx;
 using proact::region_dev;
 
+// runtime.cu: cudaFuncAttributeMaxDynamicSharedMemorySize for the current device, once per
+// (device, kernel) and never lowered; 0 or a cudaError_t
+extern "C" __attribute__((visibility("hidden"))) int proact_internal_smem_attr(const void *kernel, size_t bytes);
+
 namespace {
 
-// ---------------------------------------------------------------- commit helpers
-// Commit `nb` bytes at region offset `off` for each lane of warp 0 that has a span (has=true);
-// lanes whose spans fall in the same chunk are merged into one release atomic (a3).
-__device__ __forceinline__ void warp_commit(const launch_ctx &lc, int r, bool has, uint64_t off, uint32_t nb)
-{
-    if (!proact::uses_agent(lc)) return;
-    const region_dev &R = lc.ctx->region[r];
-    uint64_t rel = off - R.own_off;
-    uint32_t c = has ? (uint32_t)(rel / R.chunk_bytes) : 0xFFFFFFFFu;
-    bool single = has && (uint32_t)((rel + nb - 1) / R.chunk_bytes) == c;
-    uint32_t key = single ? c : 0xFFFFFFFFu;
-    uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
-    if (single) {
-        if ((__ffs(grp) - 1) == (int)(threadIdx.x & 31)) proact::commit_chunk(lc, r, c, nb * __popc(grp));
-    } else if (has) {
-        proact::commit_span(lc, r, off, nb);
-    }
-}
+using proact::warp_commit;
 
 __device__ __forceinline__ float4 ld_nc_f4(const float *p)
 {
@@ -84,13 +71,24 @@ __device__ __forceinline__ float ld_f(const float *p)
 #endif
 constexpr int JC = PROACT_JACOBI_JC;    // compute warps
 constexpr int JV = PROACT_JACOBI_JV;    // float4 column groups per compute thread (JC * JV = 8)
-// Two instantiations: TALLY = false (no remote destinations this launch: LOCAL / INLINE / BULK /
-// G = 1) has 8 compute + 1 TMA warp and the register budget of 4 CTAs/SM; TALLY = true adds a
-// committer warp that publishes the tile tallies so the compute warps never wait on a release.
-template <bool TALLY> struct JCfg {
-    static constexpr int threads = (JC + 1 + (TALLY ? 1 : 0)) * 32;
-    static constexpr int minb = TALLY ? 3 : 4;
-};
+// Three instantiations (proact_launch_mode): MODE 0 (no remote destinations this launch: LOCAL /
+// INLINE / BULK / G = 1) has 8 compute + 1 TMA warp and the register budget of 4 CTAs/SM; MODE 1
+// (tallies for a polling agent) adds a committer warp that publishes the tile tallies so the
+// compute warps never wait on a release; MODE 2 (PROACT_AGENT_PRODUCER) replaces it with a
+// transfer warp: the compute warps store each output row strip to the local replica and into a
+// shared-memory ring, and the transfer warp bulk-stores the ring's spans (JSR rows) to every
+// destination mirror, then counts the delivered bytes (proact::tile_pusher).
+#ifndef PROACT_JACOBI_RING_TP
+#define PROACT_JACOBI_RING_TP 10
+#endif
+#ifndef PROACT_JACOBI_OUT_RING
+#define PROACT_JACOBI_OUT_RING 2
+#endif
+#ifndef PROACT_JACOBI_SPAN_ROWS
+#define PROACT_JACOBI_SPAN_ROWS 4
+#endif
+constexpr uint32_t JOS = PROACT_JACOBI_OUT_RING;   // MODE 2: output slots of JSR row strips (4 KiB each)
+constexpr int JSR = PROACT_JACOBI_SPAN_ROWS;       // rows per pushed span
 constexpr int JW = JC * 32 * 4 * JV;    // strip width in columns = 4 KiB of a row
 #ifndef PROACT_JACOBI_OUT_EVICT_LAST   // G > 1: output rows evict-last until the agent has read them
 #define PROACT_JACOBI_OUT_EVICT_LAST 0
@@ -98,10 +96,16 @@ constexpr int JW = JC * 32 * 4 * JV;    // strip width in columns = 4 KiB of a r
 #ifndef PROACT_JACOBI_RING
 #define PROACT_JACOBI_RING 16
 #endif
-constexpr int JS = PROACT_JACOBI_RING;  // ring depth (rows in flight per CTA)
 constexpr int SLOT = JW + 8;            // floats per slot: columns [c0-4, c0+JW+4)
 constexpr int JTD = 32;                 // tile-id ring (stream warp -> compute -> committer)
-constexpr size_t JSMEM = (size_t)JS * SLOT * 4 + (size_t)2 * JS * 8 + 4 * 8 + JTD * 4;
+template <int MODE> struct JCfg {
+    static constexpr int threads = (JC + 1 + (MODE ? 1 : 0)) * 32;
+    static constexpr int minb = MODE ? 3 : 4;
+    static constexpr int js = MODE == 2 ? PROACT_JACOBI_RING_TP : PROACT_JACOBI_RING;   // input ring depth
+    static constexpr size_t ctl = (size_t)js * SLOT * 4 + (size_t)2 * js * 8 + 4 * 8 + JTD * 4;
+    static constexpr size_t out = (ctl + 127) / 128 * 128;   // MODE 2: output ring, then its control
+    static constexpr size_t smem = MODE == 2 ? out + (size_t)JOS * JSR * JW * 4 + sizeof(proact::tile_ring_ctl<JOS>) : ctl;
+};
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt)
@@ -159,6 +163,7 @@ __device__ __forceinline__ JTile jtile(int t, int nstrips, int nbands, int rb, i
 // (proact::claim_tile); the claimed id goes to tids[k % JTD] before the tile's first row is
 // armed, so the mbarrier arrival (release) publishes it to the compute warps.  After the last
 // tile an end marker (-1, a tx-less arrival on the next slot) lets them exit.
+template <int JS>
 __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_jacobi_params &p, float *ring,
                                            uint64_t *full, uint64_t *empty, int *tids, int ntiles,
                                            int nstrips, int nbands)
@@ -193,10 +198,12 @@ __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_ja
     }
 }
 
-template <bool TALLY>
-__global__ void __launch_bounds__(JCfg<TALLY>::threads, JCfg<TALLY>::minb)
+template <int MODE>
+__global__ void __launch_bounds__(JCfg<MODE>::threads, JCfg<MODE>::minb)
 jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
 {
+    constexpr bool TALLY = MODE == 1;
+    constexpr int JS = JCfg<MODE>::js;
     if (proact::agent_dispatch(lc)) return;
 #ifdef PROACT_TIMING_EXP
     unsigned long long *xprof = lc.ctx->prof;
@@ -221,12 +228,14 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     uint64_t *tdone = empty + JS;    // [2] compute warps finished tile k (k & 1)
     uint64_t *cdone = tdone + 2;     // [2] committer finished tile k (k & 1)
     int *tids = reinterpret_cast<int *>(cdone + 2);   // [JTD] claimed tile ids, by sequence
+    float *oring = reinterpret_cast<float *>(jsm + JCfg<MODE>::out);   // MODE 2: JOS x JSR row strips
+    auto *tp = reinterpret_cast<proact::tile_ring_ctl<JOS> *>(jsm + JCfg<MODE>::out + (size_t)JOS * JSR * JW * 4);
 #ifndef PROACT_JACOBI_RT_TALLY
 #define PROACT_JACOBI_RT_TALLY 1
 #endif
     // (the runtime test in the TALLY=false instantiation keeps its compute loop's code identical
     //  to the measured-fastest build; with tallies off at compile time it was ~15% slower)
-    const bool tally = (TALLY || PROACT_JACOBI_RT_TALLY) && proact::uses_agent(lc);
+    const bool tally = MODE != 2 && (TALLY || PROACT_JACOBI_RT_TALLY) && proact::uses_agent(lc);
     const int N = (int)p.N, row0 = (int)p.row0, rend = (int)(p.row0 + p.nrows);
     const int rb = p.rows_per_tile;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -243,10 +252,16 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             mbar_init(&cdone[s], 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        if (MODE == 2) proact::tp_init(tp, JC);
     }
     __syncthreads();
     if (warp == JC) {
-        if (lane == 0) jacobi_stream(lc, p, ring, full, empty, tids, ntiles, nstrips, nbands);
+        if (lane == 0) jacobi_stream<JS>(lc, p, ring, full, empty, tids, ntiles, nstrips, nbands);
+        return;
+    }
+    if (MODE == 2 && warp == JC + 1) {   // the transfer warp (PROACT_AGENT_PRODUCER)
+        proact::tile_pusher<JOS>(lc, p.region_out, reinterpret_cast<const unsigned char *>(oring), JSR * JW * 4, tp,
+                                 JW * 4, (uint64_t)N * 4, true);
         return;
     }
     if (TALLY && warp == JC + 1) {
@@ -273,12 +288,18 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     if (PROACT_JACOBI_OUT_EVICT_LAST) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_out));
     uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
     uint32_t kt = 0;   // tiles handed to the committer
+    uint32_t oq = 0;   // MODE 2: next output span of this CTA
     for (;;) {
         // the next tile's first stream item carries its id (or the end marker)
         mbar_wait(&full[q % JS], (q / JS) & 1u);
         const int t = tids[kt % JTD];
         if (t < 0) {
             if (tally && TALLY && lane == 0) mbar_arrive(&tdone[kt & 1u]);   // release the committer
+            if (MODE == 2) {   // end marker for the transfer warp
+                proact::tp_acquire(tp, oq);
+                if (tid == 0) tp->desc[oq % JOS] = proact::tile_desc{0, 0, proact::TD_END};
+                proact::tp_publish(tp, oq);
+            }
             break;
         }
         const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
@@ -310,12 +331,15 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
         // interior tiles (no Dirichlet row or column, full strip, plain stores) run a copy of the
         // row loop with those checks compiled out
         const bool fast = T.i0 > 0 && T.i1 < N && T.c0 > 0 && T.c0 + JW < N &&
-                          lc.mech != PROACT_MECH_INLINE && !(PROACT_JACOBI_OUT_EVICT_LAST && tally);
+                          (MODE == 2 || (lc.mech != PROACT_MECH_INLINE && !(PROACT_JACOBI_OUT_EVICT_LAST && tally)));
         auto rows = [&](auto fast_tag) {
             constexpr bool FAST = decltype(fast_tag)::value;
             for (int i = T.i0; i < T.i1; ++i) {
                 const uint32_t qdn = q;
                 const bool has_dn = i + 1 <= T.klast;
+                const int orow = (i - T.i0) % JSR;              // MODE 2: row within the span
+                float *ostrip = oring + ((oq % JOS) * JSR + orow) * JW;
+                if (MODE == 2 && orow == 0) proact::tp_acquire(tp, oq);
                 if (has_dn) {
                     mbar_wait(&full[q % JS], (q / JS) & 1u);
     #pragma unroll
@@ -345,7 +369,10 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                         if (!FAST && j + 3 == N - 1) o.w = c.w;
                     }
                     const uint64_t off = ((uint64_t)i * N + j) * 4;
-                    if (!FAST && lc.mech == PROACT_MECH_INLINE) {
+                    if (MODE == 2) {   // the local copy now, the span for the transfer warp
+                        *reinterpret_cast<float4 *>(ostrip + 4 * tid + g * GW) = o;
+                        *reinterpret_cast<float4 *>(outb + off) = o;
+                    } else if (!FAST && lc.mech == PROACT_MECH_INLINE) {
                         proact::put(lc, p.region_out, off, o);
                     } else if (!FAST && PROACT_JACOBI_OUT_EVICT_LAST && tally) {
                         // the agent pushes this chunk within microseconds: keep it in L2 for that read
@@ -355,6 +382,13 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                         *reinterpret_cast<float4 *>(outb + off) = o;
                     }
                 }
+                }
+                if (MODE == 2 && (orow == JSR - 1 || i + 1 == T.i1)) {   // hand the span to the transfer warp
+                    if (tid == 0)
+                        tp->desc[oq % JOS] = proact::tile_desc{((uint64_t)(i - orow) * N + T.c0) * 4,
+                                                               (uint32_t)(T.c1 - T.c0) * 4, proact::td_rows(orow + 1)};
+                    proact::tp_publish(tp, oq);
+                    ++oq;
                 }
                 __syncwarp();
                 if (lane == 0) {
@@ -373,6 +407,10 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             rows(std::true_type{});
         else
             rows(std::false_type{});
+        if (MODE == 2) {
+            ++kt;
+            continue;
+        }
         if (tally && TALLY) {   // hand the tile to the committer warp; never run > 2 tiles ahead
             __syncwarp();
             if (lane == 0) mbar_arrive(&tdone[kt & 1u]);
@@ -452,6 +490,65 @@ __global__ void __launch_bounds__(MB, 4) micro_kernel(launch_ctx lc, proact_micr
             proact::commit_span(lc, p.region, a * 4, (b - a) * 4);
         }
     }
+}
+
+// PROACT_AGENT_PRODUCER variant: 8 compute warps write each 4 KiB tile into a shared-memory ring
+// slot (same values and store-order options), the transfer warp bulk-stores it to the local
+// replica and every destination mirror and counts it once delivered (proact::tile_pusher); one
+// flush (system fence + counter commits) per MBLK tiles = 32 KiB, as the commits above.
+constexpr uint32_t MOS = 8;   // output ring slots (4 KiB each)
+constexpr size_t MTP_SMEM = (size_t)MOS * 4096 + sizeof(proact::tile_ring_ctl<MOS>);
+
+__global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, proact_micro_params p)
+{
+    if (proact::agent_dispatch(lc)) return;
+    extern __shared__ __align__(128) unsigned char msm[];
+    uint32_t *oring = reinterpret_cast<uint32_t *>(msm);
+    auto *tp = reinterpret_cast<proact::tile_ring_ctl<MOS> *>(msm + (size_t)MOS * 4096);
+    if (threadIdx.x == 0) proact::tp_init(tp, MB / 32);
+    __syncthreads();
+    if (threadIdx.x >= MB) {
+        proact::tile_pusher<MOS>(lc, p.region, msm, 4096, tp);
+        return;
+    }
+    const region_dev &R = lc.ctx->region[p.region];
+    const uint64_t w_lo = R.own_off / 4, w_hi = (R.own_off + R.own_bytes) / 4;
+    const uint64_t ntiles = (w_hi - w_lo + 1023) / 1024;
+    const uint64_t nblk = (ntiles + MBLK - 1) / MBLK;
+    uint32_t q = 0;
+    for (uint64_t bk = proact::producer_block(lc); bk < nblk; bk += proact::producer_grid(lc)) {
+        const uint64_t tb0 = bk * MBLK, tb1 = min(tb0 + MBLK, ntiles);
+        for (uint64_t t = tb0; t < tb1; ++t, ++q) {
+            const uint64_t t0 = w_lo + t * 1024, t1 = min(t0 + 1024, w_hi);
+            proact::tp_acquire(tp, q);
+            uint32_t *slot = oring + (q % MOS) * 1024;
+            if (!p.scattered) {
+                const uint64_t k = t0 + 4 * threadIdx.x;
+                if (k + 4 <= t1) {
+                    uint4 v;
+                    v.x = micro_value((uint32_t)k, p.phase, p.seed, p.K);
+                    v.y = micro_value((uint32_t)k + 1, p.phase, p.seed, p.K);
+                    v.z = micro_value((uint32_t)k + 2, p.phase, p.seed, p.K);
+                    v.w = micro_value((uint32_t)k + 3, p.phase, p.seed, p.K);
+                    *reinterpret_cast<uint4 *>(slot + 4 * threadIdx.x) = v;
+                } else {
+                    for (uint64_t w = k; w < t1 && w < k + 4; ++w) slot[w - t0] = micro_value((uint32_t)w, p.phase, p.seed, p.K);
+                }
+            } else {
+                for (int s = 0; s < 4; ++s) {
+                    const uint32_t jj = threadIdx.x + MB * s;
+                    const uint64_t w = t0 + ((jj * 389u) & 1023u);
+                    if (w < t1) slot[w - t0] = micro_value((uint32_t)w, p.phase, p.seed, p.K);
+                }
+            }
+            if (threadIdx.x == 0)
+                tp->desc[q % MOS] = proact::tile_desc{t0 * 4, (uint32_t)(t1 - t0) * 4, proact::td_rows(1)};
+            proact::tp_publish(tp, q);
+        }
+    }
+    proact::tp_acquire(tp, q);
+    if (threadIdx.x == 0) tp->desc[q % MOS] = proact::tile_desc{0, 0, proact::TD_END};
+    proact::tp_publish(tp, q);
 }
 
 // ---------------------------------------------------------------- banded Jacobi (NEXT-2)
@@ -548,18 +645,20 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
-    static bool attr = false;   // > 48 KiB of dynamic shared memory needs the opt-in
-    if (!attr) {
-        if (cudaFuncSetAttribute(jacobi_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) !=
-                cudaSuccess ||
-            cudaFuncSetAttribute(jacobi_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)JSMEM) !=
-                cudaSuccess)
-            return PROACT_ERR_CUDA;
-        attr = true;
+    // > 48 KiB of dynamic shared memory needs the opt-in, per device (set once per device)
+    if (proact_internal_smem_attr((const void *)jacobi_kernel<0>, JCfg<0>::smem) ||
+        proact_internal_smem_attr((const void *)jacobi_kernel<1>, JCfg<1>::smem) ||
+        proact_internal_smem_attr((const void *)jacobi_kernel<2>, JCfg<2>::smem))
+        return PROACT_ERR_CUDA;
+    switch (proact_launch_mode()) {
+    case 2:
+        return proact_launch_ex(regs, 1, (const void *)jacobi_kernel<2>, 0, JCfg<2>::threads, args, JCfg<2>::smem,
+                                stream, PROACT_LAUNCH_TILE_PUSH);
+    case 1:
+        return proact_launch(regs, 1, (const void *)jacobi_kernel<1>, 0, JCfg<1>::threads, args, JCfg<1>::smem, stream);
+    default:
+        return proact_launch(regs, 1, (const void *)jacobi_kernel<0>, 0, JCfg<0>::threads, args, JCfg<0>::smem, stream);
     }
-    if (proact_launch_tallies())
-        return proact_launch(regs, 1, (const void *)jacobi_kernel<true>, 0, JCfg<true>::threads, args, JSMEM, stream);
-    return proact_launch(regs, 1, (const void *)jacobi_kernel<false>, 0, JCfg<false>::threads, args, JSMEM, stream);
 }
 
 int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int scattered, void *stream)
@@ -575,6 +674,9 @@ int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int sca
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region};
+    if (proact_launch_mode() == 2)
+        return proact_launch_ex(regs, 1, (const void *)micro_tp_kernel, 0, MB + 32, args, MTP_SMEM, stream,
+                                PROACT_LAUNCH_TILE_PUSH);
     return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
 }
 
@@ -775,26 +877,20 @@ extern "C" int proact_banded_phase(int region_in, int region_out, const float *a
     }();
     if (!tma_off && N % 4 == 0 && w <= BW_MAX && (uintptr_t)a % 16 == 0 && (uintptr_t)b % 16 == 0) {
         const size_t tsmem = banded_smem(w);
-        static size_t tattr = 48 * 1024;
-        if (tsmem > tattr) {
-            if (cudaFuncSetAttribute(banded_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tsmem) !=
-                cudaSuccess)
-                return PROACT_ERR_CUDA;
-            tattr = tsmem;
-        }
+        if (proact_internal_smem_attr((const void *)banded_tma_kernel, tsmem)) return PROACT_ERR_CUDA;
         return proact_launch(regs, 1, (const void *)banded_tma_kernel, 0, (BCW + 1) * 32, args, tsmem, stream);
     }
     const size_t smem = (size_t)(BT + 2 * w) * 4;
-    static size_t attr = 48 * 1024;
-    if (smem > attr) {
-        if (cudaFuncSetAttribute(banded_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return PROACT_ERR_CUDA;
-        attr = smem;
-    }
+    if (proact_internal_smem_attr((const void *)banded_kernel, smem)) return PROACT_ERR_CUDA;
     return proact_launch(regs, 1, (const void *)banded_kernel, 0, BB, args, smem, stream);
 }
 
 // ================================================================ host-buffer Jacobi (e2e)
+// The host-solve entry points keep library-owned device buffers (registered regions) between
+// calls.  They belong to the calling thread's rank context: proact_finalize runs the hook below,
+// which frees them, so a later proact_init on the same thread starts clean (regions cannot be
+// unregistered individually, so the state must never outlive the context that registered it).
+extern "C" __attribute__((visibility("hidden"))) void proact_internal_on_finalize(void (*fn)(void));
 namespace {
 struct JacobiHost {
     long long N = 0;
@@ -803,6 +899,22 @@ struct JacobiHost {
     int ra = -1, rb = -1;
 };
 thread_local JacobiHost jh;
+
+void jh_release()
+{
+    cudaFree(jh.a);
+    cudaFree(jh.b);
+    jh = JacobiHost();
+}
+
+// rows of the input a rank reads before any peer pushes into its replica: its own rows and the
+// two halo rows (iteration 0 reads generation 0, identical on every rank, reading R16); every
+// other row of the replica is overwritten by the peers' pushes before it is read
+inline void input_rows(long long N, long long r0, long long r1, long long *lo, long long *hi)
+{
+    *lo = r0 > 0 ? r0 - 1 : 0;
+    *hi = r1 < N ? r1 + 1 : N;
+}
 }  // namespace
 
 extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long long N, int iters,
@@ -826,6 +938,7 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
         if (jh.rb < 0) return jh.rb;
         jh.N = N;
         jh.chunk = chunk_bytes;
+        proact_internal_on_finalize(jh_release);
     } else if (jh.chunk != chunk_bytes) {
         int rc = proact_region_rechunk(jh.ra, chunk_bytes);
         if (rc) return rc;
@@ -833,7 +946,10 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
         if (rc) return rc;
         jh.chunk = chunk_bytes;
     }
-    if (cudaMemcpyAsync(jh.a, h_x0, rowb * N, cudaMemcpyHostToDevice, s) != cudaSuccess) return PROACT_ERR_CUDA;
+    long long lo, hi;
+    input_rows(N, r0, r1, &lo, &hi);
+    if (cudaMemcpyAsync(jh.a + lo * N, h_x0 + lo * N, (hi - lo) * rowb, cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return PROACT_ERR_CUDA;
     for (int k = 0; k < iters; ++k) {
         const int in = (k & 1) ? jh.rb : jh.ra, out = (k & 1) ? jh.ra : jh.rb;
         int rc = proact_jacobi_phase(in, out, N, rows_per_tile, stream);
@@ -844,7 +960,7 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
     const float *res = (iters & 1) ? jh.b : jh.a;
     if (cudaMemcpyAsync(h_out + r0 * N, res + r0 * N, (r1 - r0) * rowb, cudaMemcpyDeviceToHost, s) != cudaSuccess)
         return PROACT_ERR_CUDA;
-    if (bytes_h2d) *bytes_h2d = (unsigned long long)(rowb * N);
+    if (bytes_h2d) *bytes_h2d = (unsigned long long)((hi - lo) * rowb);
     if (bytes_d2h) *bytes_d2h = (unsigned long long)((r1 - r0) * rowb);
     return PROACT_OK;
 }
@@ -865,6 +981,21 @@ struct JacobiPipe {
     cudaEvent_t ev_staged = nullptr, ev_stage_free = nullptr;
 };
 thread_local JacobiPipe jp;
+
+void jp_release()
+{
+    for (auto &b : jp.buf)
+        for (float *f : b) cudaFree(f);
+    cudaFree(jp.stage);
+    if (jp.h2d) cudaStreamDestroy(jp.h2d);
+    if (jp.d2h) cudaStreamDestroy(jp.d2h);
+    for (int b = 0; b < 2; ++b)
+        for (cudaEvent_t e : {jp.ev_in[b], jp.ev_done[b], jp.ev_out[b]})
+            if (e) cudaEventDestroy(e);
+    if (jp.ev_staged) cudaEventDestroy(jp.ev_staged);
+    if (jp.ev_stage_free) cudaEventDestroy(jp.ev_stage_free);
+    jp = JacobiPipe();
+}
 }  // namespace
 
 extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *const *h_outs, int nsolve,
@@ -879,9 +1010,14 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
         if (!h_outs[k]) return PROACT_ERR_INVALID;
     const long long r0 = N * g / G, r1 = N * (g + 1) / G;
     const size_t rowb = (size_t)N * 4;
+    long long lo, hi;
+    input_rows(N, r0, r1, &lo, &hi);
+    const size_t in_bytes = (size_t)(hi - lo) * rowb;
     cudaStream_t s = (cudaStream_t)stream;
     if (jp.N && jp.N != N) return PROACT_ERR_STATE;   // regions cannot be unregistered
     if (!jp.N) {
+        jp.N = N;   // from here on the finalize hook owns whatever was allocated
+        proact_internal_on_finalize(jp_release);
         const uint64_t all = G >= 64 ? ~0ull : ((1ull << G) - 1);
         for (int b = 0; b < 2; ++b)
             for (int h = 0; h < 2; ++h) {
@@ -902,7 +1038,6 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
         if (cudaEventCreateWithFlags(&jp.ev_staged, cudaEventDisableTiming) != cudaSuccess ||
             cudaEventCreateWithFlags(&jp.ev_stage_free, cudaEventDisableTiming) != cudaSuccess)
             return PROACT_ERR_CUDA;
-        jp.N = N;
         jp.chunk = chunk_bytes;
     } else if (jp.chunk != chunk_bytes) {
         for (int b = 0; b < 2; ++b)
@@ -918,25 +1053,26 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
         return PROACT_ERR_CUDA;
     // H2D of solve k lands in the staging buffer (it waits only for the previous solve's device
     // copy out of it), so it never queues behind the D2H of solve k - 2 that reads set k & 1:
-    // H2D and D2H run at the same time on the full-duplex link, both under the phases
-    auto h2d = [&](int k) -> int {
-        (void)k;
+    // H2D and D2H run at the same time on the full-duplex link, both under the phases.  Only the
+    // rows this rank reads before the peers' first pushes travel (input_rows).
+    auto h2d = [&]() -> int {
         if (cudaStreamWaitEvent(jp.h2d, jp.ev_stage_free, 0) != cudaSuccess) return PROACT_ERR_CUDA;
-        if (cudaMemcpyAsync(jp.stage, h_x0, rowb * N, cudaMemcpyHostToDevice, jp.h2d) != cudaSuccess)
+        if (cudaMemcpyAsync(jp.stage + lo * N, h_x0 + lo * N, in_bytes, cudaMemcpyHostToDevice, jp.h2d) != cudaSuccess)
             return PROACT_ERR_CUDA;
         return cudaEventRecord(jp.ev_staged, jp.h2d) == cudaSuccess ? PROACT_OK : PROACT_ERR_CUDA;
     };
-    int rc = h2d(0);
+    int rc = h2d();
     if (rc) return rc;
     for (int k = 0; k < nsolve; ++k) {
         const int b = k & 1;
         // set b is free once solve k - 2's D2H read it; the input moves in by a device copy
         if (cudaStreamWaitEvent(s, jp.ev_staged, 0) != cudaSuccess ||
             cudaStreamWaitEvent(s, jp.ev_out[b], 0) != cudaSuccess ||
-            cudaMemcpyAsync(jp.buf[b][0], jp.stage, rowb * N, cudaMemcpyDeviceToDevice, s) != cudaSuccess ||
+            cudaMemcpyAsync(jp.buf[b][0] + lo * N, jp.stage + lo * N, in_bytes, cudaMemcpyDeviceToDevice, s) !=
+                cudaSuccess ||
             cudaEventRecord(jp.ev_stage_free, s) != cudaSuccess)
             return PROACT_ERR_CUDA;
-        if (k + 1 < nsolve && (rc = h2d(k + 1))) return rc;   // overlaps this solve's phases
+        if (k + 1 < nsolve && (rc = h2d())) return rc;   // overlaps this solve's phases
         for (int it = 0; it < iters; ++it) {
             const int in = jp.rid[b][it & 1], out = jp.rid[b][(it & 1) ^ 1];
             if ((rc = proact_jacobi_phase(in, out, N, rows_per_tile, stream))) return rc;
@@ -956,7 +1092,7 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
     // completion on `stream`: the last D2H
     for (int b = 0; b < 2; ++b)
         if (cudaStreamWaitEvent(s, jp.ev_out[b], 0) != cudaSuccess) return PROACT_ERR_CUDA;
-    if (bytes_h2d) *bytes_h2d = (unsigned long long)(rowb * N);
+    if (bytes_h2d) *bytes_h2d = (unsigned long long)in_bytes;
     if (bytes_d2h) *bytes_d2h = (unsigned long long)((r1 - r0) * rowb);
     return PROACT_OK;
 }
@@ -969,8 +1105,8 @@ extern "C" {
 __attribute__((visibility("hidden"))) int proact_internal_preload_workloads(void)
 {
     cudaFuncAttributes a;
-    const void *k[] = {(const void *)jacobi_kernel<true>, (const void *)jacobi_kernel<false>,
-                       (const void *)micro_kernel, (const void *)banded_kernel,
+    const void *k[] = {(const void *)jacobi_kernel<0>, (const void *)jacobi_kernel<1>, (const void *)jacobi_kernel<2>,
+                       (const void *)micro_kernel, (const void *)micro_tp_kernel, (const void *)banded_kernel,
                        (const void *)banded_tma_kernel};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;

@@ -266,6 +266,9 @@ class PageRank(_Graph):
         """My r' (nv floats), copied on `stream` after its phases; the current torch stream is made
         to wait for that copy, so the tensor can be used (e.g. .cpu()) on it directly."""
         out = torch.empty(self.v1 - self.v0, dtype=torch.float32, device="cuda")
+        if stream is not None and stream != torch.cuda.current_stream():
+            # `out` may reuse a block whose earlier users are still queued on the current stream
+            stream.wait_stream(torch.cuda.current_stream())
         check(rt.lib().proact_pagerank_ranks(self.gid, ctypes.c_void_p(out.data_ptr()), _s(stream)),
               "pagerank_ranks")
         if stream is not None and stream != torch.cuda.current_stream():

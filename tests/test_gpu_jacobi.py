@@ -60,13 +60,37 @@ def test_jacobi_ragged_ranks_chunks_tiles(G, N, chunk, rpt):
 
 
 @pytest.mark.parametrize("cfg", [dict(push=1), dict(agent_kernel=1), dict(push=1, agent_kernel=1),
-                                 dict(discovery=1, agent_warps=5)])
+                                 dict(discovery=1, agent_warps=5), dict(agent_kernel=2)])
 def test_config1_jacobi_agent_variants(cfg):
     N, iters = 1024, 10
     want = oracle.jacobi(synth.jacobi_init(N), iters)
     outs = run_ranks(2, _run_jacobi, N, iters, 64 * 1024, _lib.MECH_FUSED, **cfg)
     for g, (rep, _, _) in enumerate(outs):
         assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), (g, cfg)
+
+
+@pytest.mark.parametrize("G,N,chunk,rpt", [(2, 2048, 4096, 16), (3, 1000, 12288, 16),
+                                           (4, 520, 4096, 7), (2, 4100, 1 << 20, 32), (3, 2056, 4112, 5)])
+def test_jacobi_tile_push_ragged(G, N, chunk, rpt):
+    """PROACT_AGENT_PRODUCER (the producer CTA's transfer warp bulk-stores its row strips to every
+    replica): ragged ranks, partial strips (N not a multiple of 1024), chunks that split a strip."""
+    iters = 6
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(G, _run_jacobi, N, iters, chunk, _lib.MECH_FUSED, rpt=rpt, agent_kernel=_lib.AGENT_PRODUCER)
+    for g, (rep, _, _) in enumerate(outs):
+        assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), f"rank {g}"
+
+
+def test_jacobi_tile_push_halo_only_and_elide():
+    """Tile push with per-chunk destinations (halo-only) and under ELIDE at G = 1."""
+    G, N, iters = 4, 512, 9
+    want = oracle.jacobi(synth.jacobi_init(N), iters)
+    outs = run_ranks(G, _run_jacobi, N, iters, 8192, _lib.MECH_FUSED, halo_only=True, agent_kernel=2)
+    for g, (rep, (r0, r1), _) in enumerate(outs):
+        lo, hi = max(r0 - 1, 0), min(r1 + 1, N)
+        assert np.array_equal(rep[lo:hi].view(np.uint32), want[lo:hi].view(np.uint32)), g
+    (rep, _, _), = run_ranks(1, _run_jacobi, 1536, 5, 65536, _lib.MECH_ELIDE, agent_kernel=2)
+    assert np.array_equal(rep.view(np.uint32), oracle.jacobi(synth.jacobi_init(1536), 5).view(np.uint32))
 
 
 def test_jacobi_mixed_mechanisms_across_phases():
@@ -99,11 +123,12 @@ def test_jacobi_halo_only_owned_rows_and_halos():
         assert np.array_equal(rep[lo:hi].view(np.uint32), want[lo:hi].view(np.uint32)), g
 
 
-def test_jacobi_exactly_once_delivery():
+@pytest.mark.parametrize("akern", [0, 2])
+def test_jacobi_exactly_once_delivery(akern):
     os.environ["PROACT_DEBUG"] = "1"
     try:
         G, N, iters = 3, 768, 4
-        outs = run_ranks(G, _run_jacobi, N, iters, 4096, _lib.MECH_FUSED, check_deliv=True)
+        outs = run_ranks(G, _run_jacobi, N, iters, 4096, _lib.MECH_FUSED, check_deliv=True, agent_kernel=akern)
     finally:
         del os.environ["PROACT_DEBUG"]
     for g, (_, _, deliv) in enumerate(outs):
@@ -165,7 +190,7 @@ def test_jacobi_e2e_host_buffers():
     outs = run_ranks(2, body)
     for rows, (r0, r1), h2d, d2h in outs:
         assert np.array_equal(rows, want[r0:r1])
-        assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
+        assert h2d == (min(r1 + 1, N) - max(r0 - 1, 0)) * N * 4 and d2h == (r1 - r0) * N * 4
 
 
 @pytest.mark.parametrize("G,iters", [(1, 7), (2, 6), (2, 0), (3, 5)])
@@ -192,7 +217,7 @@ def test_jacobi_e2e_pipelined_host_buffers(G, iters):
         for rows_list, (r0, r1), h2d, d2h in per_rank:
             for rows in rows_list:
                 assert np.array_equal(rows.view(np.uint32), want[r0:r1].view(np.uint32))
-            assert h2d == N * N * 4 and d2h == (r1 - r0) * N * 4
+            assert h2d == (min(r1 + 1, N) - max(r0 - 1, 0)) * N * 4 and d2h == (r1 - r0) * N * 4
 
 
 @pytest.mark.parametrize("G,N,chunk", [(1, 4, 4096), (2, 8, 4096), (2, 1024, 4112), (3, 36, 4096)])

@@ -57,7 +57,7 @@ def test_micro_replicas_equal_closed_form(G, words, chunk, mech, scattered, piec
             assert np.array_equal(outs[g][p], want), (p, g)
 
 
-@pytest.mark.parametrize("push,akern", [(0, 0), (1, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("push,akern", [(0, 0), (1, 0), (0, 1), (1, 1), (1, 2)])
 @pytest.mark.parametrize("G,words,chunk", [(2, (1 << 21) + 4 * 5, 1 << 20), (3, 1 << 20, 16384)])
 def test_micro_push_modes_and_agent_kernels(G, words, chunk, push, akern):
     """TMA bulk pushes and the separate agent kernel give the same bytes as the SIMT/fused path."""
@@ -70,12 +70,28 @@ def test_micro_push_modes_and_agent_kernels(G, words, chunk, push, akern):
             assert np.array_equal(outs[g][p], want), (p, g)
 
 
-@pytest.mark.parametrize("disc", [_lib.DISCOVER_QUEUE, _lib.DISCOVER_SCAN])
-def test_micro_exactly_once_and_counters(disc):
+@pytest.mark.parametrize("G,words,chunk,scattered", [
+    (2, 1 << 20, 4096, False), (2, (1 << 20) + 4 * 37, 65536, True), (4, 3_000_000, 1 << 20, False),
+    (3, 777_776, 12288, True), (1, 1 << 20, 4096, False)])
+def test_micro_tile_push_replicas(G, words, chunk, scattered):
+    """PROACT_AGENT_PRODUCER: the producer CTAs' transfer warps bulk-store their own 4 KiB tiles
+    to every replica; replicas equal the closed form; ragged slices and chunks that are not a
+    multiple of the tile size (spans split at chunk boundaries)."""
+    phases, K = 3, 3
+    outs = run_ranks(G, _run_micro, words, chunk, _lib.MECH_FUSED, phases, K, scattered, akern=_lib.AGENT_PRODUCER)
+    for p in range(phases):
+        want = oracle.micro_phase(words, p, SEED, K)
+        for g in range(G):
+            assert np.array_equal(outs[g][p], want), (p, g)
+
+
+@pytest.mark.parametrize("disc,akern", [(_lib.DISCOVER_QUEUE, 0), (_lib.DISCOVER_SCAN, 0),
+                                        (_lib.DISCOVER_QUEUE, 2)])
+def test_micro_exactly_once_and_counters(disc, akern):
     os.environ["PROACT_DEBUG"] = "1"
 
     def body(r, G):
-        rt.set_config(mech=_lib.MECH_FUSED, piece_bytes=8192, agent_warps=3, discovery=disc)
+        rt.set_config(mech=_lib.MECH_FUSED, piece_bytes=8192, agent_warps=3, discovery=disc, agent_kernel=akern)
         M = wl.Micro(1 << 20, 65536)
         s = torch.cuda.Stream()
         out = []

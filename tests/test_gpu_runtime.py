@@ -84,7 +84,7 @@ def test_bench_two_processes_json_line():
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "strong"
     # e2e through both host-buffer entry points (sequential and pipelined), two processes
     assert d["e2e"]["value"] > 0 and d["e2e"]["sequential_value"] > 0
-    assert d["e2e"]["h2d_bytes_per_step"] == 1024 * 1024 * 4
+    assert d["e2e"]["h2d_bytes_per_step"] == 513 * 1024 * 4   # rank 0: its rows + one halo row
     # the same ranks time the bulk-copy and naive-P2P baselines (NCCL needs distinct GPUs)
     assert set(d["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
     assert all(v > 0 for v in d["baselines_iters_per_s"].values())

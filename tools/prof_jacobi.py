@@ -15,7 +15,7 @@ phases = int(os.environ.get("PHASES", 6))
 mech = {v: k for k, v in _lib.MECH_NAMES.items()}[os.environ.get("MECH", "fused")]
 torch.cuda.set_device(0)
 rt.init(1, 0, rt.new_job_key())
-rt.set_config(mech=mech)
+rt.set_config(mech=mech, agent_kernel=int(os.environ.get("AKERN", 1)))
 J = wl.Jacobi(N, int(os.environ.get("CHUNK", 128 * 1024)), x0=torch.from_numpy(synth.jacobi_init(N)).cuda(),
               rows_per_tile=int(os.environ.get("RPT", 16)))
 s = torch.cuda.Stream()

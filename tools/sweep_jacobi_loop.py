@@ -29,11 +29,12 @@ warps = [int(x) for x in os.environ.get("WARPS", "16").split(",")]
 pushes = [int(x) for x in os.environ.get("PUSHES", "1").split(",")]
 akerns = [int(x) for x in os.environ.get("AKERNS", "0,1").split(",")]
 PH = int(os.environ.get("PHASES", 10))
+RPT = int(os.environ.get("RPT", 32))   # rows per tile (bench.py default)
 x0 = synth.jacobi_init(N)
 
 
 def body(r, G_):
-    J = wl.Jacobi(N, chunks[0], x0=torch.from_numpy(x0).cuda(), halo_only=HALO)
+    J = wl.Jacobi(N, chunks[0], x0=torch.from_numpy(x0).cuda(), halo_only=HALO, rows_per_tile=RPT)
     s = torch.cuda.Stream()
     out = []
     for ch in chunks:
@@ -44,6 +45,8 @@ def body(r, G_):
                 J.set_halo_only()
         for mech, w, pu, ak in itertools.product(mechs, warps, pushes, akerns):
             if mech not in ("fused", "elide") and (w != warps[0] or pu != pushes[0] or ak != akerns[0]):
+                continue
+            if mech == "nccl":
                 continue
             rt.set_config(mech={v: k for k, v in _lib.MECH_NAMES.items()}[mech], agent_warps=w, push=pu,
                           agent_kernel=ak)
@@ -58,7 +61,7 @@ def body(r, G_):
             b.record(s)
             s.synchronize()
             rt.host_barrier()
-            out.append({"chunk": ch, "mech": mech, "warps": w, "push": pu, "akern": ak,
+            out.append({"chunk": ch, "mech": mech, "warps": w, "push": pu, "akern": ak, "rpt": RPT,
                         "ms": a.elapsed_time(b) / PH})
     rt.check_device()
     return out
