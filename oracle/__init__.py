@@ -58,9 +58,11 @@ def lib():
         L.oracle_jacobi.restype = i32
         L.oracle_jacobi.argtypes = [vp, i64, i32]
         L.oracle_pagerank.restype = i32
-        L.oracle_pagerank.argtypes = [i64, i64, vp, vp, i32, ctypes.c_double, vp]
+        L.oracle_pagerank.argtypes = [i64, i64, vp, vp, i32, ctypes.c_double, vp,
+                                      ctypes.POINTER(ctypes.c_double)]
         L.oracle_sssp.restype = i32
-        L.oracle_sssp.argtypes = [i64, i64, vp, vp, vp, i64, i32, vp, ctypes.POINTER(i32), vp]
+        L.oracle_sssp.argtypes = [i64, i64, vp, vp, vp, i64, i32, vp, ctypes.POINTER(i32), vp,
+                                  ctypes.POINTER(ctypes.c_double)]
         L.oracle_banded_jacobi.restype = i32
         L.oracle_banded_jacobi.argtypes = [vp, vp, vp, i64, i64, i32]
         L.oracle_proto_run.restype = i32
@@ -129,19 +131,24 @@ def banded_jacobi(a: np.ndarray, b: np.ndarray, x0: np.ndarray, iters: int) -> n
 
 # ---------------------------------------------------------------- PageRank (L265)
 def pagerank(V: int, src: np.ndarray, dst: np.ndarray, iters: int,
-             d: float = DAMPING) -> np.ndarray:
+             d: float = DAMPING, timing: dict | None = None) -> np.ndarray:
+    """r^{iters}; timing (optional dict) receives "iter_seconds": the iterations alone."""
     src = np.ascontiguousarray(src, dtype=np.uint32)
     dst = np.ascontiguousarray(dst, dtype=np.uint32)
     r = np.empty(V, dtype=np.float32)
-    if lib().oracle_pagerank(V, src.size, _p(src), _p(dst), iters, d, _p(r)) != 0:
+    t = ctypes.c_double(0.0)
+    if lib().oracle_pagerank(V, src.size, _p(src), _p(dst), iters, d, _p(r), ctypes.byref(t)) != 0:
         raise MemoryError("oracle_pagerank")
+    if timing is not None:
+        timing["iter_seconds"] = t.value
     return r
 
 
 # ---------------------------------------------------------------- SSSP (L267)
 def sssp(V: int, src: np.ndarray, dst: np.ndarray, w: np.ndarray, s: int,
-         max_rounds: int = 0) -> tuple[np.ndarray, int, np.ndarray]:
-    """Synchronous Bellman-Ford; returns (d, rounds, changed_per_round)."""
+         max_rounds: int = 0, timing: dict | None = None) -> tuple[np.ndarray, int, np.ndarray]:
+    """Synchronous Bellman-Ford; returns (d, rounds, changed_per_round); timing (optional dict)
+    receives "iter_seconds": the rounds alone (the CSC build is input preparation)."""
     src = np.ascontiguousarray(src, dtype=np.uint32)
     dst = np.ascontiguousarray(dst, dtype=np.uint32)
     w = np.ascontiguousarray(w, dtype=np.int32)
@@ -149,9 +156,12 @@ def sssp(V: int, src: np.ndarray, dst: np.ndarray, w: np.ndarray, s: int,
     cap = max_rounds if max_rounds > 0 else max(V, 1)
     changed = np.zeros(cap + 1, dtype=np.int64)
     rounds = ctypes.c_int(0)
+    t = ctypes.c_double(0.0)
     if lib().oracle_sssp(V, src.size, _p(src), _p(dst), _p(w), s, max_rounds, _p(d),
-                         ctypes.byref(rounds), _p(changed)) != 0:
+                         ctypes.byref(rounds), _p(changed), ctypes.byref(t)) != 0:
         raise MemoryError("oracle_sssp")
+    if timing is not None:
+        timing["iter_seconds"] = t.value
     return d, rounds.value, changed[:rounds.value]
 
 

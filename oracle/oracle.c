@@ -28,6 +28,14 @@
 #include <pthread.h>
 #include <sched.h>
 #include <omp.h>
+#include <time.h>
+
+static double now_s(void)
+{
+    struct timespec t;
+    clock_gettime(CLOCK_MONOTONIC, &t);
+    return (double)t.tv_sec + 1e-9 * (double)t.tv_nsec;
+}
 
 /* OpenMP thread count (results never depend on it: every parallel loop writes disjoint cells). */
 void oracle_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
@@ -109,7 +117,7 @@ int oracle_jacobi(float *x, int64_t N, int iters)
  * result rounded to fp32 once per iteration (r is fp32 between iterations). */
 
 int oracle_pagerank(int64_t V, int64_t E, const uint32_t *src, const uint32_t *dst,
-                    int iters, double d, float *r_out)
+                    int iters, double d, float *r_out, double *iter_seconds)
 {
     int64_t *outdeg = (int64_t *)calloc((size_t)V + 1, sizeof(int64_t));
     int64_t *colptr = (int64_t *)calloc((size_t)V + 1, sizeof(int64_t));
@@ -129,6 +137,7 @@ int oracle_pagerank(int64_t V, int64_t E, const uint32_t *src, const uint32_t *d
     }
     for (int64_t v = 0; v < V; ++v) r[v] = (float)(1.0 / (double)V);
     const double base = (1.0 - d) / (double)V;
+    const double t0 = now_s();   /* iterations only (the CSC build above is input preparation) */
     for (int k = 0; k < iters; ++k) {
 #pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t v = 0; v < V; ++v) {
@@ -141,6 +150,7 @@ int oracle_pagerank(int64_t V, int64_t E, const uint32_t *src, const uint32_t *d
         }
         float *t = r; r = rn; rn = t;
     }
+    if (iter_seconds) *iter_seconds = now_s() - t0;
     memcpy(r_out, r, sizeof(float) * (size_t)V);
     free(outdeg); free(colptr); free(rowidx); free(r); free(rn);
     return 0;
@@ -152,38 +162,63 @@ int oracle_pagerank(int64_t V, int64_t E, const uint32_t *src, const uint32_t *d
  * distances, INF = INT32_MAX, synchronous rounds d^{k+1}[v] = min(d^k[v],
  * min_{u->v, d^k[u] != INF} d^k[u] + w(u->v)); stop after the first round that changes nothing
  * (that round is counted) or after V rounds.  Also records, per round, how many vertices
- * changed (used by the roofline accounting). */
+ * changed (used by the roofline accounting).  Written as the paper says it -- every vertex
+ * computes its own distance -- i.e. a pull over each vertex's in-edges (CSC, edges stably sorted
+ * by destination), one vertex per loop iteration, OpenMP over vertices: a min over a fixed set
+ * is order independent, so the result does not depend on the thread count. */
 
 int oracle_sssp(int64_t V, int64_t E, const uint32_t *src, const uint32_t *dst,
                 const int32_t *w, int64_t s, int max_rounds, int32_t *d_out,
-                int *rounds_out, int64_t *changed_per_round)
+                int *rounds_out, int64_t *changed_per_round, double *iter_seconds)
 {
     int32_t *dk = (int32_t *)malloc(sizeof(int32_t) * (size_t)(V ? V : 1));
     int32_t *dn = (int32_t *)malloc(sizeof(int32_t) * (size_t)(V ? V : 1));
-    if (!dk || !dn) return -1;
+    int64_t *colptr = (int64_t *)calloc((size_t)V + 1, sizeof(int64_t));
+    uint32_t *rowidx = (uint32_t *)malloc(sizeof(uint32_t) * (size_t)(E ? E : 1));
+    int32_t *wt = (int32_t *)malloc(sizeof(int32_t) * (size_t)(E ? E : 1));
+    if (!dk || !dn || !colptr || !rowidx || !wt) return -1;
+    /* CSC: stable counting sort of the edges by destination (input preparation) */
+    for (int64_t e = 0; e < E; ++e) colptr[dst[e] + 1]++;
+    for (int64_t v = 0; v < V; ++v) colptr[v + 1] += colptr[v];
+    {
+        int64_t *cur = (int64_t *)malloc(sizeof(int64_t) * (size_t)(V ? V : 1));
+        if (!cur) return -1;
+        memcpy(cur, colptr, sizeof(int64_t) * (size_t)V);
+        for (int64_t e = 0; e < E; ++e) {
+            const int64_t q = cur[dst[e]]++;
+            rowidx[q] = src[e];
+            wt[q] = w[e];
+        }
+        free(cur);
+    }
     for (int64_t v = 0; v < V; ++v) dk[v] = INT32_MAX;
     if (V > 0) dk[s] = 0;
     if (max_rounds <= 0 || max_rounds > V) max_rounds = (int)(V > 0 ? V : 1);
     int rounds = 0;
+    const double t0 = now_s();
     for (int k = 0; k < max_rounds; ++k) {
-        memcpy(dn, dk, sizeof(int32_t) * (size_t)V);
-        /* plain edge loop; min is order independent, so it is serial and exact */
-        for (int64_t e = 0; e < E; ++e) {
-            int32_t du = dk[src[e]];
-            if (du == INT32_MAX) continue;
-            int64_t cand = (int64_t)du + (int64_t)w[e];
-            if (cand < dn[dst[e]]) dn[dst[e]] = (int32_t)cand;
-        }
         int64_t changed = 0;
-        for (int64_t v = 0; v < V; ++v) changed += (dn[v] != dk[v]);
+#pragma omp parallel for schedule(dynamic, 4096) reduction(+ : changed)
+        for (int64_t v = 0; v < V; ++v) {
+            int32_t best = dk[v];
+            for (int64_t p = colptr[v]; p < colptr[v + 1]; ++p) {
+                const int32_t du = dk[rowidx[p]];
+                if (du == INT32_MAX) continue;
+                const int64_t cand = (int64_t)du + (int64_t)wt[p];
+                if (cand < best) best = (int32_t)cand;
+            }
+            dn[v] = best;
+            changed += best != dk[v];
+        }
         if (changed_per_round) changed_per_round[k] = changed;
         int32_t *t = dk; dk = dn; dn = t;
         rounds = k + 1;
         if (changed == 0) break;
     }
+    if (iter_seconds) *iter_seconds = now_s() - t0;
     memcpy(d_out, dk, sizeof(int32_t) * (size_t)V);
     *rounds_out = rounds;
-    free(dk); free(dn);
+    free(dk); free(dn); free(colptr); free(rowidx); free(wt);
     return 0;
 }
 

@@ -151,3 +151,20 @@ def test_rmat_generator_shape():
 def test_splitmix64_reference_output():
     # first output of splitmix64 seeded with 0 (Vigna's reference implementation)
     assert synth.splitmix64(0) == 0xE220A8397B1DCDAF
+
+
+def test_sssp_oracle_independent_of_thread_count():
+    """The OpenMP pull (one vertex per iteration, a min over its in-edges) gives the same d and
+    round count on 1 thread as on all of them (min over a fixed set is order independent)."""
+    src, dst = synth.rmat(10, 8)
+    V = 1 << 10
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    n = oracle.get_threads()
+    try:
+        oracle.set_threads(1)
+        d1, r1, c1 = oracle.sssp(V, src, dst, w, s0)
+    finally:
+        oracle.set_threads(n)
+    dn, rn, cn = oracle.sssp(V, src, dst, w, s0)
+    assert r1 == rn and np.array_equal(d1, dn) and np.array_equal(c1, cn)
