@@ -116,30 +116,68 @@ def test_sssp_disconnected_and_tiny():
         assert np.all(d[V // 2:] == oracle.INF)
 
 
+_RMAT24 = {}
+
+
+def _rmat24():
+    """RMAT-24 edge list + weights + source, generated once per test session."""
+    if not _RMAT24:
+        src, dst = synth.rmat(24, 16)
+        V = 1 << 24
+        _RMAT24.update(src=src, dst=dst, V=V, w=synth.weights(src.size),
+                       s0=int(np.bincount(src, minlength=V).argmax()))
+    return _RMAT24
+
+
+def _pr_body_cfg(r, G, V, src, dst, iters, chunk, cfg):
+    rt.set_config(**cfg)
+    return _pr_body(r, G, V, src, dst, iters, chunk, _lib.MECH_FUSED)
+
+
+def _sssp_body_cfg(r, G, V, src, dst, w, s0, chunk, cfg):
+    rt.set_config(**cfg)
+    return _sssp_body(r, G, V, src, dst, w, s0, chunk, _lib.MECH_FUSED)
+
+
+# the graph benchmarks' launch configuration (tools/bench_workloads.py): FUSED with the separate
+# agent, TMA pushes, queue discovery, 128 KiB chunks (RMAT-24: 256 chunks per rank at G = 2)
+_GCFG = [(128 * 1024, dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_BULK, discovery=_lib.DISCOVER_QUEUE)),
+         (1 << 20, dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_VEC16, discovery=_lib.DISCOVER_SCAN))]
+
+
 @pytest.mark.slow
-def test_config3_pagerank_full_size():
-    """BASELINE.json config 3 at full size (RMAT-24, ef16, 20 iterations), every vertex."""
-    src, dst = synth.rmat(24, 16)
-    V, iters = 1 << 24, 20
-    outs = run_ranks(1, _pr_body, V, src, dst, iters, 128 * 1024, _lib.MECH_FUSED)
-    want = oracle.pagerank(V, src, dst, iters).astype(np.float64)
-    (_, _, got), = outs
-    rel = np.abs(got.astype(np.float64) - want) / want
+@pytest.mark.parametrize("G", [1, 2])
+def test_config3_pagerank_full_size(G):
+    """BASELINE.json config 3 at full size (RMAT-24, ef16, 20 iterations), every vertex.  G = 1
+    runs the producer kernel alone (nothing to replicate, reading R18); G = 2 loopback runs the
+    whole protocol in the benchmarks' launch configuration."""
+    g = _rmat24()
+    V, iters = g["V"], 20
+    chunk, cfg = _GCFG[0]
+    outs = run_ranks(G, _pr_body_cfg, V, g["src"], g["dst"], iters, chunk, cfg)
+    want = oracle.pagerank(V, g["src"], g["dst"], iters).astype(np.float64)
+    got = np.zeros(V)
+    for v0, v1, r in outs:
+        got[v0:v1] = r
+    rel = np.abs(got - want) / want
     assert rel.max() <= 1e-5, rel.max()
 
 
 @pytest.mark.slow
-def test_config4_sssp_full_size():
-    """BASELINE.json config 4 at full size (RMAT-24, int32, to convergence), bit-exact."""
-    src, dst = synth.rmat(24, 16)
-    V = 1 << 24
-    w = synth.weights(src.size)
-    s0 = int(np.bincount(src, minlength=V).argmax())
-    outs = run_ranks(1, _sssp_body, V, src, dst, w, s0, 128 * 1024, _lib.MECH_FUSED)
-    want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
-    (rounds, d, _, _), = outs
-    assert rounds == want_rounds
-    assert np.array_equal(d, want)
+@pytest.mark.parametrize("G,k", [(1, 0), (2, 0), (2, 1)])
+def test_config4_sssp_full_size(G, k):
+    """BASELINE.json config 4 at full size (RMAT-24, int32, to convergence), bit-exact, every
+    vertex of every rank's full replica and the round count.  At G = 2 each rank owns >= 32
+    chunks of 1 MiB / 256 of 128 KiB, so the SPARSE push-iff-changed-now-or-last-round logic
+    (reading R13) runs on many chunks per rank and round."""
+    g = _rmat24()
+    chunk, cfg = _GCFG[k]
+    outs = run_ranks(G, _sssp_body_cfg, g["V"], g["src"], g["dst"], g["w"], g["s0"], chunk, cfg)
+    want, want_rounds, _ = oracle.sssp(g["V"], g["src"], g["dst"], g["w"], g["s0"])
+    for rounds, d, v0, v1 in outs:
+        assert (v1 - v0) * 4 // chunk >= 32 or G == 1
+        assert rounds == want_rounds
+        assert np.array_equal(d, want)
 
 
 def test_graph_without_edges():

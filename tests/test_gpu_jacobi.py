@@ -157,9 +157,10 @@ def _window_oracle(N, iters, i, j):
 
 
 @pytest.mark.slow
-def test_config2_full_size_sampled():
-    """Config 2 size (16384^2, 100 iterations) in bench.py's launch configuration (G=1, FUSED),
-    checked on sampled cells computed one by one by the oracle."""
+def test_config2_full_size_sampled_single_gpu():
+    """Config 2 size (16384^2, 100 iterations) in bench.py's N = 1 launch configuration.  At
+    G = 1 there is nothing to replicate, so FUSED runs the uninstrumented kernel (reading R18):
+    this checks the producer kernel alone, on sampled cells computed one by one by the oracle."""
     N, iters = 16384, 100
     (rep, _, _), = run_ranks(1, _run_jacobi, N, iters, 128 * 1024, _lib.MECH_FUSED, rpt=32)
     rng = np.random.default_rng(0)
@@ -171,6 +172,86 @@ def test_config2_full_size_sampled():
     # boundary rows/cols are copied through (Dirichlet)
     x0 = synth.jacobi_init(N, row0=0, nrows=1)
     assert np.array_equal(rep[0], x0[0])
+
+
+def _block_oracle(N, iters, i0, i1, j0, j1):
+    """x^iters on rows [i0, i1) x cols [j0, j1), exactly: from a square window of x0 reaching
+    iters + 1 cells beyond the block on every side that is not the grid's own boundary
+    (influence travels one cell per iteration, so a false window edge never reaches the block)."""
+    h = iters + 1
+    S = min(N, max(i1 - i0, j1 - j0) + 2 * h)
+    a = min(max(i0 - h, 0), N - S)
+    b = min(max(j0 - h, 0), N - S)
+    x0 = np.ascontiguousarray(synth.jacobi_init(N, row0=a, nrows=S)[:, b:b + S])
+    return oracle.jacobi(x0, iters)[i0 - a:i1 - a, j0 - b:j1 - b]
+
+
+def _run_jacobi_full(r, G, N, iters, chunk, cfg):
+    """bench.py's N > 1 step on G loopback ranks; returns (my replica, rows, other ranks' rows
+    of my replica are compared across ranks by the caller)."""
+    rep, rows, _ = _run_jacobi(r, G, N, iters, chunk, _lib.MECH_FUSED, rpt=32, **cfg)
+    return rep, rows
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("chunk,cfg", [
+    (128 * 1024, dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_BULK, discovery=_lib.DISCOVER_QUEUE)),
+    (1 << 20, dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_BULK, discovery=_lib.DISCOVER_QUEUE)),
+    (1 << 20, dict(agent_kernel=_lib.AGENT_PRODUCER)),
+    (128 * 1024, dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_VEC16, discovery=_lib.DISCOVER_SCAN)),
+])
+def test_config2_full_size_two_ranks(chunk, cfg):
+    """Config 2 at full size (16384^2, 100 iterations) on G = 2 loopback ranks in the launch
+    configuration bench.py times at N > 1 (FUSED: tallies, agent, pushes, flags, credits every
+    phase).  Checked: every cell of the four rows around the rank boundary (the halo rows each
+    rank waits on every phase) against exact block oracles, sampled cells elsewhere, and the two
+    replicas equal bit for bit (every pushed byte arrived: replica bytes == producer bytes)."""
+    N, iters, G = 16384, 100, 2
+    outs = run_ranks(G, _run_jacobi_full, N, iters, chunk, cfg)
+    (rep0, (r0a, r1a)), (rep1, (r0b, r1b)) = outs
+    assert r1a == r0b == N // 2
+    assert np.array_equal(rep0.view(np.uint32), rep1.view(np.uint32))
+    b = N // 2
+    for j0 in range(0, N, 1024):   # rows b-2 .. b+1, all columns, in 1024-column blocks
+        want = _block_oracle(N, iters, b - 2, b + 2, j0, j0 + 1024)
+        assert np.array_equal(rep0[b - 2:b + 2, j0:j0 + 1024].view(np.uint32), want.view(np.uint32)), j0
+    rng = np.random.default_rng(1)
+    for i, j in rng.integers(iters + 1, N - iters - 2, size=(8, 2)):
+        assert rep0[i, j] == _window_oracle(N, iters, int(i), int(j)), (i, j)
+
+
+@pytest.mark.slow
+def test_config2_full_size_two_ranks_halo_only():
+    """The halo-only variant (reading R8; per-chunk destinations = neighbours) at full size, in
+    bench.py's halo leg configuration: the rows each rank reads are exact."""
+    N, iters, G = 16384, 100, 2
+    outs = run_ranks(G, _run_jacobi, N, iters, 1 << 20, _lib.MECH_FUSED, halo_only=True, rpt=32,
+                     agent_kernel=_lib.AGENT_PRODUCER)
+    b = N // 2
+    for g, (rep, (r0, r1), _) in enumerate(outs):
+        for j0 in range(0, N, 4096):
+            want = _block_oracle(N, iters, b - 1, b + 1, j0, j0 + 4096)
+            assert np.array_equal(rep[b - 1:b + 1, j0:j0 + 4096].view(np.uint32), want.view(np.uint32)), (g, j0)
+
+
+def test_jacobi_allgather_baseline():
+    """Jacobi.step_allgather (the north star's NCCL all-gather baseline: uninstrumented kernel +
+    all_gather_into_tensor between phases) equals the oracle; NCCL needs one GPU per rank."""
+    if torch.cuda.device_count() < 2:
+        pytest.skip("NCCL all-gather needs 2 GPUs (one rank per GPU)")
+    import socket
+    import subprocess
+    import sys
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "allgather_rank.py")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), script]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert r.stdout.count("ALLGATHER_OK") == 2, r.stdout
 
 
 def test_jacobi_e2e_host_buffers():
