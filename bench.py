@@ -183,6 +183,38 @@ def cpu_baseline(N: int, budget_s: float = 12.0) -> dict:
             "sample": f"{k} Jacobi iterations of the full {N}x{N} fp32 grid (oracle.jacobi_step)"}
 
 
+def single_gpu_reference(N: int, I: int, rpt: int, steps: int = 2) -> float:
+    """Milliseconds for `steps` uninstrumented single-GPU solves (G = 1, LOCAL: the plain
+    producer kernel) of the full grid on this rank's GPU: the strong-scaling denominator,
+    measured in the same run, before the N-rank context exists (its own one-rank context)."""
+    import torch
+    import synth
+    from paper_conf_isca_muthukrishnannl21_b200 import _lib
+    from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+    from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+    rt.init(1, 0, rt.new_job_key())
+    rt.set_config(mech=_lib.MECH_LOCAL)
+    J = wl.Jacobi(N, 1 << 20, x0=torch.from_numpy(synth.jacobi_init(N)).cuda(), rows_per_tile=rpt)
+    s = torch.cuda.Stream()
+    for k in range(I):
+        J.step(s, barrier=(k == I - 1))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.synchronize()
+    a.record(s)
+    for _ in range(steps):
+        for k in range(I):
+            J.step(s, barrier=(k == I - 1))
+    b.record(s)
+    s.synchronize()
+    ms = a.elapsed_time(b)
+    rt.check_device()
+    del J
+    torch.cuda.synchronize()
+    rt.finalize()
+    torch.cuda.empty_cache()
+    return ms
+
+
 def run_reference(args, dist_rank: int) -> None:
     if dist_rank != 0:
         return
@@ -234,6 +266,8 @@ def main():
                          "with the producer, which a kernel-serialising profiler prevents)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for the timing barrier / max-over-ranks only")
+    ap.add_argument("--no-halo", action="store_true", help="N > 1: skip the halo-only legs")
+    ap.add_argument("--no-n1", action="store_true", help="N > 1: skip the single-GPU reference (speedup)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -268,6 +302,10 @@ def main():
         job = f"bench_{os.environ.get('MASTER_ADDR', '')}_{os.environ.get('MASTER_PORT', '')}"
     else:
         job = rt.new_job_key()
+    # strong-scaling denominator: the uninstrumented single-GPU solve, on every rank's GPU at once
+    n1_ms = None
+    if world > 1 and not args.no_n1:
+        n1_ms = max_over_ranks(single_gpu_reference(args.n, args.iters, args.rpt), world)
     rt.init(world, rank, job)
     # --mech nccl: the north star's bulk baseline -- uninstrumented kernels (LOCAL) with an NCCL
     # all-gather of the rows between them (workloads.Jacobi.step_allgather)
@@ -310,15 +348,17 @@ def main():
                 ts.append(a.elapsed_time(b))
             return statistics.median(ts)
 
-        best = rt.autotune(f"bench_jacobi_N{N}_G{world}", run_point,
-                           "mech=0;chunk=131072,1048576;warps=8,16,32;push=1;akern=1")
+        space = "mech=0;chunk=131072,1048576;warps=8,16,32;push=0,1;akern=0,1,2"
+        best = rt.autotune(f"bench_jacobi_N{N}_G{world}", run_point, space)
         if best["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
             for rid in J.rid:
                 rt.rechunk(rid, best["chunk_bytes"])
         cfg = rt.set_config(mech=best["mech"], agent_warps=best["agent_warps"], push=best["push"],
                             agent_kernel=best["agent_kernel"], chunk_bytes=best["chunk_bytes"])
         chunk = best["chunk_bytes"]
-        tuned = "proact_autotune: chunk {128K, 1M} x agent warps {8, 16, 32}"
+        tuned = {"space": space, "best": {k: best[k] for k in ("chunk_bytes", "agent_warps", "push", "agent_kernel")},
+                 "note": "proact_autotune (a9): chunk x agent warps x push (VEC16 / TMA) x agent placement "
+                         "(fused CTAs / separate kernel / producer-CTA transfer warps); max over ranks"}
 
     live_ev: list = []   # (start, end) CUDA event pairs around jacobi_kernel inside the timed region
 
@@ -461,6 +501,47 @@ def main():
         mode["nccl"] = nccl_base
         rt.set_config(mech=mech)
 
+    # ---- halo-only variant (reading R8: the one config-2 variant whose roofline allows
+    # >= 6x at G = 8): per-chunk destinations = the neighbours; PROACT (tuned) and the baselines
+    halo = None
+    if world > 1 and not args.no_halo:
+        J.set_halo_only()
+        kk = max(2, args.steps // 2)
+        legs = [("proact", mech), ("bulk_cudaMemcpyPeer", _lib.MECH_BULK), ("naive_p2p_inline", _lib.MECH_INLINE)]
+        hv = {}
+        for name, m in legs:
+            rt.set_config(mech=m)
+            mode["nccl"] = False
+            step()
+            hv[name] = kk * I / (timed(step, kk) / 1000.0)
+        mode["nccl"] = nccl_base
+        rt.set_config(mech=mech)
+        h_rows = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
+        h_ingress = 4.0 * N * max(1, h_rows) if world > 1 else 0.0
+        ht = 1000.0 / hv["proact"] * 1000.0   # us per phase
+        h_nvl = h_ingress / (NVL * 1e9) * 1e6
+        halo = {"value": hv["proact"], "unit": "iters/s", "baselines_iters_per_s": {k: v for k, v in hv.items() if k != "proact"},
+                "speedup_vs_n1": None,
+                "step_roofline": {"t_hbm_us": t_hbm_us, "t_nvl_us": h_nvl, "t_phase_us": ht,
+                                  "frac": max(t_hbm_us, h_nvl) / ht,
+                                  "nvlink_ingress_GBps_per_gpu": h_ingress / (ht * 1e-6) / 1e9},
+                "note": "per-chunk destinations = neighbours (boundary rows only); rows other ranks own "
+                        "are not replicated"}
+
+    n1_value = (2 * I / (n1_ms / 1000.0)) if n1_ms else (value if world == 1 else None)
+    if halo is not None and n1_value:
+        halo["speedup_vs_n1"] = halo["value"] / n1_value
+    # transfer-agent cost: SMs dedicated to the agent x phase time per GB pushed
+    egress_gb = 4.0 * N * nrows * (world - 1) / 1e9
+    akern = cfg.get("agent_kernel", 1)
+    agent_sms = 0 if akern == _lib.AGENT_PRODUCER else min(cfg["agent_warps"], 148 // 2)
+    agent_cost = None
+    if world > 1 and egress_gb > 0 and mech in (_lib.MECH_FUSED, _lib.MECH_ELIDE):
+        agent_cost = {"agent_placement": {0: "fused CTAs", 1: "separate kernel", 2: "producer-CTA transfer warps"}[akern],
+                      "dedicated_sms": agent_sms,
+                      "agent_sm_ms_per_GB_pushed": agent_sms * (t_phase_us / 1000.0) / egress_gb,
+                      "egress_GB_per_phase": egress_gb}
+
     # ---- e2e through the C-ABI host-buffer entry point
     e2e = None
     if not args.no_e2e:
@@ -499,7 +580,11 @@ def main():
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
                 "dtype": "f32", "data": "synthetic",
                 "config": {"workload": WORKLOAD, "N": N, "iters_per_step": I, "ranks": world,
-                           "mech": args.mech, "chunk_bytes": chunk,
+                           "mech": args.mech,
+                           "mech_effective": ("local (G = 1: nothing to replicate, so FUSED runs the "
+                                              "uninstrumented kernel, reading R18)"
+                                              if world == 1 and args.mech == "fused" else args.mech),
+                           "chunk_bytes": chunk,
                            "agent_warps": cfg["agent_warps"], "piece_bytes": cfg["piece_bytes"],
                            "rows_per_tile": args.rpt, "replication": "full", "tuned": tuned,
                            "l2": "inputs > L2 (two 1 GiB grids), no flush",
@@ -507,7 +592,13 @@ def main():
                            "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)]},
                 "roofline": roofline, "step_roofline": step_roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "clocks": clk.summary(), "gpu_launches": launches, "overhead": overhead,
-                "baselines_iters_per_s": baselines}
+                "baselines_iters_per_s": baselines,
+                "speedup_vs_n1": (value / n1_value) if n1_value else None,
+                "n1_reference": {"value": n1_value, "unit": "iters/s",
+                                 "what": ("this run's timed step (G = 1)" if world == 1 else
+                                          "uninstrumented single-GPU solve (LOCAL) of the full grid on every "
+                                          "rank's GPU in this run, slowest rank")},
+                "halo_only": halo, "agent_cost": agent_cost}
         print(json.dumps(line), flush=True)
     torch.cuda.synchronize()
     rt.finalize()

@@ -477,6 +477,35 @@ __global__ void sync_kernel(const dev_ctx *C, uint32_t epoch, int mode)
     }
 }
 
+// Rank metadata block layout: done[MAXR] | err | vote[2] | resident, sched[2], started | probes
+constexpr size_t META_PROBE = 256;   // [MAXR] x 32 B: pre-flight stores from each peer
+
+__device__ __host__ inline uint32_t probe_token(int rank) { return 0x9E3779B9u * (uint32_t)(rank + 1) ^ 0x50524F41u; }
+
+// Pre-flight (proact_init): one 16-byte vector store (st.global.v4, the VEC16 push path) and one
+// 16-byte TMA bulk store (cp.async.bulk smem -> peer global, the BULK / producer push path) into
+// every mapped peer's rank block, then a system-scope fence.  The host then checks that its own
+// block received both from every peer: an unusable mapping becomes PROACT_ERR_NOPEER at init
+// instead of a hang or a wrong replica on the first phase.
+__global__ void preflight_kernel(const dev_ctx *C)
+{
+    __shared__ __align__(16) uint32_t buf[4];
+    const uint32_t tok = probe_token(C->rank);
+    if (threadIdx.x < 4) buf[threadIdx.x] = tok ^ (threadIdx.x + 1);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    const int p = threadIdx.x;
+    if (p < C->world && p != C->rank) {
+        char *slot = reinterpret_cast<char *>(C->peer_done[p]) + META_PROBE + 32 * C->rank;
+        proact::st_v4(reinterpret_cast<uint4 *>(slot), make_uint4(tok, (uint32_t)C->rank, 0x50524F41u, ~tok));
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], 16;" ::"l"(slot + 16),
+                     "r"((uint32_t)__cvta_generic_to_shared(buf)) : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    }
+    proact::fence_acq_rel_sys();
+}
+
 __global__ void credit_wait_kernel(const dev_ctx *C, uint32_t epoch, uint32_t mask)
 {
     // BULK: before copying epoch-e data into peer p's replica, p must have finished phase e-1
@@ -558,7 +587,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     int coop_attr = 0;
     cudaDeviceGetAttribute(&coop_attr, cudaDevAttrCooperativeLaunch, c->device);
     // rank metadata block: done[MAXR] | err | vote[2]
-    size_t meta_bytes = 4 * MAXR + 64 + 64 + 64;
+    size_t meta_bytes = META_PROBE + 32 * MAXR;   // done | err | vote | resident, sched, started | probes
     if (cudaMalloc((void **)&c->meta, meta_bytes) != cudaSuccess) return fail(PROACT_ERR_CUDA);
     cudaMemset(c->meta, 0, meta_bytes);
     if (cudaHostAlloc((void **)&c->h_err, 64, cudaHostAllocMapped) != cudaSuccess) return fail(PROACT_ERR_CUDA);
@@ -626,7 +655,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         {
             cudaFuncAttributes fa;
             const void *k[] = {(const void *)agent_kernel, (const void *)sync_kernel,
-                               (const void *)credit_wait_kernel};
+                               (const void *)credit_wait_kernel, (const void *)preflight_kernel};
             for (const void *f : k)
                 if (cudaFuncGetAttributes(&fa, f) != cudaSuccess) return fail(PROACT_ERR_CUDA);
             if (proact_internal_preload_workloads() || proact_internal_preload_graph()) return fail(PROACT_ERR_CUDA);
@@ -637,6 +666,37 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
                                  cudaSharedmemCarveoutMaxShared) != cudaSuccess)
             return fail(PROACT_ERR_CUDA);
+    }
+    // pre-flight every peer mapping with both push instructions (PROACT_PREFLIGHT=0: skip)
+    if (ngpus > 1 && env_int("PROACT_PREFLIGHT", 1)) {
+        int bad = 0;
+        preflight_kernel<<<1, 32 * ((MAXR + 31) / 32), 0, c->side>>>(c->d);
+        cudaError_t e = cudaStreamSynchronize(c->side);
+        if (e != cudaSuccess) {
+            c->last_cuda = (int)e;
+            fprintf(stderr, "[proact] rank %d: pre-flight stores to peers failed: %s\n", rank, cudaGetErrorString(e));
+            bad = 1;
+        }
+        if ((rc = c->shm.barrier())) return fail(rc);
+        uint32_t got[MAXR][8];
+        if (!bad && cudaMemcpy(got, c->meta + META_PROBE, sizeof(got), cudaMemcpyDeviceToHost) != cudaSuccess) bad = 1;
+        for (int p = 0; p < ngpus && !bad; ++p) {
+            if (p == rank) continue;
+            const uint32_t t = probe_token(p);
+            const bool vec_ok = got[p][0] == t && got[p][1] == (uint32_t)p && got[p][2] == 0x50524F41u && got[p][3] == ~t;
+            bool tma_ok = true;
+            for (int k = 0; k < 4; ++k) tma_ok = tma_ok && got[p][4 + k] == (t ^ (uint32_t)(k + 1));
+            if (!vec_ok || !tma_ok) {
+                fprintf(stderr, "[proact] rank %d: pre-flight from rank %d: %s store did not arrive\n", rank, p,
+                        vec_ok ? "TMA bulk" : "16-byte vector");
+                bad = 1;
+            }
+        }
+        int32_t mine_bad = bad;
+        std::vector<int32_t> all_bad(ngpus);
+        if ((rc = c->shm.allgather(rank, &mine_bad, sizeof(mine_bad), all_bad.data()))) return fail(rc);
+        for (int32_t b : all_bad)
+            if (b) return fail(PROACT_ERR_NOPEER);   // every rank fails together (no one hangs)
     }
     rc = c->shm.barrier();
     if (rc) return fail(rc);
@@ -1505,9 +1565,13 @@ int proact_autotune(const char *key, const char *space, proact_run_fn fn, void *
                         for (long long di : discs)
                             for (long long ak : akerns) {
                                 bool agent = m == PROACT_MECH_FUSED || m == PROACT_MECH_ELIDE;
-                                // non-agent mechanisms ignore the agent axes: run them once
+                                // non-agent mechanisms ignore the agent axes: run them once; the
+                                // producer-CTA transfer warps ignore warps / piece / push / discovery
                                 if (!agent && (w != warps[0] || pc != pieces[0] || pu != pushes[0] ||
                                                di != discs[0] || ak != akerns[0]))
+                                    continue;
+                                if (agent && ak == PROACT_AGENT_PRODUCER &&
+                                    (w != warps[0] || pc != pieces[0] || pu != pushes[0] || di != discs[0]))
                                     continue;
                                 proact_config t = base;
                                 t.mech = (int)m;

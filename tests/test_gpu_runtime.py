@@ -88,3 +88,14 @@ def test_bench_two_processes_json_line():
     # the same ranks time the bulk-copy and naive-P2P baselines (NCCL needs distinct GPUs)
     assert set(d["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
     assert all(v > 0 for v in d["baselines_iters_per_s"].values())
+    # strong scaling against the single-GPU solve measured in the same run
+    assert d["speedup_vs_n1"] > 0 and d["n1_reference"]["value"] > 0
+    sr = d["step_roofline"]
+    assert 0 < sr["frac"] and sr["nvlink_ingress_GBps_per_gpu"] > 0 and sr["t_nvl_us"] > 0
+    # the profiler swept push engine x agent placement (incl. the producer-CTA transfer warps)
+    assert "push=0,1" in d["config"]["tuned"]["space"] and "akern=0,1,2" in d["config"]["tuned"]["space"]
+    # halo-only variant beside full replication, with its own baselines and roofline
+    h = d["halo_only"]
+    assert h["value"] > 0 and h["speedup_vs_n1"] > 0 and h["step_roofline"]["frac"] > 0
+    assert set(h["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
+    assert d["agent_cost"]["agent_sm_ms_per_GB_pushed"] >= 0
