@@ -26,7 +26,9 @@ typedef struct proact_jacobi_params {
 typedef struct proact_micro_params {
     int region;
     unsigned phase, seed;
-    int K, scattered, pad;
+    int K, scattered;
+    int verify_region;        /* litmus: region whose current generation must hold phase-1 tags, or -1 */
+    unsigned *bad;            /* litmus: device counter of stale / wrong words seen (or NULL) */
 } proact_micro_params;
 
 /* Jacobi, 2D 5-point stencil (Sec. IV-C; BASELINE.json configs 1-2; DESIGN.md
@@ -46,6 +48,25 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
  * One CTA pass per 4 KiB tile; scattered != 0 permutes the store order inside each tile
  * (position (j*389) mod 1024), which only matters for INLINE (store coalescing, L143, L318). */
 int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int scattered, void *stream);
+
+/* Protocol litmus ("no later than the succeeding global
+ * synchronization barrier", L145 visibility): a microbenchmark phase that is also a CONSUMER.
+ * Before producing, every CTA waits (proact::wait_range, i.e. the arrival flags or credits of the
+ * mechanism that produced it) for the whole current generation of region_in, then checks every
+ * word of it against its phase tag -- word k must equal the microbenchmark value of phase
+ * `phase - 1` (K = 1) -- and adds the number of words that differ (stale or torn) to *d_bad
+ * (device memory, uint32).  It then writes phase `phase` of region_out exactly like
+ * proact_micro_phase (K = 1, dense).  region_in / region_out: two registered regions of equal
+ * geometry (ping-pong).  phase 0 skips the check. */
+int proact_litmus_phase(int region_in, int region_out, unsigned phase, unsigned seed, unsigned *d_bad,
+                        void *stream);
+
+/* Fault injection (tests): one launch on `region` whose first producer CTA commits the bytes of my
+ * chunk 0 twice, as a producer with a non-deterministic store count would (PAPER.md L129:
+ * "a deterministic number of stores" is required).  Under a tallying mechanism (FUSED / ELIDE
+ * with G > 1, or DMA) the over-count is detected on the device: the next proact_phase_sync /
+ * proact_check returns PROACT_ERR_PROTOCOL (site: commit).  Other chunks are not written. */
+int proact_inject_double_commit(int region, void *stream);
 
 /* End-to-end Jacobi through host buffers (the bench's "e2e" path).  COLLECTIVE over the world.
  * h_x0: the full N x N initial grid in host memory (pinned for async copies); h_out: receives

@@ -536,6 +536,39 @@ __global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc)
 
 RankCtx *need_ctx() { return tl; }
 
+// Library streams come from a per-device pool that outlives the rank contexts.  CUDA maps streams
+// onto CUDA_DEVICE_MAX_CONNECTIONS hardware queues round-robin at creation; a queue blocked by a
+// stream memory wait (the separate agent's residency gate, the DMA mechanism) blocks every stream
+// that shares it.  Creating fresh streams at every proact_init keeps advancing that round-robin,
+// so after enough init/finalize cycles in one process (test sessions, loopback ranks) a new
+// library stream can share a queue with a long-lived stream of another rank -- observed as a rare
+// loopback deadlock (3 ranks, separate agents).  Reusing the same streams keeps the mapping fixed.
+std::mutex g_stream_mu;
+std::map<int, std::vector<cudaStream_t>> g_stream_pool;   // device -> free high-priority streams
+
+cudaError_t pool_stream(int device, cudaStream_t *out)
+{
+    {
+        std::lock_guard<std::mutex> g(g_stream_mu);
+        auto &v = g_stream_pool[device];
+        if (!v.empty()) {
+            *out = v.back();
+            v.pop_back();
+            return cudaSuccess;
+        }
+    }
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    return cudaStreamCreateWithPriority(out, cudaStreamNonBlocking, hi);
+}
+
+void pool_return(int device, cudaStream_t s)
+{
+    if (!s) return;
+    std::lock_guard<std::mutex> g(g_stream_mu);
+    g_stream_pool[device].push_back(s);
+}
+
 }  // namespace
 
 // ================================================================================== C ABI
@@ -641,11 +674,11 @@ int proact_init_ex(int ngpus, int rank, const char *job)
     {
         int lo = 0, hi = 0;
         cudaDeviceGetStreamPriorityRange(&lo, &hi);
-        if (cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        if (pool_stream(c->device, &c->side) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         if (cudaEventCreateWithFlags(&c->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         if (cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         for (int k = 0; k < RankCtx::NDMA; ++k) {
-            if (cudaStreamCreateWithPriority(&c->dma[k], cudaStreamNonBlocking, hi) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+            if (pool_stream(c->device, &c->dma[k]) != cudaSuccess) return fail(PROACT_ERR_CUDA);
             if (cudaEventCreateWithFlags(&c->ev_dma[k], cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         }
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM_MAX) !=
@@ -1374,9 +1407,9 @@ int proact_finalize(void)
     cudaFree(c->d);
     cudaFree(c->meta);
     cudaFreeHost(c->h_err);
-    if (c->side) cudaStreamDestroy(c->side);
+    pool_return(c->device, c->side);   // idle after the device synchronisation above
     for (int k = 0; k < RankCtx::NDMA; ++k) {
-        if (c->dma[k]) cudaStreamDestroy(c->dma[k]);
+        pool_return(c->device, c->dma[k]);
         if (c->ev_dma[k]) cudaEventDestroy(c->ev_dma[k]);
     }
     if (c->ev_start) cudaEventDestroy(c->ev_start);

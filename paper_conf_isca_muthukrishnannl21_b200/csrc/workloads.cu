@@ -451,9 +451,29 @@ __device__ __forceinline__ uint32_t micro_value(uint32_t k, uint32_t phase, uint
 constexpr int MB = 256;            // threads; one 4 KiB tile (1024 words) per CTA pass (L279)
 constexpr int MBLK = 8;            // tiles per CTA block: one commit per 32 KiB block
 
+// Litmus consumer prologue (proact_litmus_phase): wait for the whole current generation of the
+// verify region (flags or credits, as its producing mechanism requires), then check every word
+// against phase-1's value; this CTA checks a grid-stride share of the words.
+__device__ __forceinline__ void litmus_check(const launch_ctx &lc, const proact_micro_params &p, int nthreads)
+{
+    if (p.verify_region < 0 || p.phase == 0) return;
+    const region_dev &V = lc.ctx->region[p.verify_region];
+    if (threadIdx.x == 0) proact::wait_range(lc, p.verify_region, 0, V.total_bytes);
+    __syncthreads();
+    const uint32_t *w = reinterpret_cast<const uint32_t *>(V.base);
+    const uint64_t W = V.total_bytes / 4;
+    uint32_t bad = 0;
+    for (uint64_t k = (uint64_t)proact::producer_block(lc) * nthreads + threadIdx.x; k < W;
+         k += (uint64_t)proact::producer_grid(lc) * nthreads)
+        bad += w[k] != micro_value((uint32_t)k, p.phase - 1, p.seed, 1);
+    bad = __reduce_add_sync(0xFFFFFFFFu, bad);
+    if (bad && (threadIdx.x & 31) == 0 && p.bad) atomicAdd(p.bad, bad);
+}
+
 __global__ void __launch_bounds__(MB, 4) micro_kernel(launch_ctx lc, proact_micro_params p)
 {
     if (proact::agent_dispatch(lc)) return;
+    litmus_check(lc, p, MB);
     const region_dev &R = lc.ctx->region[p.region];
     const uint64_t w_lo = R.own_off / 4, w_hi = (R.own_off + R.own_bytes) / 4;
     const uint64_t ntiles = (w_hi - w_lo + 1023) / 1024;
@@ -511,6 +531,19 @@ __global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, pro
         proact::tile_pusher<MOS>(lc, p.region, msm, 4096, tp);
         return;
     }
+    if (p.verify_region >= 0 && p.phase > 0) {   // litmus: the producer warps check (named barrier)
+        const region_dev &V = lc.ctx->region[p.verify_region];
+        if (threadIdx.x == 0) proact::wait_range(lc, p.verify_region, 0, V.total_bytes);
+        asm volatile("bar.sync 1, %0;" ::"r"(MB) : "memory");
+        const uint32_t *w = reinterpret_cast<const uint32_t *>(V.base);
+        const uint64_t W = V.total_bytes / 4;
+        uint32_t bad = 0;
+        for (uint64_t k = (uint64_t)proact::producer_block(lc) * MB + threadIdx.x; k < W;
+             k += (uint64_t)proact::producer_grid(lc) * MB)
+            bad += w[k] != micro_value((uint32_t)k, p.phase - 1, p.seed, 1);
+        bad = __reduce_add_sync(0xFFFFFFFFu, bad);
+        if (bad && (threadIdx.x & 31) == 0 && p.bad) atomicAdd(p.bad, bad);
+    }
     const region_dev &R = lc.ctx->region[p.region];
     const uint64_t w_lo = R.own_off / 4, w_hi = (R.own_off + R.own_bytes) / 4;
     const uint64_t ntiles = (w_hi - w_lo + 1023) / 1024;
@@ -549,6 +582,20 @@ __global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, pro
     proact::tp_acquire(tp, q);
     if (threadIdx.x == 0) tp->desc[q % MOS] = proact::tile_desc{0, 0, proact::TD_END};
     proact::tp_publish(tp, q);
+}
+
+// ---------------------------------------------------------------- fault injection (tests)
+__global__ void double_commit_kernel(launch_ctx lc, int region)
+{
+    if (proact::agent_dispatch(lc)) return;
+    if (proact::producer_block(lc) == 0 && threadIdx.x == 0) {
+        const region_dev &R = lc.ctx->region[region];
+        if (R.n_own) {
+            const uint32_t b = proact::chunk_len(R, 0);
+            proact::commit_chunk(lc, region, 0, b);
+            proact::commit_chunk(lc, region, 0, b);   // the second commit over-counts chunk 0
+        }
+    }
 }
 
 // ---------------------------------------------------------------- banded Jacobi (NEXT-2)
@@ -661,6 +708,45 @@ int proact_jacobi_phase(int region_in, int region_out, long long N, int rows_per
     }
 }
 
+static int micro_launch(proact_micro_params &p, void *stream)
+{
+    launch_ctx lc;
+    void *args[2] = {&lc, &p};
+    int regs[1] = {p.region};
+    if (proact_launch_mode() == 2)
+        return proact_launch_ex(regs, 1, (const void *)micro_tp_kernel, 0, MB + 32, args, MTP_SMEM, stream,
+                                PROACT_LAUNCH_TILE_PUSH);
+    return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
+}
+
+int proact_litmus_phase(int region_in, int region_out, unsigned phase, unsigned seed, unsigned *d_bad, void *stream)
+{
+    proact_region_info ri, ro;
+    int rc = proact_region_info_get(region_in, &ri);
+    if (rc) return rc;
+    if ((rc = proact_region_info_get(region_out, &ro))) return rc;
+    if (region_in == region_out || ri.total_bytes != ro.total_bytes || ri.own_offset != ro.own_offset)
+        return PROACT_ERR_INVALID;
+    proact_micro_params p;
+    p.region = region_out;
+    p.phase = phase;
+    p.seed = seed;
+    p.K = 1;
+    p.scattered = 0;
+    p.verify_region = region_in;
+    p.bad = d_bad;
+    return micro_launch(p, stream);
+}
+
+int proact_inject_double_commit(int region, void *stream)
+{
+    launch_ctx lc;
+    int r = region;
+    void *args[2] = {&lc, &r};
+    int regs[1] = {region};
+    return proact_launch(regs, 1, (const void *)double_commit_kernel, 1, 64, args, 0, stream);
+}
+
 int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int scattered, void *stream)
 {
     if (K < 1) return PROACT_ERR_INVALID;
@@ -670,14 +756,9 @@ int proact_micro_phase(int region, unsigned phase, unsigned seed, int K, int sca
     p.seed = seed;
     p.K = K;
     p.scattered = scattered;
-    p.pad = 0;
-    launch_ctx lc;
-    void *args[2] = {&lc, &p};
-    int regs[1] = {region};
-    if (proact_launch_mode() == 2)
-        return proact_launch_ex(regs, 1, (const void *)micro_tp_kernel, 0, MB + 32, args, MTP_SMEM, stream,
-                                PROACT_LAUNCH_TILE_PUSH);
-    return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
+    p.verify_region = -1;
+    p.bad = nullptr;
+    return micro_launch(p, stream);
 }
 
 }  // extern "C"
@@ -1106,7 +1187,8 @@ __attribute__((visibility("hidden"))) int proact_internal_preload_workloads(void
 {
     cudaFuncAttributes a;
     const void *k[] = {(const void *)jacobi_kernel<0>, (const void *)jacobi_kernel<1>, (const void *)jacobi_kernel<2>,
-                       (const void *)micro_kernel, (const void *)micro_tp_kernel, (const void *)banded_kernel,
+                       (const void *)micro_kernel, (const void *)micro_tp_kernel, (const void *)double_commit_kernel,
+                       (const void *)banded_kernel,
                        (const void *)banded_tma_kernel};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;

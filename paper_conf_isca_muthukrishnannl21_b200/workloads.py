@@ -176,6 +176,18 @@ def micro_phase(rid: int, phase: int, seed: int, K: int = 1, scattered: bool = F
                                       int(scattered), _s(stream)), "micro_phase")
 
 
+def litmus_phase(r_in: int, r_out: int, phase: int, seed: int, bad: torch.Tensor, stream=None) -> None:
+    """proact_litmus_phase: check every word of r_in's current generation against phase-1's tag
+    (counting mismatches into the int32 CUDA tensor `bad`), then write phase `phase` of r_out."""
+    assert bad.is_cuda and bad.dtype == torch.int32
+    check(rt.lib().proact_litmus_phase(r_in, r_out, phase & 0xFFFFFFFF, seed & 0xFFFFFFFF,
+                                       ctypes.c_void_p(bad.data_ptr()), _s(stream)), "litmus_phase")
+
+
+def inject_double_commit(rid: int, stream=None) -> None:
+    check(rt.lib().proact_inject_double_commit(rid, _s(stream)), "inject_double_commit")
+
+
 class Micro:
     """A replicated region of `words` u32 words, all-gather shape (every rank produces W/G)."""
 

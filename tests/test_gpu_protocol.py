@@ -1,0 +1,103 @@
+"""Protocol hardening: litmus runs, fault injection.
+
+Litmus (remote data is visible "no later than the succeeding global
+synchronization barrier"; L145: the visibility the transfer must guarantee): every phase is also
+a consumer that, after its mechanism's arrival wait (flags or credits), checks every word of the
+previous generation against that phase's tag.  10^4 phases per mechanism with SIGNAL syncs (no
+barrier between phases): a consumer that ever sees a stale or torn word after a flag counts it.
+A flipped byte is detected (the checker is not blind); a double tally latches
+PROACT_ERR_PROTOCOL (over-count detection, reading R1 / L129).
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks, ProactError
+from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt
+from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl
+
+pytestmark = pytest.mark.gpu
+SEED = 0x1A7
+
+MECHS = {
+    "fused_separate_tma": dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_BULK, agent_warps=4),
+    "fused_separate_vec16_scan": dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_VEC16,
+                                      discovery=_lib.DISCOVER_SCAN, agent_warps=4),
+    "fused_in_grid": dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_FUSED, push=_lib.PUSH_VEC16, agent_warps=4),
+    "producer_tile_push": dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_PRODUCER),
+    "inline": dict(mech=_lib.MECH_INLINE),
+    "bulk": dict(mech=_lib.MECH_BULK),
+    "dma": dict(mech=_lib.MECH_DMA),
+}
+
+
+def _litmus_body(r, G, words, chunk, phases, cfg, flip_after=None):
+    rt.set_config(watchdog_ms=20000, **cfg)
+    bufs = [torch.zeros(words, dtype=torch.int32, device="cuda") for _ in range(2)]
+    bounds = [((words * p) // G) // 4 * 4 for p in range(G)] + [words]
+    lo, hi = bounds[r], bounds[r + 1]
+    torch.cuda.synchronize()
+    rid = [rt.register_region(b, lo * 4, (hi - lo) * 4, chunk) for b in bufs]
+    bad = torch.zeros(1, dtype=torch.int32, device="cuda")
+    s = torch.cuda.Stream()
+    flipped = None
+    for p in range(phases):
+        if flip_after is not None and p == flip_after:
+            # every rank is quiescent (BARRIER sync + host barrier); rank 0 flips one byte of a
+            # word rank 1 pushed into its replica, which phase p reads
+            s.synchronize()
+            rt.host_barrier()
+            if r == 0:
+                k = (bounds[1] + bounds[2]) // 2
+                bufs[p & 1][k] ^= 0x100
+                torch.cuda.synchronize()
+                flipped = k
+            rt.host_barrier()
+        wl.litmus_phase(rid[p & 1], rid[(p & 1) ^ 1], p, SEED, bad, s)
+        barrier = p == phases - 1 or (flip_after is not None and p == flip_after - 1)
+        rt.phase_sync(s, barrier=barrier)
+    s.synchronize()
+    rt.check_device()
+    return int(bad.item()), flipped
+
+
+@pytest.mark.parametrize("name", list(MECHS))
+@pytest.mark.parametrize("G", [2, 3])
+def test_litmus_no_stale_word_after_arrival(name, G):
+    phases = 10000 if G == 2 else 2000
+    words = 1 << 16                 # 256 KiB region, 16 KiB chunks: 16 chunks, ragged at G = 3
+    outs = run_ranks(G, _litmus_body, words, 16384, phases, MECHS[name], timeout=900)
+    for g, (bad, _) in enumerate(outs):
+        assert bad == 0, f"rank {g}: {bad} stale/torn words seen after the arrival wait ({name})"
+
+
+def test_litmus_detects_a_flipped_byte():
+    outs = run_ranks(2, _litmus_body, 1 << 16, 16384, 40, MECHS["fused_separate_tma"], flip_after=20)
+    (bad0, flipped), (bad1, _) = outs
+    assert flipped is not None and bad0 == 1 and bad1 == 0
+
+
+@pytest.mark.parametrize("G,cfg", [(1, dict(mech=_lib.MECH_ELIDE)),
+                                   (2, dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_SEPARATE)),
+                                   (2, dict(mech=_lib.MECH_FUSED, agent_kernel=_lib.AGENT_PRODUCER))])
+def test_double_tally_latches_protocol_error(G, cfg):
+    """A producer that commits a chunk's bytes twice (non-deterministic store count, L129) is
+    caught on the device: PROACT_ERR_PROTOCOL at the next sync, on every rank that did it."""
+
+    def body(r, G_):
+        rt.set_config(watchdog_ms=3000, **cfg)
+        M = wl.Micro(1 << 16, 4096)
+        s = torch.cuda.Stream()
+        M.step(SEED, 1, False, stream=s, barrier=True)   # one clean phase first
+        s.synchronize()
+        wl.inject_double_commit(M.rid, s)
+        try:
+            rt.phase_sync(s, barrier=False)
+            s.synchronize()
+            rt.check_device()
+        except ProactError as e:
+            return e.code
+        return 0
+
+    codes = run_ranks(G, body)
+    assert all(c == _lib.ERR_PROTOCOL for c in codes), codes
