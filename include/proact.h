@@ -254,6 +254,12 @@ int proact_last_vote(void);
  * the device.  INVALID if debug counters are off or n is too small. */
 int proact_region_debug_deliveries(int region, uint32_t *out, size_t n);
 
+/* Debug: protocol state of region `region` as this rank sees it, for post-mortems after a
+ * watchdog timeout.  Synchronises the device.  Writes n_own counters, n_own expected, n_own
+ * piece counts, n_total arrival flags, 8 queue-control words, 16 credits (done[]) and 16 host
+ * words ([0] epoch, [1] generations launched) to `out` (uint32).  INVALID if n is too small. */
+int proact_region_debug_state(int region, uint32_t *out, size_t n);
+
 /* Debug (PROACT_DEBUG=2 at init): agent cycle accounting since the last call, 8 counters:
  * [0] discovery-wait cycles, [1] batch-processing cycles, [2] batches, [3] units,
  * [4] TMA push-pipeline cycles, [5] store-drain cycles.  Synchronises the device; resets. */

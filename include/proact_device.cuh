@@ -64,7 +64,8 @@ struct region_dev {
     unsigned long long *queue;  /* [qcap] ready units (gen << 32 | unit), QUEUE discovery */
     uint32_t *qctl;             /* [8]: tail[2], head[2] by generation parity, agents_done */
     uint32_t qcap;              /* queue capacity in units */
-    uint32_t pad_q;
+    uint32_t dma_group;         /* MECH_DMA: chunks per copy-engine transfer group (>= 1) */
+    uint32_t *group_cnt;        /* MECH_DMA: [n_own / dma_group] chunks completed in the group */
     uint64_t rank_off[PROACT_MAX_RANKS + 1];
     uint32_t rank_chunk0[PROACT_MAX_RANKS + 1];
     char *peer_base[PROACT_MAX_RANKS];            /* peers' replica bases (mapped) */
@@ -333,6 +334,12 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
         raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
     } else if (old + b == ex && (lc.flags & LCF_TILE_PUSH)) {
         publish_chunk(lc, r, c);
+    } else if (old + b == ex && lc.mech == PROACT_MECH_DMA) {
+        // NEXT-3: the copy engines wait on the chunk's GROUP counter (prepared descriptors copy a
+        // whole group); the last committer resets its chunk counter (no more commits can come
+        // this generation) and counts the chunk into its group with system-scope release
+        R.counter[c] = 0u;
+        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(R.group_cnt + c / R.dma_group) : "memory");
     } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA) {
         const uint32_t piece = piece_size(lc, R);
         const uint32_t P = (R.chunk_bytes + piece - 1) / piece;

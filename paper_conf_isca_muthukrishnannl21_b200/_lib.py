@@ -104,6 +104,7 @@ def _declare(L):
         "proact_jacobi_phase": (i, [i, i, ctypes.c_longlong, i, vp]),
         "proact_micro_phase": (i, [i, ctypes.c_uint, ctypes.c_uint, i, i, vp]),
         "proact_litmus_phase": (i, [i, i, ctypes.c_uint, ctypes.c_uint, vp, vp]),
+        "proact_region_debug_state": (i, [i, vp, sz]),
         "proact_inject_double_commit": (i, [i, vp]),
         "proact_banded_phase": (i, [i, i, vp, vp, ctypes.c_longlong, ctypes.c_longlong, vp]),
         "proact_jacobi_solve_host": (i, [vp, vp, ctypes.c_longlong, i, sz, i, vp,

@@ -155,6 +155,11 @@ struct Region {
     uint32_t gen_epoch = 0;           // epoch of the latest generation
     uint8_t gen_mech = PROACT_MECH_LOCAL;   // mechanism that produced it
     int64_t last_armed_epoch = -1;
+    // MECH_DMA: the per-phase copy-engine program (wait group counter -> copy per destination ->
+    // reset), built once per geometry and replayed as a CUDA graph (NEXT-3, L166)
+    cudaGraphExec_t dma_exec = nullptr;
+    uint32_t dma_group = 1;
+    uint32_t dma_peers = 0;           // destinations the program copies to
 };
 
 struct RankCtx {
@@ -363,8 +368,8 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
     size_t off_queue = 0, off_counter = off_queue + 8 * qcap, off_expected = off_counter + 4 * n_own,
            off_piece = off_expected + 4 * n_own, off_changed = off_piece + 4 * n_own,
            off_push = off_changed + 4 * n_own, off_arrive = off_push + 4 * n_own,
-           off_count = off_arrive + 4 * n_total, off_qctl = off_count + 64, off_deliv = off_qctl + 64,
-           total = off_deliv + 4 * deliv + 64;
+           off_count = off_arrive + 4 * n_total, off_qctl = off_count + 64, off_group = off_qctl + 64,
+           off_deliv = off_group + 4 * n_own, total = off_deliv + 4 * deliv + 64;
     if (R.meta) { CK(cudaFree(R.meta)); R.meta = nullptr; }
     CK(cudaMalloc((void **)&R.meta, total));
     CK(cudaMemset(R.meta, 0, total));
@@ -397,6 +402,14 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
     D.queue = (unsigned long long *)(R.meta + off_queue);
     D.qctl = (uint32_t *)(R.meta + off_qctl);
     D.qcap = (uint32_t)qcap;
+    // copy-engine transfer groups: PROACT_DMA_GROUP_BYTES (default 16 MiB) of whole chunks
+    {
+        const uint64_t gb = (uint64_t)std::max(1, env_int("PROACT_DMA_GROUP_BYTES", 16 << 20));
+        R.dma_group = (uint32_t)std::max<uint64_t>(1, gb / R.chunk);
+        if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }
+    }
+    D.dma_group = R.dma_group;
+    D.group_cnt = (uint32_t *)(R.meta + off_group);
     D.chunk_dest = nullptr;
     R.chunk_dest.clear();
     if (R.d_chunk_dest) { CK(cudaFree(R.d_chunk_dest)); R.d_chunk_dest = nullptr; }
@@ -528,13 +541,77 @@ constexpr size_t AGENT_SMEM_SMALL = 64 * 1024 + 1024;
 constexpr size_t AGENT_SMEM_MAX = 224 * 1024 + 1024;   // PROACT_AGENT_SMEM_KB upper bound
 __global__ void __launch_bounds__(256, 1) agent_kernel(launch_ctx lc)
 {
-    // residency gate: the producer's stream waits until every agent CTA is resident, so the
-    // producer grid can never occupy the slots the agent needs (which would serialise them)
+    // residency gate: the producer is this kernel's programmatic dependent on the same stream
+    // (proact_launch); it may launch once every agent CTA has executed launch_dependents, i.e.
+    // is resident -- so the producer grid can never take the slots the agent needs
     if (threadIdx.x == 0) atomicAdd(lc.ctx->resident, 1u);
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     proact::agent_loop(lc);
 }
 
 RankCtx *need_ctx() { return tl; }
+
+// MECH_DMA program of region r (see proact_launch): captured from the DMA streams into a graph.
+// Transfer groups of R.dma_group chunks are dealt round-robin over the NDMA streams (copy engines
+// run them concurrently); inside a group, maximal runs of chunks with the same destinations are
+// copied with one cudaMemcpyAsync per destination.
+int build_dma_program(RankCtx *c, int r)
+{
+    Region &R = c->regions[r];
+    const region_dev &D = c->h.region[r];
+    R.dma_peers = 0;
+    cudaStream_t d0 = c->dma[0];
+    cudaGraph_t g = nullptr;
+    CK(cudaStreamBeginCapture(d0, cudaStreamCaptureModeThreadLocal));
+    int rc = PROACT_OK;
+    auto fail = [&](int e) {
+        cudaStreamEndCapture(d0, &g);
+        if (g) cudaGraphDestroy(g);
+        return e;
+    };
+    if (cudaEventRecord(c->ev_start, d0) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    for (int k = 1; k < RankCtx::NDMA; ++k)
+        if (cudaStreamWaitEvent(c->dma[k], c->ev_start, 0) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    const uint32_t G = R.dma_group;
+    const uint32_t ngroups = (R.n_own + G - 1) / G;
+    for (uint32_t q = 0; q < ngroups; ++q) {
+        cudaStream_t d = c->dma[q % RankCtx::NDMA];
+        const uint32_t c0 = q * G, c1 = std::min(R.n_own, c0 + G);
+        if (g_wait32((CUstream)d, (CUdeviceptr)(D.group_cnt + q), c1 - c0, CU_STREAM_WAIT_VALUE_EQ) != CUDA_SUCCESS)
+            return fail(PROACT_ERR_CUDA);
+        for (uint32_t k = c0; k < c1;) {
+            const uint32_t m = (R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k]) & ~(1u << c->rank);
+            uint32_t k1 = k + 1;
+            while (k1 < c1 && ((R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k1]) & ~(1u << c->rank)) == m)
+                ++k1;
+            const uint64_t lo = R.own_off + (uint64_t)k * R.chunk;
+            const uint64_t hi = std::min<uint64_t>(R.own_off + (uint64_t)k1 * R.chunk, R.own_off + R.own_bytes);
+            for (int p = 0; p < c->world; ++p)
+                if (m >> p & 1) {
+                    R.dma_peers |= 1u << p;
+                    if (cudaMemcpyAsync(D.peer_base[p] + lo, R.base + lo, hi - lo, cudaMemcpyDeviceToDevice, d) !=
+                        cudaSuccess)
+                        return fail(PROACT_ERR_CUDA);
+                }
+            k = k1;
+        }
+        if (g_write32((CUstream)d, (CUdeviceptr)(D.group_cnt + q), 0, 0) != CUDA_SUCCESS) return fail(PROACT_ERR_CUDA);
+    }
+    for (int k = 1; k < RankCtx::NDMA; ++k) {
+        if (cudaEventRecord(c->ev_dma[k], c->dma[k]) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+        if (cudaStreamWaitEvent(d0, c->ev_dma[k], 0) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+    }
+    CK(cudaStreamEndCapture(d0, &g));
+    cudaGraphExec_t ex = nullptr;
+    cudaError_t e = cudaGraphInstantiate(&ex, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        c->last_cuda = (int)e;
+        return PROACT_ERR_CUDA;
+    }
+    R.dma_exec = ex;
+    return rc;
+}
 
 // Library streams come from a per-device pool that outlives the rank contexts.  CUDA maps streams
 // onto CUDA_DEVICE_MAX_CONNECTIONS hardware queues round-robin at creation; a queue blocked by a
@@ -678,7 +755,7 @@ int proact_init_ex(int ngpus, int rank, const char *job)
         if (cudaEventCreateWithFlags(&c->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         if (cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         for (int k = 0; k < RankCtx::NDMA; ++k) {
-            if (pool_stream(c->device, &c->dma[k]) != cudaSuccess) return fail(PROACT_ERR_CUDA);
+            // copy-engine streams of MECH_DMA: created on its first launch (ensure_dma_streams)
             if (cudaEventCreateWithFlags(&c->ev_dma[k], cudaEventDisableTiming) != cudaSuccess) return fail(PROACT_ERR_CUDA);
         }
         if (cudaFuncSetAttribute(agent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)AGENT_SMEM_MAX) !=
@@ -898,6 +975,7 @@ int proact_region_set_chunk_dest(int id, uint32_t chunk, uint64_t mask)
         if (rc) return rc;
     }
     R.chunk_dest[chunk] = (uint32_t)mask;
+    if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }   // new geometry
     CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * (size_t)R.n_own, cudaMemcpyHostToDevice));
     return PROACT_OK;
 }
@@ -937,6 +1015,34 @@ int proact_region_debug_deliveries(int id, uint32_t *out, size_t n)
         CK(cudaMemcpy(out, D.deliv, 4 * need, cudaMemcpyDeviceToHost));
         CK(cudaMemset(D.deliv, 0, 4 * need));
     }
+    return PROACT_OK;
+}
+
+int proact_region_debug_state(int id, uint32_t *out, size_t n)
+{
+    RankCtx *c = need_ctx();
+    if (!c) return PROACT_ERR_STATE;
+    if (id < 0 || id >= c->nregions || !out) return PROACT_ERR_INVALID;
+    const Region &R = c->regions[id];
+    const region_dev &D = c->h.region[id];
+    const size_t need = 3 * (size_t)R.n_own + R.n_total + 8 + 2 * (size_t)MAXR;
+    if (n < need) return PROACT_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CK(cudaDeviceSynchronize());
+    uint32_t *o = out;
+    CK(cudaMemcpy(o, D.counter, 4 * (size_t)R.n_own, cudaMemcpyDeviceToHost));
+    o += R.n_own;
+    CK(cudaMemcpy(o, D.expected, 4 * (size_t)R.n_own, cudaMemcpyDeviceToHost));
+    o += R.n_own;
+    CK(cudaMemcpy(o, D.piecedone, 4 * (size_t)R.n_own, cudaMemcpyDeviceToHost));
+    o += R.n_own;
+    CK(cudaMemcpy(o, D.arrive, 4 * (size_t)R.n_total, cudaMemcpyDeviceToHost));
+    o += R.n_total;
+    CK(cudaMemcpy(o, D.qctl, 32, cudaMemcpyDeviceToHost));
+    o += 8;
+    CK(cudaMemcpy(o, c->h.done, 4 * MAXR, cudaMemcpyDeviceToHost));
+    o += MAXR;
+    for (int k = 0; k < MAXR; ++k) o[k] = k == 0 ? c->epoch : (k == 1 ? R.gen_done : 0);
     return PROACT_OK;
 }
 
@@ -1014,12 +1120,13 @@ thread_local const void *g_l2_base = nullptr;
 thread_local size_t g_l2_bytes = 0;
 
 cudaError_t launch_producer(const void *kernel, unsigned total, unsigned block, void **args, size_t smem,
-                            cudaStream_t s, int device, const void *l2_base, size_t l2_bytes)
+                            cudaStream_t s, int device, const void *l2_base, size_t l2_bytes, bool pdl = false)
 {
-    if (!l2_base || !l2_bytes) return cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s);
+    const bool window = l2_base && l2_bytes;
+    if (!window && !pdl) return cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s);
     static thread_local int limit_dev = -1;
     static thread_local size_t limit = 0;
-    if (limit_dev != device) {   // reserve the persisting L2 set-aside once per device
+    if (window && limit_dev != device) {   // reserve the persisting L2 set-aside once per device
         cudaDeviceProp prop;
         if (cudaGetDeviceProperties(&prop, device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
             limit = (size_t)prop.persistingL2CacheMaxSize;
@@ -1032,16 +1139,24 @@ cudaError_t launch_producer(const void *kernel, unsigned total, unsigned block, 
     cfg.blockDim = dim3(block);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeAccessPolicyWindow;
-    at[0].val.accessPolicyWindow.base_ptr = const_cast<void *>(l2_base);
-    at[0].val.accessPolicyWindow.num_bytes = l2_bytes;
-    at[0].val.accessPolicyWindow.hitRatio =
-        limit ? (float)std::min(1.0, (double)limit / (double)l2_bytes) : 0.f;
-    at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    cudaLaunchAttribute at[2];
+    unsigned n = 0;
+    if (window && limit) {
+        at[n].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[n].val.accessPolicyWindow.base_ptr = const_cast<void *>(l2_base);
+        at[n].val.accessPolicyWindow.num_bytes = l2_bytes;
+        at[n].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)limit / (double)l2_bytes);
+        at[n].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[n].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        ++n;
+    }
+    if (pdl) {   // programmatic dependent of the previous kernel on `s` (the separate agent)
+        at[n].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[n].val.programmaticStreamSerializationAllowed = 1;
+        ++n;
+    }
     cfg.attrs = at;
-    cfg.numAttrs = limit ? 1 : 0;
+    cfg.numAttrs = n;
     return cudaLaunchKernelExC(&cfg, kernel, args);
 }
 }  // namespace
@@ -1128,7 +1243,11 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     int nb = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
     if (nb < 1) return PROACT_ERR_INVALID;
-    unsigned cap = (unsigned)std::max(1, nb * c->nsm / std::max(1, c->ranks_on_device));
+    // a rank's share of the co-resident capacity; ranks sharing a device (loopback) leave a tenth of
+    // it free, so that every rank's sync / helper kernels and separate agent always find slots even
+    // while the other ranks' persistent producers spin in their arrival waits
+    const int rod = std::max(1, c->ranks_on_device);
+    unsigned cap = (unsigned)std::max(1, rod > 1 ? nb * c->nsm * 9 / (10 * rod) : nb * c->nsm);
     if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
     cudaStream_t s = (cudaStream_t)stream;
     if (after) {
@@ -1152,30 +1271,23 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
                                     cudaSharedmemCarveoutMaxShared));
             c->carveout_set.push_back(kernel);
         }
-        // the agent kernel first, on its own high-priority stream (ordered after my earlier
-        // work), so its CTAs are resident before the producer grid fills the device; the
-        // producer grid leaves one slot per agent CTA; my stream waits for the agent.
+        // the agent kernel first, then the producer on the SAME stream as its programmatic
+        // dependent (PDL): the producer may launch once every agent CTA has signalled
+        // launch_dependents (is resident), and it runs concurrently with the agent; the next work
+        // on the stream (the phase sync) waits for both.  No second stream, no stream memory
+        // wait: a cross-stream residency gate can deadlock when the two streams share a hardware
+        // queue (observed with 3 loopback ranks), a same-stream programmatic dependency cannot.
+        // The producer grid leaves room for the agent's CTAs (reserve below).
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
         la.flags |= proact::LCF_SEPARATE;
         size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
             asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
-        CK(cudaEventRecord(c->ev_start, s));
-        CK(cudaStreamWaitEvent(c->side, c->ev_start, 0));
-        agent_kernel<<<agent_ctas, agent_block, asmem, c->side>>>(la);
+        agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
         CK(cudaGetLastError());
-        CK(cudaEventRecord(c->ev_done, c->side));
         c->launches++;
-        // the producer launches only once every agent CTA is resident (wrap-safe GEQ)
         c->resident_total += agent_ctas;
-        {
-            int mrc = load_memops();
-            if (mrc) return mrc;
-            if (g_wait32((CUstream)s, (CUdeviceptr)c->h.resident, c->resident_total, CU_STREAM_WAIT_VALUE_GEQ) !=
-                CUDA_SUCCESS)
-                return PROACT_ERR_CUDA;
-        }
         lc.agent_ctas = 0;
         // producer slots an agent CTA displaces on its SM (shared memory / registers / threads)
         unsigned lost = 1;
@@ -1201,16 +1313,23 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         const unsigned reserve = std::min(cap - 1, agent_ctas * lost);
         if (total + reserve > cap) total = cap - reserve;
         *(launch_ctx *)args[0] = lc;
-        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
-        CK(cudaStreamWaitEvent(s, c->ev_done, 0));
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, true));
     } else if (lc.mech == PROACT_MECH_DMA && armed) {
-        // NEXT-3 "hardware PROACT": the copy engines are the transfer agent.  Per owned chunk,
-        // on a DMA stream: wait counter[c] == expected[c] (the producers' last tally), copy the
-        // chunk to every destination, reset the counter.  Before the first copy into peer p,
-        // wait for p's credit (it finished phase e-1, reading R6).  Prepared by the host like
-        // the paper's "descriptors for the geometry of each transfer prepared in advance" (L166).
+        // NEXT-3 "hardware PROACT": the copy engines are the transfer agent.  Per region, a
+        // program prepared once (the paper's "descriptors for the geometry of each transfer
+        // prepared in advance", L166) and replayed every phase as a CUDA graph: per transfer group
+        // of chunks, on one of the DMA streams, wait until the group counter says all its chunks
+        // are complete (the producers' last committers count them, proact::commit_chunk), copy
+        // the group to every destination, reset the counter.  Only the credit waits (peer p
+        // finished phase e-1, reading R6) depend on the epoch; they precede the replay.
         int rc = load_memops();
         if (rc) return rc;
+        for (int k = 0; k < RankCtx::NDMA; ++k)   // only contexts that use DMA hold these streams
+            if (!c->dma[k]) {
+                int lo = 0, hi = 0;
+                cudaDeviceGetStreamPriorityRange(&lo, &hi);
+                CK(cudaStreamCreateWithPriority(&c->dma[k], cudaStreamNonBlocking, hi));
+            }
         lc.agent_ctas = 0;
         *(launch_ctx *)args[0] = lc;
         CK(cudaEventRecord(c->ev_start, s));
@@ -1219,47 +1338,24 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         unsigned total = grid ? grid : cap;
         if (total > cap) total = cap;
         CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
-
-        uint32_t peers = 0;
-        for (int r = 0; r < c->nregions; ++r)
-            if (armed >> r & 1) {
-                const Region &R = c->regions[r];
-                if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
-                else peers |= (uint32_t)R.dest_mask;
-            }
-        peers &= ~(1u << c->rank);
-        for (int k = 0; k < RankCtx::NDMA; ++k) {
-            cudaStream_t d = c->dma[k];
-            CK(cudaStreamWaitEvent(d, c->ev_start, 0));
-            for (int p = 0; p < c->world; ++p)
-                if (peers >> p & 1)
-                    if (g_wait32((CUstream)d, (CUdeviceptr)(c->h.done + p), c->epoch << 1, CU_STREAM_WAIT_VALUE_GEQ) !=
-                        CUDA_SUCCESS)
-                        return PROACT_ERR_CUDA;
-        }
-        uint32_t rr = 0;
+        cudaStream_t d0 = c->dma[0];
+        CK(cudaStreamWaitEvent(d0, c->ev_start, 0));
         for (int r = 0; r < c->nregions; ++r) {
             if (!(armed >> r & 1)) continue;
-            const Region &R = c->regions[r];
-            const region_dev &D = c->h.region[r];
-            for (uint32_t k = 0; k < R.n_own; ++k) {
-                cudaStream_t d = c->dma[rr++ % RankCtx::NDMA];
-                const uint64_t lo = R.own_off + (uint64_t)k * R.chunk;
-                const uint64_t len = std::min<uint64_t>(R.chunk, R.own_bytes - (uint64_t)k * R.chunk);
-                if (g_wait32((CUstream)d, (CUdeviceptr)(D.counter + k), (cuuint32_t)len, CU_STREAM_WAIT_VALUE_EQ) !=
-                    CUDA_SUCCESS)
-                    return PROACT_ERR_CUDA;
-                const uint32_t m = R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k];
-                for (int p = 0; p < c->world; ++p)
-                    if (p != c->rank && (m >> p & 1))
-                        CK(cudaMemcpyAsync(D.peer_base[p] + lo, R.base + lo, len, cudaMemcpyDeviceToDevice, d));
-                if (g_write32((CUstream)d, (CUdeviceptr)(D.counter + k), 0, 0) != CUDA_SUCCESS) return PROACT_ERR_CUDA;
+            Region &R = c->regions[r];
+            if (!R.dma_exec) {
+                int brc = build_dma_program(c, r);
+                if (brc) return brc;
             }
+            for (int p = 0; p < c->world; ++p)
+                if (R.dma_peers >> p & 1)
+                    if (g_wait32((CUstream)d0, (CUdeviceptr)(c->h.done + p), c->epoch << 1, CU_STREAM_WAIT_VALUE_GEQ) !=
+                        CUDA_SUCCESS)
+                        return PROACT_ERR_CUDA;
+            CK(cudaGraphLaunch(R.dma_exec, d0));
         }
-        for (int k = 0; k < RankCtx::NDMA; ++k) {
-            CK(cudaEventRecord(c->ev_dma[k], c->dma[k]));
-            CK(cudaStreamWaitEvent(s, c->ev_dma[k], 0));
-        }
+        CK(cudaEventRecord(c->ev_dma[0], d0));
+        CK(cudaStreamWaitEvent(s, c->ev_dma[0], 0));
     } else {
         if (lc.mech == PROACT_MECH_INLINE && c->world > 1 && armed) {
             // PROACT-inline stores straight into the peers' replicas: like the agent (reading
@@ -1400,6 +1496,7 @@ int proact_finalize(void)
         for (void *p : R.opened) cudaIpcCloseMemHandle(p);
         if (R.meta) cudaFree(R.meta);
         if (R.d_chunk_dest) cudaFree(R.d_chunk_dest);
+        if (R.dma_exec) cudaGraphExecDestroy(R.dma_exec);
     }
     for (void *p : c->opened) cudaIpcCloseMemHandle(p);
     int rc2 = c->shm.barrier();  // nobody uses our memory any more
@@ -1409,7 +1506,7 @@ int proact_finalize(void)
     cudaFreeHost(c->h_err);
     pool_return(c->device, c->side);   // idle after the device synchronisation above
     for (int k = 0; k < RankCtx::NDMA; ++k) {
-        pool_return(c->device, c->dma[k]);
+        if (c->dma[k]) cudaStreamDestroy(c->dma[k]);
         if (c->ev_dma[k]) cudaEventDestroy(c->ev_dma[k]);
     }
     if (c->ev_start) cudaEventDestroy(c->ev_start);

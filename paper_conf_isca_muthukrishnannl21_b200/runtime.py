@@ -128,6 +128,22 @@ def debug_deliveries(rid: int):
     return out[:n].reshape(info.n_own_chunks, world())
 
 
+def debug_state(rid: int) -> dict:
+    """proact_region_debug_state as numpy arrays (post-mortem after a watchdog timeout)."""
+    import numpy as np
+    info = region_info(rid)
+    n_own, n_total = info.n_own_chunks, info.n_total_chunks
+    buf = np.zeros(3 * n_own + n_total + 8 + 32, dtype=np.uint32)
+    check(lib().proact_region_debug_state(rid, ctypes.c_void_p(buf.ctypes.data), buf.size), "debug_state")
+    o = 0
+    out = {}
+    for k, n in (("counter", n_own), ("expected", n_own), ("piecedone", n_own), ("arrive", n_total),
+                 ("qctl", 8), ("done", 16), ("host", 16)):
+        out[k] = buf[o:o + n].copy()
+        o += n
+    return out
+
+
 # ------------------------------------------------------------------ phases
 def phase_sync(stream=None, barrier: bool = False) -> None:
     check(lib().proact_phase_sync(ctypes.c_void_p(_stream_handle(stream)),

@@ -55,10 +55,29 @@ def _litmus_body(r, G, words, chunk, phases, cfg, flip_after=None):
             rt.host_barrier()
         wl.litmus_phase(rid[p & 1], rid[(p & 1) ^ 1], p, SEED, bad, s)
         barrier = p == phases - 1 or (flip_after is not None and p == flip_after - 1)
-        rt.phase_sync(s, barrier=barrier)
+        try:
+            rt.phase_sync(s, barrier=barrier)
+        except ProactError:
+            _post_mortem(r, p, rid)
+            raise
     s.synchronize()
-    rt.check_device()
+    try:
+        rt.check_device()
+    except ProactError:
+        _post_mortem(r, phases, rid)
+        raise
     return int(bad.item()), flipped
+
+
+def _post_mortem(r, p, rid):
+    import sys
+    for k, x in enumerate(rid):
+        st = rt.debug_state(x)
+        info = rt.region_info(x)
+        print(f"[post-mortem] rank {r} phase {p} region {x} base {info.replica_base:#x}: epoch/gens {st['host'][:2].tolist()} "
+              f"counter {st['counter'].tolist()} expected {st['expected'].tolist()} piecedone {st['piecedone'].tolist()} "
+              f"arrive_raw {st['arrive'].tolist()} "
+              f"qctl {st['qctl'].tolist()} done_raw {st['done'][:4].tolist()}", file=sys.stderr)
 
 
 @pytest.mark.parametrize("name", list(MECHS))
