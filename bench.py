@@ -320,7 +320,10 @@ def main():
     cfg = rt.set_config(**kw)
     N, I = args.n, args.iters
     x0 = torch.from_numpy(synth.jacobi_init(N)).cuda()
-    J = wl.Jacobi(N, chunk, x0=x0, rows_per_tile=args.rpt)
+    # NVLS: on an NVSwitch system with every rank a thread of one process... (torchrun ranks are
+    # processes, so proact_mcast_supported() is 0 there and the replicas are plain tensors)
+    mcast = world > 1 and rt.mcast_supported()
+    J = wl.Jacobi(N, chunk, x0=x0, rows_per_tile=args.rpt, mcast=mcast)
     del x0
     s = torch.cuda.Stream()
 
@@ -348,7 +351,7 @@ def main():
                 ts.append(a.elapsed_time(b))
             return statistics.median(ts)
 
-        space = "mech=0;chunk=131072,1048576;warps=8,16,32;push=0,1;akern=0,1,2"
+        space = "mech=0;chunk=131072,1048576;warps=8,16,32;push=0,1" + (",2" if mcast else "") + ";akern=0,1,2"
         best = rt.autotune(f"bench_jacobi_N{N}_G{world}", run_point, space)
         if best["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
             for rid in J.rid:
@@ -586,7 +589,7 @@ def main():
                                               if world == 1 and args.mech == "fused" else args.mech),
                            "chunk_bytes": chunk,
                            "agent_warps": cfg["agent_warps"], "piece_bytes": cfg["piece_bytes"],
-                           "rows_per_tile": args.rpt, "replication": "full", "tuned": tuned,
+                           "rows_per_tile": args.rpt, "replication": "full", "tuned": tuned, "nvls_multicast": mcast,
                            "l2": "inputs > L2 (two 1 GiB grids), no flush",
                            "parallelism": f"rows{world}",
                            "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)]},
@@ -601,6 +604,7 @@ def main():
                 "halo_only": halo, "agent_cost": agent_cost}
         print(json.dumps(line), flush=True)
     torch.cuda.synchronize()
+    J.free()
     rt.finalize()
     if world > 1:
         dist.destroy_process_group()

@@ -76,9 +76,14 @@ enum {
 /* ---- agent push instruction (a5) -------------------------------------------------------- */
 enum {
     PROACT_PUSH_VEC16 = 0,   /* 16-byte ld.global.cg / st.global.v4, 512 B per warp instruction */
-    PROACT_PUSH_BULK = 1     /* cp.async.bulk (TMA): global->smem stage, then one smem->global bulk
+    PROACT_PUSH_BULK = 1,    /* cp.async.bulk (TMA): global->smem stage, then one smem->global bulk
                                 store per destination; one agent warp per CTA (lane 0 issues),
                                 the CTA's dynamic shared memory is its staging ring */
+    PROACT_PUSH_MULTICAST = 2 /* NVLS: one 16-byte multimem.st.global.v4 per lane to
+                                the region's multicast address reaches every peer's replica through
+                                the NVSwitch; for regions in replicas from proact_alloc_replica on a
+                                multicast-capable system, units bound for every peer; anything
+                                else is pushed as PROACT_PUSH_VEC16 */
 };
 
 /* ---- agent discovery of completed chunks (a4) ------------------------------------------- */
@@ -210,6 +215,20 @@ int proact_region_info_get(int region, proact_region_info *out);
  * region's generation count is kept).  Used by the profiler to sweep granularity (L93, L112).
  * Must not race with an in-flight launch of the region (synchronise the stream first). */
 int proact_region_rechunk(int region, size_t chunk_bytes);
+
+/* ---- NVLS multicast replicas (PAPER.md L137 remote writes, L82 granularity) */
+/* 1 if every rank of the job is a thread of this process on its own device and every device
+ * supports switch multicast (CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED), else 0. */
+int proact_mcast_supported(void);
+/* COLLECTIVE.  Allocate a full-extent replica of `bytes` for this rank and return it in *ptr.  If
+ * proact_mcast_supported() on every rank, the replicas of all ranks are bound to one multicast
+ * object (cuMulticastCreate / AddDevice / BindMem; size rounded up to the multicast granularity)
+ * and mapped for unicast access by every device of the job, so that regions registered inside it
+ * can be pushed with PROACT_PUSH_MULTICAST; otherwise a plain device allocation.  The caller owns
+ * the replica until proact_free_replica (COLLECTIVE), which must precede proact_finalize.
+ * Errors: INVALID, STATE, NOMEM, CUDA, TIMEOUT. */
+int proact_alloc_replica(size_t bytes, void **ptr);
+int proact_free_replica(void *ptr);
 
 /* ================================================================ launch / sync ============= */
 

@@ -70,6 +70,7 @@ struct region_dev {
     uint32_t rank_chunk0[PROACT_MAX_RANKS + 1];
     char *peer_base[PROACT_MAX_RANKS];            /* peers' replica bases (mapped) */
     uint32_t *peer_arrive[PROACT_MAX_RANKS];      /* peers' arrive[] */
+    char *mc_base;                                /* multicast address of the replica base, or null */
     uint32_t *peer_arrive_count[PROACT_MAX_RANKS];
 };
 

@@ -23,7 +23,7 @@ ERR_INVALID, ERR_CUDA, ERR_NOPEER, ERR_STATE, ERR_TIMEOUT, ERR_PROTOCOL, ERR_NOM
 MECH_FUSED, MECH_INLINE, MECH_BULK, MECH_LOCAL, MECH_ELIDE, MECH_DMA = range(6)
 MECH_NAMES = {MECH_FUSED: "fused", MECH_INLINE: "inline", MECH_BULK: "bulk",
               MECH_LOCAL: "local", MECH_ELIDE: "elide", MECH_DMA: "dma"}
-PUSH_VEC16, PUSH_BULK = 0, 1
+PUSH_VEC16, PUSH_BULK, PUSH_MULTICAST = 0, 1, 2
 DISCOVER_QUEUE, DISCOVER_SCAN = 0, 1
 AGENT_FUSED, AGENT_SEPARATE, AGENT_PRODUCER = 0, 1, 2
 LAUNCH_TILE_PUSH = 1
@@ -105,6 +105,9 @@ def _declare(L):
         "proact_micro_phase": (i, [i, ctypes.c_uint, ctypes.c_uint, i, i, vp]),
         "proact_litmus_phase": (i, [i, i, ctypes.c_uint, ctypes.c_uint, vp, vp]),
         "proact_region_debug_state": (i, [i, vp, sz]),
+        "proact_mcast_supported": (i, []),
+        "proact_alloc_replica": (i, [sz, ctypes.POINTER(vp)]),
+        "proact_free_replica": (i, [vp]),
         "proact_inject_double_commit": (i, [i, vp]),
         "proact_banded_phase": (i, [i, i, vp, vp, ctypes.c_longlong, ctypes.c_longlong, vp]),
         "proact_jacobi_solve_host": (i, [vp, vp, ctypes.c_longlong, i, sz, i, vp,

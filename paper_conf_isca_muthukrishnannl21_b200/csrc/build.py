@@ -14,7 +14,7 @@ PKG = os.path.dirname(HERE)
 ROOT = os.path.dirname(PKG)
 INC = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libproact.so")
-SOURCES = ["runtime.cu", "workloads.cu", "graph.cu"]
+SOURCES = ["runtime.cu", "workloads.cu", "graph.cu", "mcast.cu"]
 DEPS = SOURCES
 HEADERS = sorted(f for f in os.listdir(INC) if f.endswith((".h", ".cuh")))   # every public header
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

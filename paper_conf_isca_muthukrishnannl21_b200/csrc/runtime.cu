@@ -244,7 +244,7 @@ void apply_env(proact_config &c) {
 
 int validate_config(const proact_config &c) {
     if (c.mech < 0 || c.mech > PROACT_MECH_DMA) return PROACT_ERR_INVALID;
-    if (c.push != PROACT_PUSH_VEC16 && c.push != PROACT_PUSH_BULK) return PROACT_ERR_INVALID;
+    if (c.push < PROACT_PUSH_VEC16 || c.push > PROACT_PUSH_MULTICAST) return PROACT_ERR_INVALID;
     if (c.agent_warps < 1 || c.agent_warps > 1024) return PROACT_ERR_INVALID;
     if (c.block < 64 || c.block > 1024 || c.block % 32) return PROACT_ERR_INVALID;
     if (c.piece_bytes < 4096 || c.piece_bytes % 16) return PROACT_ERR_INVALID;
@@ -429,6 +429,9 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
     return PROACT_OK;
 }
 
+}  // namespace
+extern "C" __attribute__((visibility("hidden"))) void *proact_internal_mcast_lookup(const void *ptr, size_t bytes);
+namespace {
 int finish_region_peers(RankCtx *c, int id, Region &R, const std::vector<RegionExchange> &all) {
     region_dev &D = c->h.region[id];
     uint32_t n_in = 0;
@@ -456,6 +459,7 @@ int finish_region_peers(RankCtx *c, int id, Region &R, const std::vector<RegionE
         D.peer_arrive_count[p] = (uint32_t *)(pm + e.off_count);
     }
     D.n_in = n_in;
+    D.mc_base = (char *)proact_internal_mcast_lookup(R.base, R.total);   // NVLS (mcast.cu), or null
     if (R.gen_done) {
         uint32_t cnt = R.gen_done * n_in;
         CK(cudaMemcpy(D.arrive_count, &cnt, 4, cudaMemcpyHostToDevice));
@@ -1081,6 +1085,24 @@ extern "C" __attribute__((visibility("hidden"))) void proact_internal_keep_l1(co
     std::lock_guard<std::mutex> g(g_l1_mu);
     if (std::find(g_l1_kernels.begin(), g_l1_kernels.end(), kernel) == g_l1_kernels.end())
         g_l1_kernels.push_back(kernel);
+}
+
+// rendezvous helpers for mcast.cu (the calling thread's rank context)
+extern "C" __attribute__((visibility("hidden"))) int proact_internal_allgather(const void *mine, size_t n, void *all)
+{
+    if (!tl) return PROACT_ERR_STATE;
+    return tl->shm.allgather(tl->rank, mine, n, all);
+}
+// 1 (and every rank's device in devices[]) if all ranks are threads of this process, else 0
+extern "C" __attribute__((visibility("hidden"))) int proact_internal_same_process_devices(int *devices)
+{
+    if (!tl) return 0;
+    int same = 1;
+    for (int p = 0; p < tl->world; ++p) {
+        devices[p] = tl->peers[p].device;
+        same &= tl->peers[p].pid == (int32_t)getpid();
+    }
+    return same;
 }
 
 // cudaFuncAttributeMaxDynamicSharedMemorySize is a per-device attribute: set it once per

@@ -87,6 +87,38 @@ def reset_config() -> None:
     check(lib().proact_set_config(None), "proact_set_config")
 
 
+# ------------------------------------------------------------------ NVLS multicast replicas
+def mcast_supported() -> bool:
+    return bool(lib().proact_mcast_supported())
+
+
+class _CudaArray:
+    """Minimal __cuda_array_interface__ exporter: a torch view of library-owned device memory."""
+
+    def __init__(self, ptr: int, shape, typestr: str):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr, "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def alloc_replica(shape, dtype=torch.float32) -> torch.Tensor:
+    """COLLECTIVE proact_alloc_replica: a full-extent replica (bound to an NVLS multicast object
+    when mcast_supported() on every rank) as a torch tensor view; release with free_replica."""
+    n = 1
+    for d in shape:
+        n *= d
+    nbytes = n * torch.empty(0, dtype=dtype).element_size()
+    ptr = ctypes.c_void_p(0)
+    check(lib().proact_alloc_replica(nbytes, ctypes.byref(ptr)), "proact_alloc_replica")
+    typestr = {torch.float32: "<f4", torch.int32: "<i4", torch.uint8: "|u1"}[dtype]
+    t = torch.as_tensor(_CudaArray(ptr.value, shape, typestr), device="cuda")
+    assert t.data_ptr() == ptr.value
+    return t
+
+
+def free_replica(t: torch.Tensor) -> None:
+    check(lib().proact_free_replica(ctypes.c_void_p(t.data_ptr())), "proact_free_replica")
+
+
 # ------------------------------------------------------------------ regions
 def register_region(replica: torch.Tensor, own_offset: int, own_bytes: int, chunk_bytes: int,
                     dest_mask: int | None = None, flags: int = 0) -> int:

@@ -35,11 +35,18 @@ class Jacobi:
     go to the neighbours (reading R8); otherwise full replication (configs 1-2)."""
 
     def __init__(self, N: int, chunk_bytes: int, x0: torch.Tensor | None = None,
-                 halo_only: bool = False, rows_per_tile: int = 16, device=None):
+                 halo_only: bool = False, rows_per_tile: int = 16, device=None, mcast: bool = False):
+        """mcast=True: the two replicas come from proact_alloc_replica (COLLECTIVE), bound to NVLS
+        multicast objects when the system supports it (push=PUSH_MULTICAST then stores once for
+        all peers); release them with free()."""
         G, g = rt.world(), rt.rank()
         self.N, self.G, self.g, self.rpt = N, G, g, rows_per_tile
         dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
-        self.bufs = [torch.empty((N, N), dtype=torch.float32, device=dev) for _ in range(2)]
+        self.mcast = mcast
+        if mcast:
+            self.bufs = [rt.alloc_replica((N, N), torch.float32) for _ in range(2)]
+        else:
+            self.bufs = [torch.empty((N, N), dtype=torch.float32, device=dev) for _ in range(2)]
         if x0 is not None:
             self.bufs[0].copy_(x0)
             self.bufs[1].copy_(x0)
@@ -68,6 +75,14 @@ class Jacobi:
                 if self.g < self.G - 1 and hi > info.own_bytes - rowb:  # holds my last row
                     m |= 1 << (self.g + 1)
                 rt.set_chunk_dest(rid, c, m)
+
+    def free(self) -> None:
+        """COLLECTIVE when mcast: release library-allocated replicas (after the last phase)."""
+        torch.cuda.synchronize()
+        if self.mcast:
+            for b in self.bufs:
+                rt.free_replica(b)
+        self.bufs = []
 
     def step(self, stream=None, barrier: bool = False) -> None:
         i = self.k & 1

@@ -80,8 +80,14 @@ def _post_mortem(r, p, rid):
               f"qctl {st['qctl'].tolist()} done_raw {st['done'][:4].tolist()}", file=sys.stderr)
 
 
-@pytest.mark.parametrize("name", list(MECHS))
-@pytest.mark.parametrize("G", [2, 3])
+# G = 3 loopback ranks whose every producer CTA waits for all peers' previous generation need all
+# three ranks' persistent grids co-resident on one GPU at once; next to separately launched agent
+# kernels CUDA does not guarantee that (one rank per GPU, the deployment case, needs nothing of the
+# kind), so the separate-agent configurations run at G = 2 only
+_G3 = [n for n in MECHS if not n.startswith("fused_separate")]
+
+
+@pytest.mark.parametrize("name,G", [(n, 2) for n in MECHS] + [(n, 3) for n in _G3])
 def test_litmus_no_stale_word_after_arrival(name, G):
     phases = 10000 if G == 2 else 2000
     words = 1 << 16                 # 256 KiB region, 16 KiB chunks: 16 chunks, ragged at G = 3
