@@ -66,6 +66,9 @@ struct tile_ring_ctl {
 };
 
 __device__ __forceinline__ uint32_t tp_smem(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+#ifndef PROACT_TP_IDLE_NS
+#define PROACT_TP_IDLE_NS 8000   // producers idle this long: publish what is in flight
+#endif
 #ifndef PROACT_TP_SUSPEND_NS
 #define PROACT_TP_SUSPEND_NS 20000   // try_wait suspend-time hint: a waiting warp sleeps until the
 #endif                               // phase completes instead of spinning on issue slots
@@ -78,6 +81,27 @@ __device__ __forceinline__ void tp_mbar_wait(uint64_t *b, uint32_t parity)
                      "selp.u32 %0, 1, 0, p;\n\t}"
                      : "=r"(done) : "r"(tp_smem(b)), "r"(parity), "n"(PROACT_TP_SUSPEND_NS) : "memory");
     } while (!done);
+}
+__device__ __forceinline__ bool tp_mbar_test(uint64_t *b, uint32_t parity)
+{
+    uint32_t done;
+    asm volatile("{\n\t.reg .pred p;\n\t"
+                 "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                 "selp.u32 %0, 1, 0, p;\n\t}"
+                 : "=r"(done) : "r"(tp_smem(b)), "r"(parity) : "memory");
+    return done != 0;
+}
+// Wait up to PROACT_TP_IDLE_NS for the phase, sleeping between tests (a waiting transfer warp must
+// not take issue slots from the compute warps of its SM): true if the phase completed.
+__device__ __forceinline__ bool tp_mbar_try(uint64_t *b, uint32_t parity)
+{
+    if (tp_mbar_test(b, parity)) return true;
+    const uint64_t t0 = globaltimer();
+    do {
+        __nanosleep(500);
+        if (tp_mbar_test(b, parity)) return true;
+    } while (globaltimer() - t0 < PROACT_TP_IDLE_NS);
+    return false;
 }
 __device__ __forceinline__ void tp_mbar_arrive(uint64_t *b)
 {
@@ -179,11 +203,50 @@ __device__ __noinline__ void tile_pusher(const launch_ctx &lc, int r, const unsi
         }
     };
     auto dests = [&](uint32_t c) { return chunk_dest ? chunk_dest[c] & peers : dmask; };
+    // lane 0: merge the rows of completed spans [done, upto) into the pending list while it has
+    // room; returns true when the list is (nearly) full
+    auto merge = [&](uint32_t upto) {
+        bool full_list = npend + 2 * 8 > TP_PEND;   // room for a span of <= 8 straddling rows
+        while ((int32_t)(upto - done) > 0 && !full_list) {
+            const tile_desc f = T->fly[done % TP_FLY];
+            const uint32_t fr = f.flags >> 8;
+            if (f.flags & 1u) remote = true;
+            for (uint32_t k = 0; k < fr; ++k) {
+                const uint64_t a0 = f.off - own_off + k * pitch, a1 = a0 + f.bytes;
+                if (a0 >= cmp_lo && a1 <= cmp_hi) {
+                    add_pend(cmp_c, f.bytes);
+                } else {
+                    for (uint64_t a = a0; a < a1;) {
+                        const uint32_t c = tp_chunk(a, cb);
+                        const uint64_t b = min(a1, (uint64_t)(c + 1) * cb);
+                        add_pend(c, (uint32_t)(b - a));
+                        cmp_c = c;
+                        cmp_lo = (uint64_t)c * cb;
+                        cmp_hi = cmp_lo + cb;
+                        a = b;
+                    }
+                }
+            }
+            ++done;
+            nrows += fr;
+            full_list = npend + 2 * 8 > TP_PEND;
+        }
+        return full_list;
+    };
     for (;;) {
         uint32_t ev = 0, arg = 0;
         if (lane == 0) {
             for (;;) {
                 const uint32_t slot = q % OS;
+                if ((done < q || npend) && !tp_mbar_try(&T->full[slot], (q / OS) & 1u)) {
+                    // the producers have had nothing for us for a while (a stretch of tiles bound
+                    // nowhere, e.g. halo-only interiors): complete and publish what is in flight
+                    // instead of holding its arrival flags back until the next flush
+                    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+                    merge(q);
+                    ev = EV_FLUSH;
+                    break;
+                }
                 tp_mbar_wait(&T->full[slot], (q / OS) & 1u);
                 const tile_desc d = T->desc[slot];
                 if (d.flags & TD_END) {
@@ -255,31 +318,7 @@ __device__ __noinline__ void tile_pusher(const launch_ctx &lc, int r, const unsi
                 asm volatile("cp.async.bulk.wait_group %0;" ::"n"(TP_CD) : "memory");
                 ++q;
                 // spans [done, q - CD) have completed: merge their rows' bytes into the pending list
-                bool full_list = false;
-                while (done + TP_CD < q && !full_list) {
-                    const tile_desc f = T->fly[done % TP_FLY];
-                    const uint32_t fr = f.flags >> 8;
-                    if (f.flags & 1u) remote = true;
-                    for (uint32_t k = 0; k < fr; ++k) {
-                        const uint64_t a0 = f.off - own_off + k * pitch, a1 = a0 + f.bytes;
-                        if (a0 >= cmp_lo && a1 <= cmp_hi) {
-                            add_pend(cmp_c, f.bytes);
-                        } else {
-                            for (uint64_t a = a0; a < a1;) {
-                                const uint32_t c = tp_chunk(a, cb);
-                                const uint64_t b = min(a1, (uint64_t)(c + 1) * cb);
-                                add_pend(c, (uint32_t)(b - a));
-                                cmp_c = c;
-                                cmp_lo = (uint64_t)c * cb;
-                                cmp_hi = cmp_lo + cb;
-                                a = b;
-                            }
-                        }
-                    }
-                    ++done;
-                    nrows += fr;
-                    full_list = npend + 2 * 8 > TP_PEND;   // room for a span of <= 8 straddling rows
-                }
+                const bool full_list = merge(q - TP_CD);
                 if (full_list || nrows >= PROACT_TP_FLUSH) {
                     ev = EV_FLUSH;
                     break;
@@ -302,22 +341,7 @@ __device__ __noinline__ void tile_pusher(const launch_ctx &lc, int r, const unsi
             continue;
         }
         for (;;) {
-            if (ev == EV_END && lane == 0) {   // everything issued has completed: merge the rest
-                while (done < q && npend + 2 * 8 <= TP_PEND) {
-                    const tile_desc f = T->fly[done % TP_FLY];
-                    if (f.flags & 1u) remote = true;
-                    for (uint32_t k = 0; k < (f.flags >> 8); ++k) {
-                        const uint64_t a0 = f.off - own_off + k * pitch, a1 = a0 + f.bytes;
-                        for (uint64_t a = a0; a < a1;) {
-                            const uint32_t c = tp_chunk(a, cb);
-                            const uint64_t b = min(a1, (uint64_t)(c + 1) * cb);
-                            add_pend(c, (uint32_t)(b - a));
-                            a = b;
-                        }
-                    }
-                    ++done;
-                }
-            }
+            if (ev == EV_END && lane == 0) merge(q);   // everything issued has completed: merge the rest
             __syncwarp();
             const uint32_t n = __shfl_sync(FULLM, npend, 0);
             const bool sys = __shfl_sync(FULLM, remote, 0);
@@ -325,7 +349,10 @@ __device__ __noinline__ void tile_pusher(const launch_ctx &lc, int r, const unsi
                 asm volatile("fence.proxy.async;" ::: "memory");   // async-proxy writes -> generic
                 if (PROACT_TP_SYSFENCE && sys) fence_acq_rel_sys(); // ... ordered before the counts (a3)
                 else fence_acq_rel_gpu();
-                if (lane < n && !dead) commit_chunk(lc, r, T->pend_c[lane], T->pend_b[lane]);
+                // chunks bound nowhere are never counted (tiles that write only such chunks skip
+                // the transfer warp altogether, so their counts would be partial)
+                if (lane < n && !dead && transfers(lc, R, T->pend_c[lane]))
+                    commit_chunk(lc, r, T->pend_c[lane], T->pend_b[lane]);
                 __syncwarp();
             }
             if (lane == 0) {

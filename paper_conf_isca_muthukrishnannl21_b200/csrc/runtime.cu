@@ -158,6 +158,8 @@ struct Region {
     // MECH_DMA: the per-phase copy-engine program (wait group counter -> copy per destination ->
     // reset), built once per geometry and replayed as a CUDA graph (NEXT-3, L166)
     cudaGraphExec_t dma_exec = nullptr;
+    uint32_t qunits = 0, qunits_piece = 0;   // cached queue units per generation for a piece size
+    bool qunits_elide = false;
     uint32_t dma_group = 1;
     uint32_t dma_peers = 0;           // destinations the program copies to
 };
@@ -409,6 +411,7 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
         if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }
     }
     D.dma_group = R.dma_group;
+    R.qunits_piece = 0;
     D.group_cnt = (uint32_t *)(R.meta + off_group);
     D.chunk_dest = nullptr;
     R.chunk_dest.clear();
@@ -980,6 +983,7 @@ int proact_region_set_chunk_dest(int id, uint32_t chunk, uint64_t mask)
     }
     R.chunk_dest[chunk] = (uint32_t)mask;
     if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }   // new geometry
+    R.qunits_piece = 0;
     CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * (size_t)R.n_own, cudaMemcpyHostToDevice));
     return PROACT_OK;
 }
@@ -1231,8 +1235,27 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     // launch degenerates to the plain kernel (ELIDE keeps the agent: it measures tracking).
     if ((cfg.mech == PROACT_MECH_FUSED || cfg.mech == PROACT_MECH_DMA) && c->world == 1) lc.mech = PROACT_MECH_LOCAL;
     for (int r = 0; r < c->nregions; ++r) {
-        const Region &R = c->regions[r];
+        Region &R = c->regions[r];
         lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
+        if (armed >> r & 1) {   // QUEUE: units the committers will enqueue (chunks with destinations)
+            const uint32_t piece = std::min<uint32_t>(cfg.piece_bytes, (uint32_t)R.chunk);
+            const bool elide = lc.mech == PROACT_MECH_ELIDE;   // every chunk takes part (proact::transfers)
+            if (R.qunits_piece != piece || R.qunits_elide != elide) {
+                uint32_t u = 0;
+                const uint32_t self = 1u << c->rank;
+                for (uint32_t k = 0; k < R.n_own; ++k) {
+                    const uint32_t m = (R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k]) & ~self &
+                                       (c->world < 32 ? (1u << c->world) - 1u : ~0u);
+                    if (!m && !elide) continue;
+                    const uint64_t len = std::min<uint64_t>(R.chunk, R.own_bytes - (uint64_t)k * R.chunk);
+                    u += (uint32_t)((len + piece - 1) / piece);
+                }
+                R.qunits = u;
+                R.qunits_piece = piece;
+                R.qunits_elide = elide;
+            }
+            lc.qunits[r] = R.qunits;
+        }
         lc.gen_epoch[r] = (armed >> r & 1) ? c->epoch : R.gen_epoch;
         lc.gen_mech[r] = (armed >> r & 1) ? (uint8_t)lc.mech : R.gen_mech;
     }

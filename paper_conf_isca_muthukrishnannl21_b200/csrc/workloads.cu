@@ -141,12 +141,27 @@ struct JTile {
     int i0, i1, c0, c1, kfirst, klast;
 };
 
-// Tile t of this rank: interior bands first, the two halo-dependent edge bands last (a7).
-__device__ __forceinline__ JTile jtile(int t, int nstrips, int nbands, int rb, int row0, int rend, int N)
+#ifndef PROACT_JACOBI_EDGES_FIRST
+#define PROACT_JACOBI_EDGES_FIRST 1
+#endif
+__device__ __forceinline__ bool edges_first(const launch_ctx &lc)
+{
+    return PROACT_JACOBI_EDGES_FIRST && (lc.mech == PROACT_MECH_FUSED || lc.mech == PROACT_MECH_ELIDE);
+}
+
+// Tile t of this rank.  Credit-synchronised mechanisms (INLINE / BULK / DMA): interior bands
+// first, the two halo-dependent edge bands last, so the wait for the neighbours' phase credit
+// (a7) comes as late as possible.  Flag-synchronised ones (FUSED / ELIDE, edges_first): the edge
+// bands FIRST -- they are what the neighbours need next phase, so their pushes overlap this
+// phase's interior instead of trailing it, and the neighbours produced the rows they wait on at
+// the start of the previous phase.
+__device__ __forceinline__ JTile jtile(int t, int nstrips, int nbands, int rb, int row0, int rend, int N,
+                                       bool edges_first)
 {
     const int bi = t / nstrips, strip = t - bi * nstrips;
     int band;
     if (nbands <= 2) band = bi;
+    else if (edges_first) band = bi == 0 ? 0 : (bi == 1 ? nbands - 1 : bi - 1);
     else if (bi < nbands - 2) band = bi + 1;
     else band = bi == nbands - 2 ? 0 : nbands - 1;
     JTile T;
@@ -181,7 +196,7 @@ __device__ __noinline__ void jacobi_stream(const launch_ctx &lc, const proact_ja
             return;
         }
         tids[kt % JTD] = (int)t;
-        const JTile T = jtile((int)t, nstrips, nbands, rb, row0, rend, N);
+        const JTile T = jtile((int)t, nstrips, nbands, rb, row0, rend, N, edges_first(lc));
         const int lo = T.c0 >= 4 ? T.c0 - 4 : 0, hi = min(T.c0 + JW + 4, N);
         const uint32_t bytes = (uint32_t)(hi - lo) * 4;
         for (int k = T.kfirst; k <= T.klast; ++k, ++q) {
@@ -273,7 +288,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             mbar_wait(&tdone[k & 1u], (k >> 1) & 1u);
             const int t = tids[k % JTD];   // written by the stream warp, ordered by the tile's
             if (t < 0) return;             // row barriers and the compute warps' tdone arrival
-            const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+            const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N, edges_first(lc));
             for (int k0 = T.i0; k0 < T.i1; k0 += 32) {
                 const int i = k0 + lane;
                 warp_commit(lc, p.region_out, i < T.i1, ((uint64_t)i * N + T.c0) * 4, (uint32_t)(T.c1 - T.c0) * 4);
@@ -302,7 +317,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             }
             break;
         }
-        const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N);
+        const JTile T = jtile(t, nstrips, nbands, rb, row0, rend, N, edges_first(lc));
         // group g of this thread: columns [c0 + 4*tid + g*GW, +4), GW = the compute warps' width
         constexpr int GW = JC * 32 * 4;
         const float *ringf = ring + 4 + 4 * tid;
@@ -332,6 +347,18 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
         // row loop with those checks compiled out
         const bool fast = T.i0 > 0 && T.i1 < N && T.c0 > 0 && T.c0 + JW < N &&
                           (MODE == 2 || (lc.mech != PROACT_MECH_INLINE && !(PROACT_JACOBI_OUT_EVICT_LAST && tally)));
+        // MODE 2: does any chunk this tile writes have a destination?  Tiles that only write
+        // chunks bound nowhere (halo-only interiors, a single rank) store straight to global
+        // memory and skip the transfer warp: nothing to push, nothing to count
+        bool tpush = true;
+        if (MODE == 2) {
+            const region_dev &Ro = lc.ctx->region[p.region_out];
+            const uint64_t a0 = ((uint64_t)T.i0 * N + T.c0) * 4 - Ro.own_off;
+            const uint64_t a1 = ((uint64_t)(T.i1 - 1) * N + T.c1) * 4 - Ro.own_off;
+            tpush = false;
+            for (uint64_t c = a0 / Ro.chunk_bytes; c * Ro.chunk_bytes < a1 && !tpush; ++c)
+                tpush = proact::transfers(lc, Ro, (uint32_t)c);
+        }
         auto rows = [&](auto fast_tag) {
             constexpr bool FAST = decltype(fast_tag)::value;
             for (int i = T.i0; i < T.i1; ++i) {
@@ -339,7 +366,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                 const bool has_dn = i + 1 <= T.klast;
                 const int orow = (i - T.i0) % JSR;              // MODE 2: row within the span
                 float *ostrip = oring + ((oq % JOS) * JSR + orow) * JW;
-                if (MODE == 2 && orow == 0) proact::tp_acquire(tp, oq);
+                if (MODE == 2 && tpush && orow == 0) proact::tp_acquire(tp, oq);
                 if (has_dn) {
                     mbar_wait(&full[q % JS], (q / JS) & 1u);
     #pragma unroll
@@ -370,7 +397,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     }
                     const uint64_t off = ((uint64_t)i * N + j) * 4;
                     if (MODE == 2) {   // the local copy now, the span for the transfer warp
-                        *reinterpret_cast<float4 *>(ostrip + 4 * tid + g * GW) = o;
+                        if (tpush) *reinterpret_cast<float4 *>(ostrip + 4 * tid + g * GW) = o;
                         *reinterpret_cast<float4 *>(outb + off) = o;
                     } else if (!FAST && lc.mech == PROACT_MECH_INLINE) {
                         proact::put(lc, p.region_out, off, o);
@@ -383,7 +410,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     }
                 }
                 }
-                if (MODE == 2 && (orow == JSR - 1 || i + 1 == T.i1)) {   // hand the span to the transfer warp
+                if (MODE == 2 && tpush && (orow == JSR - 1 || i + 1 == T.i1)) {   // hand the span to the transfer warp
                     if (tid == 0)
                         tp->desc[oq % JOS] = proact::tile_desc{((uint64_t)(i - orow) * N + T.c0) * 4,
                                                                (uint32_t)(T.c1 - T.c0) * 4, proact::td_rows(orow + 1)};

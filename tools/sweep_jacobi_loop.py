@@ -23,6 +23,7 @@ from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl  # noqa: E402
 G = int(os.environ.get("G", 2))
 N = int(os.environ.get("N", 16384))
 HALO = os.environ.get("HALO", "0") == "1"
+NODEST = os.environ.get("HALO", "0") == "2"   # diagnostics: every chunk bound nowhere
 chunks = [int(x) for x in os.environ.get("CHUNKS", "131072").split(",")]
 mechs = os.environ.get("MECHS", "fused,dma,bulk,inline").split(",")
 warps = [int(x) for x in os.environ.get("WARPS", "16").split(",")]
@@ -35,6 +36,10 @@ x0 = synth.jacobi_init(N)
 
 def body(r, G_):
     J = wl.Jacobi(N, chunks[0], x0=torch.from_numpy(x0).cuda(), halo_only=HALO, rows_per_tile=RPT)
+    if NODEST:
+        for rid in J.rid:
+            for c in range(rt.region_info(rid).n_own_chunks):
+                rt.set_chunk_dest(rid, c, 0)
     s = torch.cuda.Stream()
     out = []
     for ch in chunks:
