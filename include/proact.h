@@ -116,8 +116,12 @@ enum {
 
 /* ---- proact_launch_ex flags ------------------------------------------------------------- */
 enum {
-    PROACT_LAUNCH_TILE_PUSH = 1  /* the kernel implements proact::tile_pusher (a transfer warp that
+    PROACT_LAUNCH_TILE_PUSH = 1, /* the kernel implements proact::tile_pusher (a transfer warp that
                                     pushes its own tiles) and may run under PROACT_AGENT_PRODUCER */
+    PROACT_LAUNCH_CLUSTER_SHIFT = 8 /* bits 8..11: thread-block cluster size (2, 4 or 8; 0/1 = none)
+                                    of the producer grid; the grid is a whole number of clusters
+                                    sized by cudaOccupancyMaxActiveClusters.  Not with agent CTAs in
+                                    the producer grid (PROACT_AGENT_FUSED): INVALID */
 };
 
 /* ---- phase synchronisation modes (a8) ----------------------------------------------------- */

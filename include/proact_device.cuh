@@ -110,8 +110,6 @@ struct launch_ctx {
     uint32_t piece_bytes;                      /* agent work unit */
     uint16_t discovery;                        /* PROACT_DISCOVER_* */
     uint16_t flags;                            /* LCF_* */
-    uint32_t qunits[PROACT_MAX_REGIONS];       /* QUEUE: units the producers enqueue this generation
-                                                  (pieces of the chunks that have destinations) */
 };
 
 /* launch_ctx::flags */
@@ -350,9 +348,6 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
         // this generation) and counts the chunk into its group with system-scope release
         R.counter[c] = 0u;
         asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(R.group_cnt + c / R.dma_group) : "memory");
-    } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA &&
-               !transfers(lc, R, c)) {
-        publish_chunk(lc, r, c);   // nothing to push (per-chunk destinations): no agent round trip
     } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA) {
         const uint32_t piece = piece_size(lc, R);
         const uint32_t P = (R.chunk_bytes + piece - 1) / piece;

@@ -115,8 +115,44 @@ constexpr int MAXGRAPH = 4;
 // 1024-thread CTAs per SM: one CTA with the 45056-entry table halves the warps in flight and runs
 // 2.4x slower (the gathers are latency-bound, tools/sweep_pagerank.py).
 constexpr uint32_t HOT_BIT = 0x80000000u;
-constexpr uint32_t HOT_MAX = 45056;   // 176 KiB table + 4 item groups x 12 KiB <= 227 KiB per CTA
-constexpr uint32_t HOT_DEFAULT = 8192;
+constexpr uint32_t HOT_MAX = 65536;   // 16-bit slots; above HOT_SLICE the table spans a cluster
+constexpr uint32_t HOT_SLICE = 8192;  // entries one CTA holds (32 KiB; 2 CTAs of 1024 threads per SM)
+constexpr uint32_t HOT_SHIFT = 13;
+#ifndef PROACT_GRAPH_HOT_DEFAULT
+#define PROACT_GRAPH_HOT_DEFAULT 8192
+#endif
+constexpr uint32_t HOT_DEFAULT = PROACT_GRAPH_HOT_DEFAULT;
+
+// Hot tables larger than one CTA's slice live in the distributed shared memory of a thread-block
+// cluster (CL CTAs): CTA rank q of the cluster stages slots [q * HOT_SLICE, (q + 1) * HOT_SLICE)
+// and a lookup of slot s reads CTA (s >> HOT_SHIFT)'s slice -- its own shared memory, or a peer's
+// through DSMEM (mapa + ld.shared::cluster).  A lookup that leaves the SM goes over the cluster's
+// SM-to-SM network instead of the L1 -> L2 request path the remaining gathers saturate, and the
+// table covers (RMAT-24) 30 % of the in-edges at 2 CTAs, 37 % at 4, 48 % at 8 instead of 22 %.
+__device__ __forceinline__ uint32_t cluster_rank()
+{
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+template <int CL, class T>
+__device__ __forceinline__ T hot_lookup(const T *hot, uint32_t hot_s, uint32_t my, uint32_t s)
+{
+    if (CL == 1) return hot[s];
+    const uint32_t o = s >> HOT_SHIFT, li = s & (HOT_SLICE - 1u);
+    if (o == my) return hot[li];
+    uint32_t ra;
+    asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(hot_s + 4u * li), "r"(o));
+    uint32_t v;
+    asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(ra) : "memory");
+    T out;
+    memcpy(&out, &v, 4);
+    return out;
+}
 #ifndef PROACT_PRH_PG
 #define PROACT_PRH_PG 4
 #endif
@@ -566,6 +602,7 @@ __device__ __forceinline__ uint32_t claim_group(const launch_ctx &lc, uint32_t n
     return t;
 }
 
+template <int CL>
 __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(launch_ctx lc, PrParams p)
 {
     constexpr int RUN = PROACT_PRH_RUN;
@@ -590,8 +627,15 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         nout = 0u;
     }
     __syncthreads();
-    for (uint32_t s = threadIdx.x; s < p.g.nhot; s += blockDim.x) hot[s] = ld_gather_f(cin + __ldg(p.g.hot_ids + s), pl);
+    const uint32_t my = CL > 1 ? cluster_rank() : 0u;
+    const uint32_t hot_s = (uint32_t)__cvta_generic_to_shared(hot);
+    {   // my slice of the hot table (all of it without a cluster)
+        const uint32_t s0 = my * HOT_SLICE;
+        const uint32_t ns = CL == 1 ? p.g.nhot : (p.g.nhot > s0 ? min(HOT_SLICE, p.g.nhot - s0) : 0u);
+        for (uint32_t s = threadIdx.x; s < ns; s += blockDim.x) hot[s] = ld_gather_f(cin + __ldg(p.g.hot_ids + s0 + s), pl);
+    }
     __syncthreads();
+    if (CL > 1) cluster_sync_all();   // every slice staged before any peer reads it
     const uint32_t lane = t & 31u;
 #if PROACT_PRH_SEGRED
     const uint32_t lrun = t;   // natural order: a warp's lanes hold 32 consecutive runs
@@ -668,7 +712,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     const bool h = x[q] & HOT_BIT;
-                    g[q] = h ? hot[x[q] & ~HOT_BIT & 0xFFFFu] : 0.f;
+                    g[q] = h ? hot_lookup<CL>(hot, hot_s, my, x[q] & ~HOT_BIT & 0xFFFFu) : 0.f;
                     if (!h) g[q] = ld_gather_f(cin + x[q], pl);
                 }
                 uint32_t nxt = cp[i + 1];
@@ -730,7 +774,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) {
                     const bool h = x[q] & HOT_BIT;
-                    g[q] = h ? hot[x[q] & ~HOT_BIT & 0xFFFFu] : 0.f;
+                    g[q] = h ? hot_lookup<CL>(hot, hot_s, my, x[q] & ~HOT_BIT & 0xFFFFu) : 0.f;
                     if (!h) g[q] = ld_gather_f(cin + x[q], pl);
                 }
                 uint32_t nxt = cp[i + 1];
@@ -790,6 +834,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         }
         grp_bar(grp);
     }
+    if (CL > 1) cluster_sync_all();   // my slice stays readable until every peer is done
 }
 
 constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
@@ -937,6 +982,7 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
 // ---- SSSP with the hot-source table and the pipelined index stream (as pagerank_hot_kernel).
 // hot[s] = d[hot_ids[s]] if that source's chunk changed in the previous round (or first round),
 // else INT32_MAX, so a hot in-edge needs neither the bitmap test nor the global gather.
+template <int CL>
 __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(launch_ctx lc, SsspParams p)
 {
 #if PROACT_SSH_VEC
@@ -987,11 +1033,18 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         }
     }
     __syncthreads();
-    for (uint32_t s = threadIdx.x; s < p.g.nhot; s += blockDim.x) {
-        const uint32_t u = __ldg(p.g.hot_ids + s);
-        hot[s] = changed_src(u) ? ld_gather_i(din + u, pl) : INT32_MAX;
+    const uint32_t my = CL > 1 ? cluster_rank() : 0u;
+    const uint32_t hot_s = (uint32_t)__cvta_generic_to_shared(hot);
+    {   // my slice of the hot table (all of it without a cluster)
+        const uint32_t s0 = my * HOT_SLICE;
+        const uint32_t ns = CL == 1 ? p.g.nhot : (p.g.nhot > s0 ? min(HOT_SLICE, p.g.nhot - s0) : 0u);
+        for (uint32_t s = threadIdx.x; s < ns; s += blockDim.x) {
+            const uint32_t u = __ldg(p.g.hot_ids + s0 + s);
+            hot[s] = changed_src(u) ? ld_gather_i(din + u, pl) : INT32_MAX;
+        }
     }
     __syncthreads();
+    if (CL > 1) cluster_sync_all();
     const uint32_t lane = t & 31u;
     const uint32_t lrun = (t & ~31u) + ((lane & 3u) << 3) + (lane >> 2);   // as in sssp_kernel
     for (;;) {
@@ -1049,7 +1102,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
                 for (int q = 0; q < RUN; ++q) {
                     int32_t du = INT32_MAX;
                     if (r0 + q < r1 && r0 + q >= it.e0) {
-                        if (x[q] & HOT_BIT) du = hot[x[q] & ~HOT_BIT & 0xFFFFu];
+                        if (x[q] & HOT_BIT) du = hot_lookup<CL>(hot, hot_s, my, x[q] & ~HOT_BIT & 0xFFFFu);
                         else if (changed_src(x[q])) du = ld_gather_i(din + x[q], pl);
                     }
                     c[q] = du;
@@ -1150,6 +1203,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         }
         grp_bar(grp);
     }
+    if (CL > 1) cluster_sync_all();   // my slice stays readable until every peer is done
 }
 
 __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t V, float r0)
@@ -1161,6 +1215,7 @@ __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t 
 }  // namespace
 extern "C" __attribute__((visibility("hidden"))) void proact_internal_l2_window(const void *base, size_t bytes);
 extern "C" __attribute__((visibility("hidden"))) void proact_internal_keep_l1(const void *kernel);
+extern "C" __attribute__((visibility("hidden"))) int proact_internal_smem_attr(const void *kernel, size_t bytes);
 namespace {
 
 // PROACT_L2_WINDOW=1: mark the gathered replica persisting in L2 for the phase launch
@@ -1171,6 +1226,21 @@ int l2_window_on()
         return e ? atoi(e) : 0;
     }();
     return on;
+}
+
+// Cluster size of the hot-table kernels for a table of nhot entries: 0 = no table (plain kernels),
+// 1 = one CTA holds it all (nhot <= HOT_SLICE), else the power of two of CTAs whose slices cover
+// it.  A cluster kernel cannot share its grid with fused agent CTAs (PROACT_AGENT_FUSED while the
+// launch tallies): then the plain kernels run (same results: the sums are exact).
+int hot_cluster(uint32_t nhot)
+{
+    if (!nhot) return 0;
+    if (nhot <= HOT_SLICE) return 1;
+    int cl = 2;
+    while ((uint32_t)cl * HOT_SLICE < nhot) cl *= 2;
+    proact_config c;
+    if (proact_get_config(&c) == PROACT_OK && c.agent_kernel == PROACT_AGENT_FUSED && proact_launch_tallies()) return 0;
+    return cl;
 }
 
 int graph_dev(int id, GraphDev *g)
@@ -1378,13 +1448,26 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
         }
     }
     GCK(cudaStreamSynchronize(s));
-    GCK(cudaFuncSetAttribute((const void *)pagerank_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)(4 * (PG * CPS + HOT_MAX))));
-    for (const void *k : {(const void *)pagerank_hot_kernel, (const void *)pagerank_kernel,
-                          (const void *)sssp_hot_kernel, (const void *)sssp_kernel})
-        proact_internal_keep_l1(k);
-    GCK(cudaFuncSetAttribute((const void *)sssp_hot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)(4 * (PG * CPS + HOT_MAX)) - (int)(4 * CHG_WORDS)));
+    {
+        // the opt-in stays at the round-1 value (a 45056-entry table): besides allowing the launch,
+        // it steers the driver's default shared-memory carve-out for these kernels (they keep the
+        // default, proact_internal_keep_l1) -- with a smaller opt-in the SMs they run on are
+        // configured with less shared memory, so a separate agent (200 KiB) cannot be placed next
+        // to them and 4 loopback ranks' agents no longer find SMs (observed: start-up timeout)
+        const size_t b = 4 * ((size_t)PG * CPS + 45056);
+        const void *pr[] = {(const void *)pagerank_hot_kernel<1>, (const void *)pagerank_hot_kernel<2>,
+                            (const void *)pagerank_hot_kernel<4>, (const void *)pagerank_hot_kernel<8>};
+        const void *ss[] = {(const void *)sssp_hot_kernel<1>, (const void *)sssp_hot_kernel<2>,
+                            (const void *)sssp_hot_kernel<4>, (const void *)sssp_hot_kernel<8>};
+        for (int k = 0; k < 4; ++k) {
+            if (proact_internal_smem_attr(pr[k], b) || proact_internal_smem_attr(ss[k], b - 4 * CHG_WORDS))
+                return PROACT_ERR_CUDA;
+            proact_internal_keep_l1(pr[k]);
+            proact_internal_keep_l1(ss[k]);
+        }
+        proact_internal_keep_l1((const void *)pagerank_kernel);
+        proact_internal_keep_l1((const void *)sssp_kernel);
+    }
     G.used = true;
     graphs[id] = G;
     return id;
@@ -1470,9 +1553,14 @@ int proact_pagerank_phase(int graph, int region_in, int region_out, double dampi
         if (proact_region_info_get(region_in, &ri) == PROACT_OK)
             proact_internal_l2_window(ri.replica_base, ri.total_bytes);
     }
-    if (!plain)
-        return proact_launch(regs, 1, (const void *)pagerank_hot_kernel, 0, GB * PG, args,
-                             4 * ((size_t)PG * CPS + p.g.nhot), stream);
+    const int cl = hot_cluster(p.g.nhot);
+    if (!plain && cl > 0) {
+        const void *k = cl == 1 ? (const void *)pagerank_hot_kernel<1>
+                      : cl == 2 ? (const void *)pagerank_hot_kernel<2>
+                      : cl == 4 ? (const void *)pagerank_hot_kernel<4> : (const void *)pagerank_hot_kernel<8>;
+        return proact_launch_ex(regs, 1, k, 0, GB * PG, args, 4 * ((size_t)PG * CPS + (cl == 1 ? p.g.nhot : HOT_SLICE)),
+                                stream, cl > 1 ? (unsigned)cl << PROACT_LAUNCH_CLUSTER_SHIFT : 0u);
+    }
     return proact_launch(regs, 1, (const void *)pagerank_kernel, 0, GB, args, 0, stream);
 }
 
@@ -1510,9 +1598,14 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
         if (proact_region_info_get(region_in, &ri) == PROACT_OK)
             proact_internal_l2_window(ri.replica_base, ri.total_bytes);
     }
-    if (p.g.nhot && p.g.nhot <= HOT_MAX - CHG_WORDS)   // hot table (room for the changed bitmap)
-        return proact_launch(regs, 1, (const void *)sssp_hot_kernel, 0, GB * PG, args,
-                             4 * ((size_t)PG * CPS + p.g.nhot), stream);
+    const int cl = hot_cluster(p.g.nhot);
+    if (cl > 0) {
+        const void *k = cl == 1 ? (const void *)sssp_hot_kernel<1>
+                      : cl == 2 ? (const void *)sssp_hot_kernel<2>
+                      : cl == 4 ? (const void *)sssp_hot_kernel<4> : (const void *)sssp_hot_kernel<8>;
+        return proact_launch_ex(regs, 1, k, 0, GB * PG, args, 4 * ((size_t)PG * CPS + (cl == 1 ? p.g.nhot : HOT_SLICE)),
+                                stream, cl > 1 ? (unsigned)cl << PROACT_LAUNCH_CLUSTER_SHIFT : 0u);
+    }
     return proact_launch(regs, 1, (const void *)sssp_kernel, 0, GB, args, 0, stream);
 }
 
@@ -1523,8 +1616,11 @@ __attribute__((visibility("hidden"))) int proact_internal_preload_graph(void)
     const void *k[] = {(const void *)count_kernel, (const void *)scan_blocks, (const void *)scan_totals,
                        (const void *)scan_add, (const void *)scatter_kernel, (const void *)pagerank_kernel,
                        (const void *)sssp_kernel, (const void *)pr_init_kernel, (const void *)runv_kernel,
-                       (const void *)pagerank_hot_kernel, (const void *)hot_slot_kernel,
-                       (const void *)hot_encode_kernel, (const void *)sssp_hot_kernel};
+                       (const void *)pagerank_hot_kernel<1>, (const void *)pagerank_hot_kernel<2>,
+                       (const void *)pagerank_hot_kernel<4>, (const void *)pagerank_hot_kernel<8>,
+                       (const void *)hot_slot_kernel, (const void *)hot_encode_kernel,
+                       (const void *)sssp_hot_kernel<1>, (const void *)sssp_hot_kernel<2>,
+                       (const void *)sssp_hot_kernel<4>, (const void *)sssp_hot_kernel<8>};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
     return PROACT_OK;

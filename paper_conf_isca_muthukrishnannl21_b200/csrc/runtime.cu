@@ -158,8 +158,6 @@ struct Region {
     // MECH_DMA: the per-phase copy-engine program (wait group counter -> copy per destination ->
     // reset), built once per geometry and replayed as a CUDA graph (NEXT-3, L166)
     cudaGraphExec_t dma_exec = nullptr;
-    uint32_t qunits = 0, qunits_piece = 0;   // cached queue units per generation for a piece size
-    bool qunits_elide = false;
     uint32_t dma_group = 1;
     uint32_t dma_peers = 0;           // destinations the program copies to
 };
@@ -411,7 +409,7 @@ int build_region_tables(RankCtx *c, int id, Region &R, RegionExchange &ex) {
         if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }
     }
     D.dma_group = R.dma_group;
-    R.qunits_piece = 0;
+
     D.group_cnt = (uint32_t *)(R.meta + off_group);
     D.chunk_dest = nullptr;
     R.chunk_dest.clear();
@@ -983,7 +981,6 @@ int proact_region_set_chunk_dest(int id, uint32_t chunk, uint64_t mask)
     }
     R.chunk_dest[chunk] = (uint32_t)mask;
     if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }   // new geometry
-    R.qunits_piece = 0;
     CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * (size_t)R.n_own, cudaMemcpyHostToDevice));
     return PROACT_OK;
 }
@@ -1146,10 +1143,11 @@ thread_local const void *g_l2_base = nullptr;
 thread_local size_t g_l2_bytes = 0;
 
 cudaError_t launch_producer(const void *kernel, unsigned total, unsigned block, void **args, size_t smem,
-                            cudaStream_t s, int device, const void *l2_base, size_t l2_bytes, bool pdl = false)
+                            cudaStream_t s, int device, const void *l2_base, size_t l2_bytes, bool pdl = false,
+                            unsigned cluster = 1)
 {
     const bool window = l2_base && l2_bytes;
-    if (!window && !pdl) return cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s);
+    if (!window && !pdl && cluster <= 1) return cudaLaunchKernel(kernel, dim3(total), dim3(block), args, smem, s);
     static thread_local int limit_dev = -1;
     static thread_local size_t limit = 0;
     if (window && limit_dev != device) {   // reserve the persisting L2 set-aside once per device
@@ -1165,8 +1163,15 @@ cudaError_t launch_producer(const void *kernel, unsigned total, unsigned block, 
     cfg.blockDim = dim3(block);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = s;
-    cudaLaunchAttribute at[2];
+    cudaLaunchAttribute at[3];
     unsigned n = 0;
+    if (cluster > 1) {
+        at[n].id = cudaLaunchAttributeClusterDimension;
+        at[n].val.clusterDim.x = cluster;
+        at[n].val.clusterDim.y = 1;
+        at[n].val.clusterDim.z = 1;
+        ++n;
+    }
     if (window && limit) {
         at[n].id = cudaLaunchAttributeAccessPolicyWindow;
         at[n].val.accessPolicyWindow.base_ptr = const_cast<void *>(l2_base);
@@ -1237,25 +1242,6 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     for (int r = 0; r < c->nregions; ++r) {
         Region &R = c->regions[r];
         lc.gen[r] = (armed >> r & 1) ? R.gen_done + 1 : R.gen_done;
-        if (armed >> r & 1) {   // QUEUE: units the committers will enqueue (chunks with destinations)
-            const uint32_t piece = std::min<uint32_t>(cfg.piece_bytes, (uint32_t)R.chunk);
-            const bool elide = lc.mech == PROACT_MECH_ELIDE;   // every chunk takes part (proact::transfers)
-            if (R.qunits_piece != piece || R.qunits_elide != elide) {
-                uint32_t u = 0;
-                const uint32_t self = 1u << c->rank;
-                for (uint32_t k = 0; k < R.n_own; ++k) {
-                    const uint32_t m = (R.chunk_dest.empty() ? (uint32_t)R.dest_mask : R.chunk_dest[k]) & ~self &
-                                       (c->world < 32 ? (1u << c->world) - 1u : ~0u);
-                    if (!m && !elide) continue;
-                    const uint64_t len = std::min<uint64_t>(R.chunk, R.own_bytes - (uint64_t)k * R.chunk);
-                    u += (uint32_t)((len + piece - 1) / piece);
-                }
-                R.qunits = u;
-                R.qunits_piece = piece;
-                R.qunits_elide = elide;
-            }
-            lc.qunits[r] = R.qunits;
-        }
         lc.gen_epoch[r] = (armed >> r & 1) ? c->epoch : R.gen_epoch;
         lc.gen_mech[r] = (armed >> r & 1) ? (uint8_t)lc.mech : R.gen_mech;
     }
@@ -1281,26 +1267,51 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     // at most half of this rank's share of the SMs hosts agent CTAs: beyond that the producer
     // starves (loopback G = 2, 96 agent warps: 7.8 ms per microbenchmark phase instead of 0.76,
     // tools/sweep_micro.py; one rank, 128 idle agent warps: 2x the producer time)
-    const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / (2u * (unsigned)std::max(1, c->ranks_on_device)));
+    // (ranks sharing a device -- loopback -- get half of that again: several ranks' agents must find
+    // room next to each other's persistent producer grids)
+    const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / ((c->ranks_on_device > 1 ? 4u : 2u) *
+                                                                (unsigned)std::max(1, c->ranks_on_device)));
     agent_ctas = std::min(agent_ctas, agent_cap);
     if (agent && !separate && cfg.push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
     lc.agent_warps = (uint16_t)(agent ? std::min<unsigned>(cfg.agent_warps, agent_ctas * wpc) : 0);
     int nb = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
     if (nb < 1) return PROACT_ERR_INVALID;
-    // a rank's share of the co-resident capacity; ranks sharing a device (loopback) leave a tenth of
+    // thread-block clusters (DSMEM users): whole clusters, capacity from the cluster occupancy
+    const unsigned cluster = std::max(1u, (flags >> PROACT_LAUNCH_CLUSTER_SHIFT) & 15u);
+    int ncl = 0;
+    if (cluster > 1) {
+        if (agent && cfg.agent_kernel == PROACT_AGENT_FUSED) return PROACT_ERR_INVALID;
+        cudaLaunchConfig_t oc = {};
+        oc.gridDim = dim3(cluster * 1024);
+        oc.blockDim = dim3(block);
+        oc.dynamicSmemBytes = smem;
+        cudaLaunchAttribute ca;
+        ca.id = cudaLaunchAttributeClusterDimension;
+        ca.val.clusterDim.x = cluster;
+        ca.val.clusterDim.y = 1;
+        ca.val.clusterDim.z = 1;
+        oc.attrs = &ca;
+        oc.numAttrs = 1;
+        CK(cudaOccupancyMaxActiveClusters(&ncl, kernel, &oc));
+        if (ncl < 1) return PROACT_ERR_INVALID;
+    }
+    // a rank's share of the co-resident capacity; ranks sharing a device (loopback) leave 15 % of
     // it free, so that every rank's sync / helper kernels and separate agent always find slots even
     // while the other ranks' persistent producers spin in their arrival waits
     const int rod = std::max(1, c->ranks_on_device);
-    unsigned cap = (unsigned)std::max(1, rod > 1 ? nb * c->nsm * 9 / (10 * rod) : nb * c->nsm);
+    unsigned cap = (unsigned)std::max(1, rod > 1 ? nb * c->nsm * 17 / (20 * rod) : nb * c->nsm);
+    if (cluster > 1)   // whole clusters (at least one)
+        cap = cluster * (unsigned)std::max(1, rod > 1 ? ncl * 17 / (20 * rod) : ncl);
     if (cfg.grid_cap > 0) cap = std::min(cap, (unsigned)cfg.grid_cap);
     cudaStream_t s = (cudaStream_t)stream;
     if (after) {
         lc.agent_ctas = 0;
         unsigned total = grid ? grid : cap;
         if (total > cap) total = cap;
+        if (cluster > 1) total = std::max(cluster, total / cluster * cluster);
         *(launch_ctx *)args[0] = lc;
-        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, false, cluster));
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
         const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
@@ -1326,7 +1337,11 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
         la.flags |= proact::LCF_SEPARATE;
-        size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+        // ranks sharing a device (loopback) use the small ring: an agent CTA that needs a whole SM's
+        // shared memory can find no SM once several ranks' persistent grids are spread over the
+        // device (observed with 4 ranks x 16 agent CTAs: the agent never becomes resident)
+        size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0
+                       : (agent_ctas > 32 || c->ranks_on_device > 1 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
             asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
         agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
@@ -1357,8 +1372,9 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         unsigned total = grid ? grid : cap;
         const unsigned reserve = std::min(cap - 1, agent_ctas * lost);
         if (total + reserve > cap) total = cap - reserve;
+        if (cluster > 1) total = std::max(cluster, total / cluster * cluster);
         *(launch_ctx *)args[0] = lc;
-        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, true));
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, true, cluster));
     } else if (lc.mech == PROACT_MECH_DMA && armed) {
         // NEXT-3 "hardware PROACT": the copy engines are the transfer agent.  Per region, a
         // program prepared once (the paper's "descriptors for the geometry of each transfer
@@ -1382,7 +1398,8 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         // can buffer, and enqueueing them must never block the launch that satisfies them
         unsigned total = grid ? grid : cap;
         if (total > cap) total = cap;
-        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
+        if (cluster > 1) total = std::max(cluster, total / cluster * cluster);
+        CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, false, cluster));
         cudaStream_t d0 = c->dma[0];
         CK(cudaStreamWaitEvent(d0, c->ev_start, 0));
         for (int r = 0; r < c->nregions; ++r) {
@@ -1423,11 +1440,12 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         unsigned total = agent_ctas + (grid ? grid : cap);
         if (total > cap) total = cap;
         if (total <= agent_ctas) return PROACT_ERR_INVALID;
+        if (cluster > 1) total = std::max(cluster, total / cluster * cluster);
         *(launch_ctx *)args[0] = lc;
         if (c->coop && agent)
             CK(cudaLaunchCooperativeKernel(kernel, dim3(total), dim3(block), args, smem, s));
         else
-            CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n));
+            CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, false, cluster));
     }
     for (int r = 0; r < c->nregions; ++r) {
         if (!(armed >> r & 1)) continue;

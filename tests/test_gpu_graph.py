@@ -61,9 +61,28 @@ def test_pagerank_hot_table_is_bit_identical():
     sums: r' is bit-identical with no table, a partial table and the default table."""
     src, dst = synth.rmat(16, 16)
     V = 1 << 16
-    got = [run_ranks(1, _pr_body, V, src, dst, 5, 4096, _lib.MECH_FUSED, hot)[0][2] for hot in (0, 333, -1)]
-    assert np.array_equal(got[0].view(np.uint32), got[1].view(np.uint32))
-    assert np.array_equal(got[0].view(np.uint32), got[2].view(np.uint32))
+    hots = (0, 333, -1, 12000, 30000, 65536)   # 12000 / 30000 / 65536: DSMEM tables of 2 / 4 / 8 CTAs
+    got = [run_ranks(1, _pr_body, V, src, dst, 5, 4096, _lib.MECH_FUSED, hot)[0][2] for hot in hots]
+    for k in range(1, len(hots)):
+        assert np.array_equal(got[0].view(np.uint32), got[k].view(np.uint32)), hots[k]
+
+
+@pytest.mark.parametrize("G,hot", [(1, 12000), (2, 30000), (3, 65536)])
+def test_cluster_hot_tables_match_oracle(G, hot):
+    """Hot tables spread over thread-block clusters (DSMEM): PageRank within 1e-5 and SSSP
+    bit-exact against the oracle, multi-rank included (separate agent next to cluster grids)."""
+    src, dst = synth.rmat(16, 16)
+    V = 1 << 16
+    want = oracle.pagerank(V, src, dst, 10).astype(np.float64)
+    got = np.zeros(V)
+    for v0, v1, r in run_ranks(G, _pr_body, V, src, dst, 10, 16384, _lib.MECH_FUSED, hot):
+        got[v0:v1] = r
+    assert (np.abs(got - want) / want).max() <= 1e-5
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    want_d, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
+    for rounds, d, _, _ in run_ranks(G, _sssp_body, V, src, dst, w, s0, 16384, _lib.MECH_FUSED, hot):
+        assert rounds == want_rounds and np.array_equal(d, want_d)
 
 
 def _sssp_body(r, G, V, src, dst, w, s0, chunk, mech, hot=-1):
