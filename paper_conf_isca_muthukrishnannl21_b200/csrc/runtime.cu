@@ -1267,9 +1267,9 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     // at most half of this rank's share of the SMs hosts agent CTAs: beyond that the producer
     // starves (loopback G = 2, 96 agent warps: 7.8 ms per microbenchmark phase instead of 0.76,
     // tools/sweep_micro.py; one rank, 128 idle agent warps: 2x the producer time)
-    // (ranks sharing a device -- loopback -- get half of that again: several ranks' agents must find
-    // room next to each other's persistent producer grids)
-    const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / ((c->ranks_on_device > 1 ? 4u : 2u) *
+    // (three or more ranks sharing a device -- loopback -- get half of that again: several ranks'
+    // agents must find room next to each other's persistent producer grids)
+    const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / ((c->ranks_on_device > 2 ? 4u : 2u) *
                                                                 (unsigned)std::max(1, c->ranks_on_device)));
     agent_ctas = std::min(agent_ctas, agent_cap);
     if (agent && !separate && cfg.push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
@@ -1337,11 +1337,11 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
         la.flags |= proact::LCF_SEPARATE;
-        // ranks sharing a device (loopback) use the small ring: an agent CTA that needs a whole SM's
+        // three or more ranks sharing a device (loopback) use the small ring: an agent CTA that needs a whole SM's
         // shared memory can find no SM once several ranks' persistent grids are spread over the
         // device (observed with 4 ranks x 16 agent CTAs: the agent never becomes resident)
         size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0
-                       : (agent_ctas > 32 || c->ranks_on_device > 1 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+                       : (agent_ctas > 32 || c->ranks_on_device > 2 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
             asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
         agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
