@@ -563,7 +563,9 @@ def main():
         # the pipelined entry point: K solves (steps), each with its own H2D of the input and D2H
         # of its result inside the timed region, solve k's phases overlapping the copies of k +- 1
         outs = [out, torch.empty((N, N), dtype=torch.float32).pin_memory()]
-        K = max(4, min(args.steps, 8))
+        # a stream of K solves: the first H2D and the last D2H (each ~19 ms over PCIe, measured
+        # full duplex by tools/probes/pcie_duplex.py) cannot overlap compute; K amortises them
+        K = max(4, min(2 * args.steps, 20))
 
         def e2e_pipe(k):
             h, d = wl.jacobi_solve_host_pipelined(xh, [outs[j & 1] for j in range(k)], N, I, chunk, args.rpt, s)
