@@ -91,15 +91,20 @@ __device__ __forceinline__ bool tp_mbar_test(uint64_t *b, uint32_t parity)
                  : "=r"(done) : "r"(tp_smem(b)), "r"(parity) : "memory");
     return done != 0;
 }
-// Wait up to PROACT_TP_IDLE_NS for the phase, sleeping between tests (a waiting transfer warp must
-// not take issue slots from the compute warps of its SM): true if the phase completed.
+// Wait up to (about) PROACT_TP_IDLE_NS for the phase: suspending try_waits (the hardware wakes
+// the thread when the phase completes, so a waiting transfer warp takes no issue slots from the
+// compute warps and reacts at once), the elapsed time checked between them.  True if completed.
 __device__ __forceinline__ bool tp_mbar_try(uint64_t *b, uint32_t parity)
 {
     if (tp_mbar_test(b, parity)) return true;
     const uint64_t t0 = globaltimer();
     do {
-        __nanosleep(500);
-        if (tp_mbar_test(b, parity)) return true;
+        uint32_t done;
+        asm volatile("{\n\t.reg .pred p;\n\t"
+                     "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+                     "selp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(done) : "r"(tp_smem(b)), "r"(parity), "n"(1000) : "memory");
+        if (done) return true;
     } while (globaltimer() - t0 < PROACT_TP_IDLE_NS);
     return false;
 }
