@@ -504,6 +504,31 @@ def main():
         mode["nccl"] = nccl_base
         rt.set_config(mech=mech)
 
+    # ---- NEXT-1, the paper's decomposition (Sec. V-C; Fig. 8/9) on the same
+    # ranks: LOCAL = no transfer at all and no waits (the infinite-bandwidth bound; replicas go
+    # stale, timing only), ELIDE = tracking + agent without remote stores (tracking overhead), BULK
+    # = transfers after the kernel.  opportunity = T_bulk - T_local; captured = (T_bulk - T_proact)
+    # / opportunity; overlap = captured with the tracking overhead added back
+    decomposition = None
+    if world > 1 and not args.no_baselines and baselines and mech in (_lib.MECH_FUSED, _lib.MECH_ELIDE):
+        kk = max(2, args.steps // 2)
+        dv = {}
+        for name, m in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE)):
+            rt.set_config(mech=m)
+            step()
+            dv[name] = timed(step, kk) / (kk * I)   # ms per phase
+        rt.set_config(mech=mech)
+        t_p = ms / (args.steps * I)
+        t_b = 1000.0 / baselines["bulk_cudaMemcpyPeer"]
+        opp = t_b - dv["local"]
+        decomposition = {"ms_per_phase": {"proact": t_p, "bulk": t_b, "local_no_transfer": dv["local"],
+                                          "elide_tracking_only": dv["elide"]},
+                         "tracking_overhead_frac": dv["elide"] / dv["local"] - 1.0,
+                         "opportunity_ms": opp,
+                         "opportunity_captured": (t_b - t_p) / opp if opp > 0 else None,
+                         "overlap_frac": (t_b - t_p + dv["elide"] - dv["local"]) / opp if opp > 0 else None,
+                         "note": "paper Sec. V-C: infinite-BW bound = LOCAL, tracking overhead = ELIDE vs LOCAL"}
+
     # ---- halo-only variant (reading R8: the one config-2 variant whose roofline allows
     # >= 6x at G = 8): per-chunk destinations = the neighbours; PROACT (tuned) and the baselines
     halo = None
@@ -603,7 +628,7 @@ def main():
                                  "what": ("this run's timed step (G = 1)" if world == 1 else
                                           "uninstrumented single-GPU solve (LOCAL) of the full grid on every "
                                           "rank's GPU in this run, slowest rank")},
-                "halo_only": halo, "agent_cost": agent_cost}
+                "halo_only": halo, "agent_cost": agent_cost, "decomposition": decomposition}
         print(json.dumps(line), flush=True)
     torch.cuda.synchronize()
     J.free()

@@ -99,3 +99,6 @@ def test_bench_two_processes_json_line():
     assert h["value"] > 0 and h["speedup_vs_n1"] > 0 and h["step_roofline"]["frac"] > 0
     assert set(h["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
     assert d["agent_cost"]["agent_sm_ms_per_GB_pushed"] >= 0
+    dc = d["decomposition"]   # NEXT-1: infinite-bandwidth bound, tracking overhead, captured
+    assert dc["ms_per_phase"]["local_no_transfer"] > 0 and dc["ms_per_phase"]["elide_tracking_only"] > 0
+    assert "opportunity_captured" in dc
