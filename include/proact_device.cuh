@@ -114,9 +114,10 @@ struct launch_ctx {
 
 /* launch_ctx::flags */
 enum { LCF_SEPARATE = 1,   /* this is the SEPARATE agent kernel's copy (start-up deadline armed) */
-       LCF_TILE_PUSH = 2   /* PROACT_AGENT_PRODUCER: every producer CTA's transfer warp pushes its
+       LCF_TILE_PUSH = 2,  /* PROACT_AGENT_PRODUCER: every producer CTA's transfer warp pushes its
                               own tiles (proact::tile_pusher); counters count DELIVERED bytes and
                               the last contributor of a chunk publishes its arrival flags */
+       LCF_BULK_WARPS_SHIFT = 8   /* bits 8..11: issuing warps per BULK (TMA) agent CTA (0 = 1) */
 };
 
 /* error word encoding: (site << 8) | (-PROACT_ERR_*) */

@@ -1262,7 +1262,11 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     // VEC16: agent_warps warps packed into CTAs; BULK (TMA): one agent warp per CTA, which
     // uses the CTA's whole dynamic shared memory as its staging ring (>= PROACT_BULK_SMEM)
     const unsigned agent_block = separate ? 256u : block;
-    unsigned wpc = cfg.push == PROACT_PUSH_BULK ? 1 : agent_block / 32;
+    // TMA (BULK) agents: issuing warps per agent CTA, each with its slice of the CTA's staging
+    // memory (PROACT_AGENT_BULK_WARPS, default 1; separate agent kernel only)
+    static const unsigned bulk_w = (unsigned)std::min(8, std::max(1, env_int("PROACT_AGENT_BULK_WARPS", 1)));
+    const unsigned bw = separate && cfg.push == PROACT_PUSH_BULK ? bulk_w : 1u;
+    unsigned wpc = cfg.push == PROACT_PUSH_BULK ? bw : agent_block / 32;
     unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
     // at most half of this rank's share of the SMs hosts agent CTAs: beyond that the producer
     // starves (loopback G = 2, 96 agent warps: 7.8 ms per microbenchmark phase instead of 0.76,
@@ -1314,6 +1318,7 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, false, cluster));
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
+        la.flags |= (uint16_t)(bw << proact::LCF_BULK_WARPS_SHIFT);
         const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
         CK(cudaGetLastError());
@@ -1336,7 +1341,7 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         // The producer grid leaves room for the agent's CTAs (reserve below).
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
-        la.flags |= proact::LCF_SEPARATE;
+        la.flags |= proact::LCF_SEPARATE | (uint16_t)(bw << proact::LCF_BULK_WARPS_SHIFT);
         // three or more ranks sharing a device (loopback) use the small ring: an agent CTA that needs a whole SM's
         // shared memory can find no SM once several ranks' persistent grids are spread over the
         // device (observed with 4 ranks x 16 agent CTAs: the agent never becomes resident)
