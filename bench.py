@@ -15,7 +15,10 @@ CUDA events on its stream), cpu_baseline (the oracle, rank 0, bounded sample), e
 (proact_jacobi_solve_host with pinned host buffers: H2D of the grid + I phases + D2H),
 clocks (nvidia-smi sampled during the timed region), gpu_launches, overhead (the
 same step with the uninstrumented LOCAL mechanism: the paper's tracking-overhead
-decomposition, Sec. V-C).
+decomposition, Sec. V-C).  N = 1 also adds `secondary` (outside the timed
+region): config 2 on two loopback ranks of this GPU with every transfer mechanism (the
+PROACT path itself; at G = 1 nothing is replicated) and BASELINE.json configs 3-4
+(PageRank / SSSP, RMAT-24) with their rooflines and oracle baselines.
 
 --impl reference: the CPU oracle (oracle/) timed as it stands on the host cores, on
 the same config/metric; rank 0 only under torchrun.
@@ -215,6 +218,82 @@ def single_gpu_reference(N: int, I: int, rpt: int, steps: int = 2) -> float:
     return ms
 
 
+def _json_lines(cmd: list, env: dict, timeout: float) -> list:
+    """Run a helper (tools/) in its own process; its stdout JSON lines, or an error record."""
+    try:
+        r = subprocess.run(cmd, env=env, cwd=ROOT, capture_output=True, text=True, timeout=timeout)
+    except subprocess.TimeoutExpired:
+        return [{"error": f"timeout after {timeout:.0f}s"}]
+    out = []
+    for line in r.stdout.splitlines():
+        line = line.strip()
+        if line.startswith("{"):
+            try:
+                out.append(json.loads(line))
+            except ValueError:
+                pass
+    if r.returncode != 0 or not out:
+        out.append({"error": f"rc={r.returncode}: {r.stderr.strip().splitlines()[-1:] if r.stderr else ''}"})
+    return out
+
+
+def secondary_legs(N: int, peak: float) -> dict:
+    """N = 1 only, after the headline's context is finalised and its memory freed (nothing here is
+    inside the timed region).  At G = 1 nothing is replicated (reading R18), so the PROACT
+    transfer path is measured here on this one GPU the only way it can be: two ranks as threads
+    ("loopback") of config 2, every mechanism on the same ranks -- the replica
+    bytes cross HBM, not NVLink, so these rank the mechanisms on this box; they are not NVLink
+    numbers.  Also BASELINE.json configs 3 and 4 (PageRank / SSSP on RMAT-24) with their own
+    roofline and oracle baseline (tools/bench_workloads.py)."""
+    py = sys.executable
+    env = dict(os.environ)
+    env.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+    names = {("fused", 2): "proact_producer_tile_push", ("fused", 1): "proact_separate_agent",
+             ("fused", 0): "proact_agent_in_grid", ("elide", 2): "elide_tracking_only_tile_push",
+             ("elide", 1): "elide_tracking_only_separate_agent", ("inline", None): "naive_p2p_inline",
+             ("bulk", None): "bulk_cudaMemcpyPeer", ("dma", None): "dma_copy_engine_program",
+             ("local", None): "local_no_transfer"}
+    legs = {
+        "full": dict(HALO="0", CHUNKS="1048576", MECHS="fused,elide,inline,bulk,dma,local", AKERNS="2,1",
+                     PUSHES="1", WARPS="32"),
+        "halo_only": dict(HALO="1", CHUNKS="131072", MECHS="fused,inline,bulk,dma,local", AKERNS="1,2",
+                          PUSHES="0", WARPS="2"),
+    }
+    gib = float(1 << 30)
+    # loopback HBM floor per phase (whole device): both ranks' stencil traffic (8 B/cell of the
+    # grid) + the replicated half each rank writes into the other's replica (4 B/cell), full
+    # replication; halo-only adds two rows
+    floor_bytes = {"full": 8.0 * N * N + 4.0 * N * N, "halo_only": 8.0 * N * N + 2 * 4.0 * N}
+    out = {"note": ("G = 2 loopback ranks of config 2 on this one GPU (replica bytes cross HBM, not NVLink: "
+                    "mechanism ranking on this box, not an NVLink result); ms per phase, max over ranks, "
+                    "20 phases after 3 warm-up")}
+    for leg, kv in legs.items():
+        e = dict(env, G="2", N=str(N), PHASES="20", **kv)
+        pts = _json_lines([py, os.path.join(ROOT, "tools", "sweep_jacobi_loop.py")], e, 600)
+        ms = {}
+        for p in pts:
+            if "error" in p:
+                ms.setdefault("errors", []).append(p["error"])
+                continue
+            key = (p["mech"], p["akern"] if p["mech"] in ("fused", "elide") else None)
+            ms[names.get(key, f"{p['mech']}_{p['akern']}")] = p["ms"]
+        proact = {k: v for k, v in ms.items() if k.startswith("proact_")}
+        base = {k: ms[k] for k in ("naive_p2p_inline", "bulk_cudaMemcpyPeer", "dma_copy_engine_program") if k in ms}
+        best = min(proact, key=proact.get) if proact else None
+        out[leg] = {"ms_per_phase": ms, "chunk_bytes": int(kv["CHUNKS"]),
+                    "hbm_floor_ms": floor_bytes[leg] / (peak * 1e9) * 1e3,
+                    "best_proact": best,
+                    "best_proact_vs_baselines": ({k: v / proact[best] for k, v in base.items()} if best else None)}
+        if "local_no_transfer" in ms and "bulk_cudaMemcpyPeer" in ms and best:
+            opp = ms["bulk_cudaMemcpyPeer"] - ms["local_no_transfer"]
+            out[leg]["opportunity_captured"] = ((ms["bulk_cudaMemcpyPeer"] - proact[best]) / opp) if opp > 0 else None
+    for wk in ("pagerank", "sssp"):
+        pts = _json_lines([py, os.path.join(ROOT, "tools", "bench_workloads.py"), "--workload", wk,
+                           "--steps", "3", "--warmup", "1"], env, 900)
+        out[wk] = pts[0] if len(pts) == 1 else pts
+    return out
+
+
 def run_reference(args, dist_rank: int) -> None:
     if dist_rank != 0:
         return
@@ -268,6 +347,8 @@ def main():
                     help="process-group backend for the timing barrier / max-over-ranks only")
     ap.add_argument("--no-halo", action="store_true", help="N > 1: skip the halo-only legs")
     ap.add_argument("--no-n1", action="store_true", help="N > 1: skip the single-GPU reference (speedup)")
+    ap.add_argument("--no-secondary", action="store_true",
+                    help="N = 1: skip the loopback mechanism legs and the PageRank / SSSP configs")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -535,6 +616,37 @@ def main():
     if world > 1 and not args.no_halo:
         J.set_halo_only()
         kk = max(2, args.steps // 2)
+        # the halo exchange moves two rows per rank: the profiler picks again, over few agent warps
+        # (chunks bound nowhere never reach the agent) and the producer-CTA placement
+        full_cfg = rt.get_config()
+        halo_tuned = None
+        if tuned is not None:
+            def run_halo(c):
+                if c["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+                    for rid in J.rid:
+                        rt.rechunk(rid, c["chunk_bytes"])
+                    J.set_halo_only()   # rechunk drops per-chunk destinations
+                for _ in range(3):
+                    J.step(s)
+                ts = []
+                for _ in range(5):
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(s)
+                    J.step(s, barrier=True)
+                    b.record(s)
+                    s.synchronize()
+                    ts.append(a.elapsed_time(b))
+                return statistics.median(ts)
+
+            hspace = "mech=0;chunk=131072,1048576;warps=1,2,4;push=0,1;akern=0,1,2"
+            hb = rt.autotune(f"bench_jacobi_halo_N{N}_G{world}", run_halo, hspace)
+            if hb["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+                for rid in J.rid:
+                    rt.rechunk(rid, hb["chunk_bytes"])
+                J.set_halo_only()
+            rt.set_config(agent_warps=hb["agent_warps"], push=hb["push"], agent_kernel=hb["agent_kernel"])
+            halo_tuned = {"space": hspace, "best": {k: hb[k] for k in ("chunk_bytes", "agent_warps", "push",
+                                                                     "agent_kernel")}}
         legs = [("proact", mech), ("bulk_cudaMemcpyPeer", _lib.MECH_BULK), ("naive_p2p_inline", _lib.MECH_INLINE)]
         hv = {}
         for name, m in legs:
@@ -543,12 +655,14 @@ def main():
             step()
             hv[name] = kk * I / (timed(step, kk) / 1000.0)
         mode["nccl"] = nccl_base
-        rt.set_config(mech=mech)
+        rt.set_config(mech=mech, agent_warps=full_cfg["agent_warps"], push=full_cfg["push"],
+                      agent_kernel=full_cfg["agent_kernel"])
         h_rows = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
         h_ingress = 4.0 * N * max(1, h_rows) if world > 1 else 0.0
         ht = 1000.0 / hv["proact"] * 1000.0   # us per phase
         h_nvl = h_ingress / (NVL * 1e9) * 1e6
-        halo = {"value": hv["proact"], "unit": "iters/s", "baselines_iters_per_s": {k: v for k, v in hv.items() if k != "proact"},
+        halo = {"value": hv["proact"], "unit": "iters/s", "tuned": halo_tuned,
+                "baselines_iters_per_s": {k: v for k, v in hv.items() if k != "proact"},
                 "speedup_vs_n1": None,
                 "step_roofline": {"t_hbm_us": t_hbm_us, "t_nvl_us": h_nvl, "t_phase_us": ht,
                                   "frac": max(t_hbm_us, h_nvl) / ht,
@@ -603,7 +717,9 @@ def main():
                "h2d_bytes_per_step": nb[0], "d2h_bytes_per_step": nb[1],
                "api": "proact_jacobi_solve_host_pipelined", "steps": K,
                "sequential_value": seq, "sequential_api": "proact_jacobi_solve_host"}
+        del xh, out, outs   # 3 GiB of pinned host memory: release before the secondary legs
 
+    line = None
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "iters/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
@@ -629,12 +745,17 @@ def main():
                                           "uninstrumented single-GPU solve (LOCAL) of the full grid on every "
                                           "rank's GPU in this run, slowest rank")},
                 "halo_only": halo, "agent_cost": agent_cost, "decomposition": decomposition}
-        print(json.dumps(line), flush=True)
     torch.cuda.synchronize()
     J.free()
+    del J
     rt.finalize()
     if world > 1:
         dist.destroy_process_group()
+    if line is not None:
+        if world == 1 and not args.no_secondary:
+            torch.cuda.empty_cache()
+            line["secondary"] = secondary_legs(N, peak)
+        print(json.dumps(line), flush=True)
 
 
 if __name__ == "__main__":

@@ -349,6 +349,10 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
         // this generation) and counts the chunk into its group with system-scope release
         R.counter[c] = 0u;
         asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(R.group_cnt + c / R.dma_group) : "memory");
+    } else if (old + b == ex && !transfers(lc, R, c)) {
+        // bound nowhere (halo-only interiors): nothing to push, no agent round trip -- the last
+        // committer sets my own flag and resets the counter; the agent never sees the chunk
+        publish_chunk(lc, r, c);
     } else if (old + b == ex && lc.discovery == PROACT_DISCOVER_QUEUE && lc.mech != PROACT_MECH_DMA) {
         const uint32_t piece = piece_size(lc, R);
         const uint32_t P = (R.chunk_bytes + piece - 1) / piece;

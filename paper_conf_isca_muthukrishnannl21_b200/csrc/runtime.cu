@@ -972,16 +972,26 @@ int proact_region_set_chunk_dest(int id, uint32_t chunk, uint64_t mask)
     if (chunk >= R.n_own) return PROACT_ERR_INVALID;
     cudaSetDevice(c->device);
     if (R.chunk_dest.empty()) {
-        R.chunk_dest.assign(R.n_own, (uint32_t)R.dest_mask);
-        CK(cudaMalloc((void **)&R.d_chunk_dest, 4 * (size_t)R.n_own));
+        // device copy: the n_own masks, then two words the agent sizes its work with (chunks
+        // bound nowhere never reach it): [n_own] = my chunks with a destination, [n_own + 1] =
+        // 1 if my last (possibly partial) chunk has one
+        R.chunk_dest.assign(R.n_own + 2, (uint32_t)R.dest_mask);
+        CK(cudaMalloc((void **)&R.d_chunk_dest, 4 * ((size_t)R.n_own + 2)));
         c->h.region[id].chunk_dest = R.d_chunk_dest;
         c->h.region[id].n_in = 0xFFFFFFFFu;
         int rc = upload_ctx(c);
         if (rc) return rc;
     }
     R.chunk_dest[chunk] = (uint32_t)mask;
+    {
+        const uint32_t peers = (c->world < 32 ? (1u << c->world) - 1u : 0xFFFFFFFFu) & ~(1u << c->rank);
+        uint32_t nb = 0;
+        for (uint32_t k = 0; k < R.n_own; ++k) nb += (R.chunk_dest[k] & peers) != 0u;
+        R.chunk_dest[R.n_own] = nb;
+        R.chunk_dest[R.n_own + 1] = R.n_own && (R.chunk_dest[R.n_own - 1] & peers) != 0u ? 1u : 0u;
+    }
     if (R.dma_exec) { cudaGraphExecDestroy(R.dma_exec); R.dma_exec = nullptr; }   // new geometry
-    CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * (size_t)R.n_own, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(R.d_chunk_dest, R.chunk_dest.data(), 4 * ((size_t)R.n_own + 2), cudaMemcpyHostToDevice));
     return PROACT_OK;
 }
 
@@ -1431,7 +1441,7 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
             for (int r = 0; r < c->nregions; ++r)
                 if (armed >> r & 1) {
                     const Region &R = c->regions[r];
-                    if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
+                    if (!R.chunk_dest.empty()) for (uint32_t k = 0; k < R.n_own; ++k) peers |= R.chunk_dest[k];
                     else peers |= (uint32_t)R.dest_mask;
                 }
             peers &= ~(1u << c->rank);
@@ -1480,7 +1490,7 @@ int proact_phase_sync(void *stream, int mode)
         for (int r = 0; r < c->nregions; ++r)
             if (c->bulk_mask >> r & 1) {
                 const Region &R = c->regions[r];
-                if (!R.chunk_dest.empty()) for (uint32_t m : R.chunk_dest) peers |= m;
+                if (!R.chunk_dest.empty()) for (uint32_t k = 0; k < R.n_own; ++k) peers |= R.chunk_dest[k];
                 else peers |= (uint32_t)R.dest_mask;
             }
         peers &= ~(1u << c->rank);

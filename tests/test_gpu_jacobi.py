@@ -114,13 +114,45 @@ def test_jacobi_mixed_mechanisms_across_phases():
         assert np.array_equal(rep.view(np.uint32), want.view(np.uint32)), g
 
 
-def test_jacobi_halo_only_owned_rows_and_halos():
-    G, N, iters = 4, 512, 9
-    want = oracle.jacobi(synth.jacobi_init(N), iters)
-    outs = run_ranks(G, _run_jacobi, N, iters, 8192, _lib.MECH_FUSED, halo_only=True)
-    for g, (rep, (r0, r1), _) in enumerate(outs):
-        lo, hi = max(r0 - 1, 0), min(r1 + 1, N)
-        assert np.array_equal(rep[lo:hi].view(np.uint32), want[lo:hi].view(np.uint32)), g
+@pytest.mark.parametrize("cfg", [dict(), dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_BULK),
+                                 dict(agent_kernel=_lib.AGENT_SEPARATE, push=_lib.PUSH_VEC16,
+                                      discovery=_lib.DISCOVER_SCAN, agent_warps=2),
+                                 dict(agent_kernel=_lib.AGENT_FUSED, agent_warps=1),
+                                 dict(agent_kernel=_lib.AGENT_FUSED, discovery=_lib.DISCOVER_SCAN, agent_warps=1)])
+def test_jacobi_halo_only_owned_rows_and_halos(cfg):
+    """Halo-only: chunks bound nowhere are published by their last committer and never reach
+    the agent (queue sized / scan windows skipped from the per-chunk destinations), for every
+    agent placement and discovery mode; ragged last chunk (N = 520 rows of 2080 B, 8 KiB chunks)."""
+    for G, N, iters in ((4, 512, 9), (2, 520, 7)):
+        want = oracle.jacobi(synth.jacobi_init(N), iters)
+        outs = run_ranks(G, _run_jacobi, N, iters, 8192, _lib.MECH_FUSED, halo_only=True, **cfg)
+        for g, (rep, (r0, r1), _) in enumerate(outs):
+            lo, hi = max(r0 - 1, 0), min(r1 + 1, N)
+            assert np.array_equal(rep[lo:hi].view(np.uint32), want[lo:hi].view(np.uint32)), (g, G, cfg)
+
+
+def test_jacobi_halo_only_exactly_once():
+    """Halo-only delivery counters: every chunk with a destination is delivered once per phase
+    to each destination, chunks bound nowhere never."""
+    os.environ["PROACT_DEBUG"] = "1"
+    try:
+        G, N, iters = 3, 768, 4
+        outs = run_ranks(G, _run_jacobi, N, iters, 8192, _lib.MECH_FUSED, halo_only=True, check_deliv=True,
+                         agent_kernel=_lib.AGENT_SEPARATE)
+    finally:
+        os.environ.pop("PROACT_DEBUG", None)
+    rowb = N * 4
+    for g, (_, (r0, r1), deliv) in enumerate(outs):
+        own = (r1 - r0) * rowb
+        nch = (own + 8191) // 8192
+        assert len(deliv) == iters
+        for k, d in enumerate(deliv):
+            assert d.shape == (nch, G)
+            for c in range(nch):
+                lo, hi = c * 8192, min((c + 1) * 8192, own)
+                for q in range(G):
+                    bound = (q == g - 1 and lo < rowb) or (q == g + 1 and hi > own - rowb)
+                    assert d[c, q] == (1 if bound else 0), (g, k, c, q, d[c, q])
 
 
 @pytest.mark.parametrize("akern", [0, 2])

@@ -97,6 +97,7 @@ def test_bench_two_processes_json_line():
     # halo-only variant beside full replication, with its own baselines and roofline
     h = d["halo_only"]
     assert h["value"] > 0 and h["speedup_vs_n1"] > 0 and h["step_roofline"]["frac"] > 0
+    assert "warps=1,2,4" in h["tuned"]["space"] and h["tuned"]["best"]["agent_kernel"] in (0, 1, 2)
     assert set(h["baselines_iters_per_s"]) == {"bulk_cudaMemcpyPeer", "naive_p2p_inline"}
     assert d["agent_cost"]["agent_sm_ms_per_GB_pushed"] >= 0
     dc = d["decomposition"]   # NEXT-1: infinite-bandwidth bound, tracking overhead, captured
