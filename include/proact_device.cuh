@@ -247,11 +247,13 @@ __device__ __forceinline__ uint32_t dests_of(const launch_ctx &lc, const region_
     return m;
 }
 
-/* Does my chunk c take part in the transfer this launch?  Chunks with destinations do; under
- * ELIDE every chunk does (tracking and agent run as if pushing: the overhead methodology). */
+/* Does my chunk c take part in the transfer this launch?  Chunks with destinations do.  Under
+ * ELIDE (tracking and agent run as if pushing: the overhead methodology) every chunk does when
+ * the region has one default destination mask -- at G = 1 it is empty -- and the chunks with
+ * destinations do when per-chunk destinations are set (halo-only: as if pushing the halo). */
 __device__ __forceinline__ bool transfers(const launch_ctx &lc, const region_dev &R, uint32_t c)
 {
-    return lc.mech == PROACT_MECH_ELIDE || dests_of(lc, R, c) != 0u;
+    return (lc.mech == PROACT_MECH_ELIDE && !R.chunk_dest) || dests_of(lc, R, c) != 0u;
 }
 
 /* ---------------------------------------------------------------- producer side (a2, a3) -- */
@@ -364,6 +366,25 @@ __device__ __forceinline__ void commit_chunk(const launch_ctx &lc, int r, uint32
             const unsigned long long e = ((unsigned long long)gen << 32) | (unsigned long long)(c * P + k);
             asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(R.queue + idx + k), "l"(e) : "memory");
         }
+    }
+}
+
+/* PROACT_AGENT_PRODUCER count of DELIVERED bytes (reading R21), for a caller that has already
+ * fenced after its bulk stores completed (fence.proxy.async + fence.acq_rel.sys/gpu, tile_pusher's
+ * flush): that fence is the release, so the count is a relaxed RMW -- no per-chunk membar -- and only
+ * the contributor that completes the chunk acquires (fence.acq_rel.gpu: every other contributor's
+ * fence-then-count is ordered before it) and publishes the chunk's flags. */
+__device__ __forceinline__ void commit_delivered(const launch_ctx &lc, int r, uint32_t c, uint32_t b)
+{
+    const region_dev &R = lc.ctx->region[r];
+    uint32_t old;
+    asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(&R.counter[c]), "r"(b) : "memory");
+    const uint32_t ex = R.expected[c];
+    if (old + b > ex) {
+        raise_error(lc.ctx, SITE_COMMIT, PROACT_ERR_PROTOCOL);
+    } else if (old + b == ex) {
+        fence_acq_rel_gpu();
+        publish_chunk(lc, r, c);
     }
 }
 

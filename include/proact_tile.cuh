@@ -33,7 +33,7 @@ enum { TD_END = 1 };   // no more spans: the transfer warp drains and returns
 __host__ __device__ constexpr uint32_t td_rows(uint32_t rows) { return rows << 8; }
 
 #ifndef PROACT_TP_RD
-#define PROACT_TP_RD 2
+#define PROACT_TP_RD 0   // release a slot as soon as its bulk stores have read it (r02z sweep: 0.650 vs 0.715 ms loopback G = 2)
 #endif
 #ifndef PROACT_TP_CD
 #define PROACT_TP_CD 8
@@ -41,8 +41,14 @@ __host__ __device__ constexpr uint32_t td_rows(uint32_t rows) { return rows << 8
 #ifndef PROACT_TP_SYSFENCE
 #define PROACT_TP_SYSFENCE 1
 #endif
+// completed rows per flush (one fence + the merged counter commits).  Under full HBM load a fence
+// waits ~4 us for the SM's write queue to drain, and the transfer warp issues no span meanwhile, so
+// flushes are rare (r02z sweep, loopback G = 2 at 1 MiB chunks: 64 -> 256 rows 0.647 -> 0.553 ms)
 #ifndef PROACT_TP_FLUSH
-#define PROACT_TP_FLUSH 64   // completed rows per flush (one fence + the merged counter commits)
+#define PROACT_TP_FLUSH 256
+#endif
+#ifndef PROACT_TP_RELAXED_COMMIT   // flush commits: relaxed counts after the flush fence
+#define PROACT_TP_RELAXED_COMMIT 1
 #endif
 #ifndef PROACT_TP_PROXYFENCE
 #define PROACT_TP_PROXYFENCE 1
@@ -50,7 +56,10 @@ __host__ __device__ constexpr uint32_t td_rows(uint32_t rows) { return rows << 8
 constexpr uint32_t TP_FLY = 16;   // descriptors of in-flight spans (> TP_CD)
 constexpr int TP_RD = PROACT_TP_RD;   // bulk groups whose shared-memory reads may still be pending
 constexpr int TP_CD = PROACT_TP_CD;   // bulk groups that may still be in flight (not complete)
-constexpr uint32_t TP_PEND = 32;  // (chunk, bytes) entries of completed, uncommitted rows
+#ifndef PROACT_TP_PEND
+#define PROACT_TP_PEND 128   // 128 KiB chunks: a 32-row tile strip touches 16 chunks
+#endif
+constexpr uint32_t TP_PEND = PROACT_TP_PEND;  // (chunk, bytes) entries of completed, uncommitted rows
 static_assert(TP_CD < (int)TP_FLY, "in-flight descriptors");
 
 // Shared-memory block of a tile pusher (placed in the kernel's dynamic shared memory).
@@ -159,7 +168,8 @@ __device__ __forceinline__ uint32_t tp_chunk(uint64_t rel, uint32_t cb)
 // dependent chain per row); completed bytes are merged per chunk into a pending list, and the
 // whole warp joins only for credit waits and for the flushes that commit the list -- one fence
 // (proxy fence + fence.acq_rel.sys when a pending byte went to a peer) per PROACT_TP_FLUSH rows,
-// then one release RMW per pending chunk (lane j: entry j).
+// then one relaxed RMW per pending chunk (lane j: entries j, j + 32, ...; commit_delivered: the
+// flush fence is the release, the completing contributor acquires before publishing).
 //
 // local_done = true: the producer warps already stored the span to the local replica themselves
 // (plain st.global, before their tp_publish, whose release the transfer warp acquires): only the
@@ -356,8 +366,14 @@ __device__ __noinline__ void tile_pusher(const launch_ctx &lc, int r, const unsi
                 else fence_acq_rel_gpu();
                 // chunks bound nowhere are never counted (tiles that write only such chunks skip
                 // the transfer warp altogether, so their counts would be partial)
-                if (lane < n && !dead && transfers(lc, R, T->pend_c[lane]))
-                    commit_chunk(lc, r, T->pend_c[lane], T->pend_b[lane]);
+                for (uint32_t j = lane; j < n; j += 32) {
+                    if (dead || !transfers(lc, R, T->pend_c[j])) continue;
+#if PROACT_TP_RELAXED_COMMIT
+                    commit_delivered(lc, r, T->pend_c[j], T->pend_b[j]);
+#else
+                    commit_chunk(lc, r, T->pend_c[j], T->pend_b[j]);
+#endif
+                }
                 __syncwarp();
             }
             if (lane == 0) {

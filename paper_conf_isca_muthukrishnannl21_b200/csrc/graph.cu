@@ -116,8 +116,11 @@ constexpr int MAXGRAPH = 4;
 // 2.4x slower (the gathers are latency-bound, tools/sweep_pagerank.py).
 constexpr uint32_t HOT_BIT = 0x80000000u;
 constexpr uint32_t HOT_MAX = 65536;   // 16-bit slots; above HOT_SLICE the table spans a cluster
-constexpr uint32_t HOT_SLICE = 8192;  // entries one CTA holds (32 KiB; 2 CTAs of 1024 threads per SM)
-constexpr uint32_t HOT_SHIFT = 13;
+#ifndef PROACT_HOT_SLICE_LOG2
+#define PROACT_HOT_SLICE_LOG2 13
+#endif
+constexpr uint32_t HOT_SHIFT = PROACT_HOT_SLICE_LOG2;
+constexpr uint32_t HOT_SLICE = 1u << HOT_SHIFT;  // entries one CTA holds (8192: 32 KiB; 2 CTAs of 1024 threads per SM)
 #ifndef PROACT_GRAPH_HOT_DEFAULT
 #define PROACT_GRAPH_HOT_DEFAULT 8192
 #endif

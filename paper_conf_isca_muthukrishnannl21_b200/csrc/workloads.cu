@@ -358,6 +358,9 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             tpush = false;
             for (uint64_t c = a0 / Ro.chunk_bytes; c * Ro.chunk_bytes < a1 && !tpush; ++c)
                 tpush = proact::transfers(lc, Ro, (uint32_t)c);
+#if defined(PROACT_TP_EXP) && PROACT_TP_EXP == 2   // timing experiment: no staging at all
+            tpush = false;
+#endif
         }
         auto rows = [&](auto fast_tag) {
             constexpr bool FAST = decltype(fast_tag)::value;
@@ -397,7 +400,9 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     }
                     const uint64_t off = ((uint64_t)i * N + j) * 4;
                     if (MODE == 2) {   // the local copy now, the span for the transfer warp
+#if !defined(PROACT_TP_EXP) || PROACT_TP_EXP != 1   // (1: timing experiment, no staging stores)
                         if (tpush) *reinterpret_cast<float4 *>(ostrip + 4 * tid + g * GW) = o;
+#endif
                         *reinterpret_cast<float4 *>(outb + off) = o;
                     } else if (!FAST && lc.mech == PROACT_MECH_INLINE) {
                         proact::put(lc, p.region_out, off, o);
@@ -539,23 +544,32 @@ __global__ void __launch_bounds__(MB, 4) micro_kernel(launch_ctx lc, proact_micr
     }
 }
 
-// PROACT_AGENT_PRODUCER variant: 8 compute warps write each 4 KiB tile into a shared-memory ring
-// slot (same values and store-order options), the transfer warp bulk-stores it to the local
-// replica and every destination mirror and counts it once delivered (proact::tile_pusher); one
-// flush (system fence + counter commits) per MBLK tiles = 32 KiB, as the commits above.
-constexpr uint32_t MOS = 8;   // output ring slots (4 KiB each)
-constexpr size_t MTP_SMEM = (size_t)MOS * 4096 + sizeof(proact::tile_ring_ctl<MOS>);
+// PROACT_AGENT_PRODUCER variant: 8 compute warps write each 4 KiB tile (L279) into a shared-memory
+// ring slot (same values and store-order options); MTS consecutive tiles of the CTA's block form
+// one span (contiguous in the region), which the transfer warp bulk-stores to the local replica
+// and every destination mirror with one TMA store each, and counts once delivered
+// (proact::tile_pusher).  Spans of 4 tiles: the transfer warp's per-span work is amortised over
+// 16 KiB instead of 4 KiB.
+#ifndef PROACT_MICRO_SPAN_TILES
+#define PROACT_MICRO_SPAN_TILES 4
+#endif
+#ifndef PROACT_MICRO_OUT_RING
+#define PROACT_MICRO_OUT_RING 3
+#endif
+constexpr uint32_t MTS = PROACT_MICRO_SPAN_TILES;   // 4 KiB tiles per pushed span
+constexpr uint32_t MOS = PROACT_MICRO_OUT_RING;     // output ring slots (MTS x 4 KiB each)
+constexpr size_t MTP_SMEM = (size_t)MOS * MTS * 4096 + sizeof(proact::tile_ring_ctl<MOS>);
 
 __global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, proact_micro_params p)
 {
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ __align__(128) unsigned char msm[];
     uint32_t *oring = reinterpret_cast<uint32_t *>(msm);
-    auto *tp = reinterpret_cast<proact::tile_ring_ctl<MOS> *>(msm + (size_t)MOS * 4096);
+    auto *tp = reinterpret_cast<proact::tile_ring_ctl<MOS> *>(msm + (size_t)MOS * MTS * 4096);
     if (threadIdx.x == 0) proact::tp_init(tp, MB / 32);
     __syncthreads();
     if (threadIdx.x >= MB) {
-        proact::tile_pusher<MOS>(lc, p.region, msm, 4096, tp);
+        proact::tile_pusher<MOS>(lc, p.region, msm, MTS * 4096, tp);
         return;
     }
     if (p.verify_region >= 0 && p.phase > 0) {   // litmus: the producer warps check (named barrier)
@@ -578,10 +592,11 @@ __global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, pro
     uint32_t q = 0;
     for (uint64_t bk = proact::producer_block(lc); bk < nblk; bk += proact::producer_grid(lc)) {
         const uint64_t tb0 = bk * MBLK, tb1 = min(tb0 + MBLK, ntiles);
-        for (uint64_t t = tb0; t < tb1; ++t, ++q) {
+        for (uint64_t t = tb0; t < tb1; ++t) {
             const uint64_t t0 = w_lo + t * 1024, t1 = min(t0 + 1024, w_hi);
-            proact::tp_acquire(tp, q);
-            uint32_t *slot = oring + (q % MOS) * 1024;
+            const uint32_t sub = (uint32_t)((t - tb0) % MTS);   // tile within the span
+            if (sub == 0) proact::tp_acquire(tp, q);
+            uint32_t *slot = oring + ((q % MOS) * MTS + sub) * 1024;
             if (!p.scattered) {
                 const uint64_t k = t0 + 4 * threadIdx.x;
                 if (k + 4 <= t1) {
@@ -601,9 +616,14 @@ __global__ void __launch_bounds__(MB + 32, 4) micro_tp_kernel(launch_ctx lc, pro
                     if (w < t1) slot[w - t0] = micro_value((uint32_t)w, p.phase, p.seed, p.K);
                 }
             }
-            if (threadIdx.x == 0)
-                tp->desc[q % MOS] = proact::tile_desc{t0 * 4, (uint32_t)(t1 - t0) * 4, proact::td_rows(1)};
-            proact::tp_publish(tp, q);
+            if (sub == MTS - 1 || t + 1 == tb1) {   // hand the span (tiles t - sub .. t) over
+                if (threadIdx.x == 0) {
+                    const uint64_t s0 = t0 - (uint64_t)sub * 1024;
+                    tp->desc[q % MOS] = proact::tile_desc{s0 * 4, (uint32_t)(t1 - s0) * 4, proact::td_rows(1)};
+                }
+                proact::tp_publish(tp, q);
+                ++q;
+            }
         }
     }
     proact::tp_acquire(tp, q);
@@ -740,9 +760,11 @@ static int micro_launch(proact_micro_params &p, void *stream)
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {p.region};
-    if (proact_launch_mode() == 2)
+    if (proact_launch_mode() == 2) {
+        if (proact_internal_smem_attr((const void *)micro_tp_kernel, MTP_SMEM)) return PROACT_ERR_CUDA;
         return proact_launch_ex(regs, 1, (const void *)micro_tp_kernel, 0, MB + 32, args, MTP_SMEM, stream,
                                 PROACT_LAUNCH_TILE_PUSH);
+    }
     return proact_launch(regs, 1, (const void *)micro_kernel, 0, MB, args, 0, stream);
 }
 
