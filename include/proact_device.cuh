@@ -124,7 +124,8 @@ enum { LCF_SEPARATE = 1,   /* this is the SEPARATE agent kernel's copy (start-up
 enum { SITE_AGENT_POLL = 1, SITE_AGENT_CREDIT = 2, SITE_WAIT_RANGE = 3, SITE_WAIT_ALL = 4,
        SITE_SYNC = 5, SITE_COMMIT = 6, SITE_AGENT_COUNT = 7, SITE_AGENT_PUSH = 8,
        SITE_AGENT_START = 9,   /* SEPARATE agent: its producer grid never started (serialised?) */
-       SITE_TILE_PUSH = 10 };  /* tile pusher: credit wait / store completion */
+       SITE_TILE_PUSH = 10,    /* tile pusher: credit wait / store completion */
+       SITE_GRID_BARRIER = 11 };  /* a producer's grid-wide barrier (SSSP push rounds) */
 
 #ifdef __CUDACC__
 

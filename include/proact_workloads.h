@@ -158,6 +158,18 @@ int proact_pagerank_ranks(int graph, float *d_out, void *stream);
  * registered with PROACT_REGION_SPARSE and chunk_bytes a multiple of 4096.  A round that
  * changes anything casts a proact::vote (read it with a BARRIER phase_sync + proact_last_vote). */
 int proact_sssp_phase(int graph, int region_in, int region_out, int first, void *stream);
+/* (Same call.)  Weighted graphs also hold my in-edges grouped by source, and each round is either
+ * a PULL round (above) or a PUSH round (reading R24, PAPER.md L267's Bellman-Ford with only the
+ * sources whose distance changed in the previous round relaxing their edges into my vertices,
+ * atomicMin into a private array; identical d').  The choice is made per rank from the out-degree
+ * of the vertices this rank changed in the previous round (copied to the host after that round's
+ * kernel: call after synchronising with it for a current decision); env PROACT_SSSP_PUSH = 0 / 1
+ * forces pull / push, PROACT_SSSP_PUSH_PCT (default 8) is the frontier share of the edges below
+ * which a round pushes.  Every rank keeps a private copy of the previous round's input (V ints),
+ * refreshed by push rounds and by pull rounds whose frontier is below 4x that share (a round
+ * pushes only after a round that refreshed it). */
+/* Mode of the graph's last launched SSSP round: 0 pull, 1 push; PROACT_ERR_INVALID for a bad id. */
+int proact_sssp_last_mode(int graph);
 
 #ifdef __cplusplus
 }

@@ -130,6 +130,7 @@ def _declare(L):
         "proact_pagerank_phase": (i, [i, i, i, ctypes.c_double, vp]),
         "proact_pagerank_ranks": (i, [i, vp, vp]),
         "proact_sssp_phase": (i, [i, i, i, i, vp]),
+        "proact_sssp_last_mode": (i, [i]),
     }
     missing = []
     for name, (res, args) in sigs.items():

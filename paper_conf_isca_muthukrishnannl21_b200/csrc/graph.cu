@@ -105,6 +105,22 @@ struct Graph {
     uint32_t *rowidx_h = nullptr, *hot_ids = nullptr;
     uint32_t nhot = 0;
     uint64_t e_hot = 0;   // my in-edges whose source is hot
+    // SSSP push rounds (weighted graphs): my in-edges grouped by SOURCE, the private copy of the
+    // previous round's input, the round's relaxation minima, the frontier's heavy sources
+    uint64_t E_all = 0;                    // global edge count (the build's E)
+    uint32_t *prp = nullptr;               // [V + 1] row pointers over global source ids
+    uint32_t *pcol = nullptr;              // [E_own] local destination v - v0
+    int32_t *pwt = nullptr;                // [E_own] weight
+    int32_t *dprev = nullptr;              // [V] previous round's input distances
+    int32_t *ptmp = nullptr;               // [nv] minima of the round, INT32_MAX between rounds
+    uint32_t *heavy = nullptr;             // [nheavy_max] frontier sources with > PUSH_HEAVY edges here
+    uint32_t nheavy_max = 0;
+    uint32_t *pctl = nullptr;              // [4]: heavy count, barrier arrivals, barrier generation
+    unsigned long long *dcnt = nullptr;    // [2] per round parity: out-degree sum of my changed vertices
+    unsigned long long *hcnt = nullptr;    // pinned: the last round's sum (read for the next decision)
+    uint32_t round = 0;
+    bool tracked = false;                  // the last round left dprev = its input
+    int last_mode = 0;                     // 0 pull, 1 push (last launched round)
 };
 constexpr int MAXGRAPH = 4;
 
@@ -315,11 +331,22 @@ struct PrParams {
     int region_in, region_out;
     double d, base;   // damping, (1-d)/V
 };
+// SSSP push rounds (direction-optimised Bellman-Ford, reading R24): device pointers of the Graph's
+// push arrays; track = keep dprev current (every round, pull or push), par = round parity
+struct PushDev {
+    const uint32_t *prp, *pcol;
+    const int32_t *pwt;
+    int32_t *dprev, *ptmp;
+    uint32_t *heavy, *pctl;
+    unsigned long long *dcnt;
+    uint32_t track, par;   // track: pull kernels keep dprev current this round
+};
 struct SsspParams {
     GraphDev g;
     int region_in, region_out;
     int first;        // phase 0: every source is "changed"
     int pad;
+    PushDev q;
 };
 
 // L2 policies: the CSC stream (read once per phase) is evict-first, the gathered vertex vector
@@ -840,6 +867,79 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
     if (CL > 1) cluster_sync_all();   // my slice stays readable until every peer is done
 }
 
+// Helpers of the SSSP push rounds (reading R24; see sssp_push_kernel) shared with the pull kernels.
+constexpr uint32_t PUSH_HEAVY = 1024;   // frontier sources with more edges here: spread over the grid
+constexpr uint32_t PB = 256;            // threads per push-round CTA (x 4 vertices = one 4 KiB block)
+
+__device__ __forceinline__ int32_t ld_cg_i(const int32_t *p)
+{
+    int32_t v;
+    asm volatile("ld.global.cg.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+// Grid-wide barrier of the producer CTAs (all co-resident: proact_launch caps the persistent grid
+// at the co-resident capacity).  ctl[1] arrivals, ctl[2] generation; watchdog-guarded.
+__device__ __forceinline__ bool grid_barrier(const launch_ctx &lc, uint32_t *ctl)
+{
+    __shared__ uint32_t gb_bad;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        gb_bad = 0u;
+        const uint32_t gen = proact::ld_acquire_gpu(&ctl[2]);   // before arriving
+        __threadfence();
+        if (atomicAdd(&ctl[1], 1u) + 1u == proact::producer_grid(lc)) {
+            ctl[1] = 0u;            // re-armed before the release
+            __threadfence();
+            atomicAdd(&ctl[2], 1u);
+        } else {
+            const uint64_t t0 = proact::globaltimer();
+            uint32_t it = 0;
+            while (proact::ld_acquire_gpu(&ctl[2]) == gen)
+                if (proact::spin_step(lc.ctx, t0, it, proact::SITE_GRID_BARRIER)) { gb_bad = 1u; break; }
+        }
+        __threadfence();
+    }
+    __syncthreads();
+    return gb_bad == 0u;
+}
+// dprev := the arrived input (pull rounds; the push kernel does it while finding the frontier):
+// 16-byte vectors, two in flight per thread (the loop is latency-bound otherwise)
+__device__ __forceinline__ void track_input(const launch_ctx &lc, const SsspParams &p, const int32_t *din)
+{
+    if (!p.q.track) return;
+    const uint64_t n4 = p.g.V / 4, stride = (uint64_t)proact::producer_grid(lc) * blockDim.x;
+    const int4 *a = reinterpret_cast<const int4 *>(din);
+    int4 *b = reinterpret_cast<int4 *>(p.q.dprev);
+    for (uint64_t i = (uint64_t)proact::producer_block(lc) * blockDim.x + threadIdx.x; i < n4; i += 2 * stride) {
+        const bool two = i + stride < n4;
+        const int4 x0 = a[i], y0 = b[i];
+        int4 x1 = x0, y1 = y0;
+        if (two) {
+            x1 = a[i + stride];
+            y1 = b[i + stride];
+        }
+        if (x0.x != y0.x || x0.y != y0.y || x0.z != y0.z || x0.w != y0.w) b[i] = x0;
+        if (two && (x1.x != y1.x || x1.y != y1.y || x1.z != y1.z || x1.w != y1.w)) b[i + stride] = x1;
+    }
+    if (proact::producer_block(lc) == 0)
+        for (uint64_t u = n4 * 4 + threadIdx.x; u < p.g.V; u += blockDim.x) p.q.dprev[u] = din[u];
+}
+// out-degree sum of my changed vertices, for the next round's pull / push decision (host)
+__device__ __forceinline__ void count_changed(const SsspParams &p, unsigned long long cs)
+{
+    if (!p.q.dcnt) return;   // (callers accumulate in 32 bits: a thread's vertices' out-degrees)
+    for (int o = 16; o > 0; o >>= 1) cs += __shfl_xor_sync(0xFFFFFFFFu, cs, o);
+    if ((threadIdx.x & 31u) == 0u && cs) atomicAdd(&p.q.dcnt[p.q.par], cs);
+}
+// relax edge e (source distance du) into my vertex pcol[e]: a fire-and-forget atomicMin (RED)
+__device__ __forceinline__ void push_relax(const SsspParams &p, uint32_t e, int32_t du)
+{
+    const uint32_t v = __ldg(p.q.pcol + e);
+    const int64_t c = (int64_t)du + (int64_t)__ldg(p.q.pwt + e);
+    const int32_t cand = c < (int64_t)INT32_MAX ? (int32_t)c : INT32_MAX;
+    atomicMin(p.q.ptmp + v, cand);
+}
+
 constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
 
 // SSSP: merge-path over the item's in-edges; a source is relaxed only if its chunk changed in
@@ -860,6 +960,14 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
     const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
     __shared__ uint32_t kclaim;
     bool ready = false;
+    if (p.q.dcnt) {   // every CTA keeps its share of dprev current (if asked), items or not
+        if (threadIdx.x == 0) {
+            proact::wait_all(lc, p.region_in);
+            if (proact::producer_block(lc) == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;
+        }
+        __syncthreads();
+        track_input(lc, p, din);
+    }
     for (;;) {
         if (threadIdx.x == 0) kclaim = proact::claim_tile(lc, p.g.nitems);   // items dealt dynamically
         __syncthreads();
@@ -957,13 +1065,16 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
         }
         if (fin) {
             bool changed = false;
+            uint32_t cs = 0;   // out-degree sum of the tile's changed vertices (push decision, R24)
             for (uint32_t i = threadIdx.x; i < nvt; i += GB) {
                 const uint32_t v = lo + i;
                 const int32_t old = din[v];
                 const int32_t best = min(old, acc[i]);
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
                 changed |= best != old;
+                if (best != old) cs += __ldg(p.g.outdeg + v);
             }
+            count_changed(p, cs);
             // per-tile chunk state (SPARSE region): changed now -> flag bit + vote; push if
             // changed now or in the previous round (the peers' ping-pong copy holds d^{k-1})
             const int any = __syncthreads_or(changed);
@@ -1016,8 +1127,10 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
     if (threadIdx.x == 0) {
         proact::wait_all(lc, p.region_in);
         nout = 0u;
+        if (p.q.dcnt && proact::producer_block(lc) == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;
     }
     __syncthreads();
+    track_input(lc, p, din);   // dprev := this round's input (push rounds, reading R24)
     {
         const uint32_t gen = lc.gen[p.region_in];
         const uint32_t pm = lc.gen_mech[p.region_in];
@@ -1183,13 +1296,16 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
             if (t == 0) any_a[grp] = 0u;
             grp_bar(grp);
             bool changed = false;
+            uint32_t cs = 0;   // out-degree sum of the tile's changed vertices (push decision, R24)
             for (uint32_t i = t; i < nvt; i += GB) {
                 const uint32_t v = lo + i;
                 const int32_t old = din[v];
                 const int32_t best = min(old, acc[i]);
                 proact::put(lc, p.region_out, (uint64_t)v * 4, best);
                 changed |= best != old;
+                if (best != old) cs += __ldg(p.g.outdeg + v);
             }
+            count_changed(p, cs);
             if (__any_sync(0xFFFFFFFFu, changed) && lane == 0) any_a[grp] = 1u;
             grp_bar(grp);   // orders the group's puts before the commit (a3)
             if (t == 0) {   // chunk state as in sssp_kernel
@@ -1207,6 +1323,227 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         grp_bar(grp);
     }
     if (CL > 1) cluster_sync_all();   // my slice stays readable until every peer is done
+}
+
+// ---- SSSP push rounds (reading R24: direction-optimised Bellman-Ford).  PAPER.md L267 fixes the
+// result -- "every vertex computes its shortest distance ... using the Bellman-Ford algorithm" --
+// d^{k+1}[v] = min(d^k[v], min_{u->v} d^k[u] + w); a source u with d^k[u] = d^{k-1}[u] was already
+// relaxed into v in round k, so only the FRONTIER (sources whose distance changed in round k)
+// matters.  When the frontier's out-edges are few (late rounds), the rank pushes from them over
+// its in-edges grouped by source (prp / pcol / pwt) with atomicMin into a private array, instead
+// of pulling over every in-edge; the same d^{k+1}, bit for bit (min is order independent).  The
+// frontier is found by comparing the arrived input with a PRIVATE copy of the previous input
+// (dprev, kept current in every round): the output replica itself cannot serve, peers' agents
+// already write this round's chunks into it.
+__global__ void __launch_bounds__(PB, 4) sssp_push_kernel(launch_ctx lc, SsspParams p)
+{
+    if (proact::agent_dispatch(lc)) return;
+    const region_dev &Ri = lc.ctx->region[p.region_in];
+    const int32_t *din = reinterpret_cast<const int32_t *>(Ri.base);
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t P = proact::producer_grid(lc), pb = proact::producer_block(lc);
+    if (threadIdx.x == 0) {
+        proact::wait_all(lc, p.region_in);   // (a7) the previous generation is here
+        if (pb == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;   // the next round's accumulator
+    }
+    __syncthreads();
+    // 1. frontier: sources whose input changed since the previous round (dprev := input); the
+    //    light ones are relaxed at once, warp-cooperatively, the heavy ones queued.  Each lane
+    //    takes 4 consecutive sources (16-byte loads of input and dprev; V % 4 sources at the end
+    //    by the first warp)
+    {
+        const uint64_t W = (uint64_t)P * (PB / 32), gw = (uint64_t)pb * (PB / 32) + (threadIdx.x >> 5);
+        const uint64_t n4 = p.g.V / 4;
+        const int4 *a4 = reinterpret_cast<const int4 *>(din);
+        int4 *b4 = reinterpret_cast<int4 *>(p.q.dprev);
+        auto frontier = [&](uint64_t u, int32_t du, int32_t dp) {   // -> (du, e0, e1) or e1 == e0
+            uint32_t e0 = 0, e1 = 0;
+            if ((p.first || du != dp) && du != INT32_MAX) {
+                e0 = __ldg(p.q.prp + u);
+                e1 = __ldg(p.q.prp + u + 1);
+                if (e1 - e0 > PUSH_HEAVY) {
+                    p.q.heavy[atomicAdd(&p.q.pctl[0], 1u)] = (uint32_t)u;
+                    e1 = e0;
+                }
+            }
+            return make_uint2(e0, e1);
+        };
+        auto relax_ballot = [&](int32_t du, uint2 r) {
+            uint32_t m = __ballot_sync(0xFFFFFFFFu, r.y > r.x);
+            while (m) {
+                const int j = __ffs(m) - 1;
+                m &= m - 1;
+                const int32_t dj = __shfl_sync(0xFFFFFFFFu, du, j);
+                const uint32_t x = __shfl_sync(0xFFFFFFFFu, r.x, j), y = __shfl_sync(0xFFFFFFFFu, r.y, j);
+                for (uint32_t e = x + lane; e < y; e += 32) push_relax(p, e, dj);
+            }
+        };
+        // the warp's light frontier sources of one window (<= 128) as a flat edge list: entry k =
+        // (first edge, source distance, end offset in the list); lane f relaxes edges f, f+32, ..
+        // -- independent loads in every lane instead of one source at a time
+        __shared__ uint32_t fl_e0[PB / 32][128], fl_end[PB / 32][128];
+        __shared__ int32_t fl_du[PB / 32][128];
+        uint32_t *we0 = fl_e0[threadIdx.x >> 5], *wend = fl_end[threadIdx.x >> 5];
+        int32_t *wdu = fl_du[threadIdx.x >> 5];
+        auto relax_flat = [&](const int32_t *dus, const uint2 *rs) {
+            uint32_t ne = 0, ned = 0;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                ne += rs[q].y > rs[q].x;
+                ned += rs[q].y - rs[q].x;
+            }
+            uint32_t pe = ne, pd = ned;   // inclusive warp scans
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t a = __shfl_up_sync(0xFFFFFFFFu, pe, o), b = __shfl_up_sync(0xFFFFFFFFu, pd, o);
+                if (lane >= (uint32_t)o) {
+                    pe += a;
+                    pd += b;
+                }
+            }
+            const uint32_t n = __shfl_sync(0xFFFFFFFFu, pe, 31), T = __shfl_sync(0xFFFFFFFFu, pd, 31);
+            if (T == 0) return;
+            uint32_t k = pe - ne, end = pd - ned;
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (rs[q].y > rs[q].x) {
+                    end += rs[q].y - rs[q].x;
+                    we0[k] = rs[q].x;
+                    wdu[k] = dus[q];
+                    wend[k] = end;
+                    ++k;
+                }
+            __syncwarp();
+            for (uint32_t f = lane; f < T; f += 32) {
+                uint32_t lo = 0, hi = n - 1;   // first entry whose end > f
+                while (lo < hi) {
+                    const uint32_t mid = (lo + hi) >> 1;
+                    if (wend[mid] > f) hi = mid;
+                    else lo = mid + 1;
+                }
+                const uint32_t start = lo ? wend[lo - 1] : 0u;
+                push_relax(p, we0[lo] + (f - start), wdu[lo]);
+            }
+            __syncwarp();
+        };
+        for (uint64_t base = gw * 32; base < n4; base += W * 32) {
+            const uint64_t i = base + lane;
+            int4 x = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX), y = x;
+            if (i < n4) {
+                x = a4[i];
+                y = b4[i];
+                if (x.x != y.x || x.y != y.y || x.z != y.z || x.w != y.w) b4[i] = x;
+            }
+            const int32_t xs[4] = {x.x, x.y, x.z, x.w}, ys[4] = {y.x, y.y, y.z, y.w};
+            uint2 rs[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) rs[q] = i < n4 ? frontier(4 * i + q, xs[q], ys[q]) : make_uint2(0u, 0u);
+            relax_flat(xs, rs);
+        }
+        if (pb == 0 && threadIdx.x < 32)   // the last V % 4 sources
+            for (uint64_t u0 = n4 * 4; u0 < p.g.V; u0 += 32) {
+                const uint64_t u = u0 + lane;
+                int32_t du = INT32_MAX;
+                uint2 r = make_uint2(0u, 0u);
+                if (u < p.g.V) {
+                    du = din[u];
+                    const int32_t dp = p.q.dprev[u];
+                    if (dp != du) p.q.dprev[u] = du;
+                    r = frontier(u, du, dp);
+                }
+                relax_ballot(du, r);
+            }
+    }
+    if (!grid_barrier(lc, p.q.pctl)) return;
+    // 2. heavy frontier sources: their edges spread over every producer thread
+    {
+        const uint32_t nh = __ldcg(p.q.pctl);
+        const uint64_t gt = (uint64_t)pb * PB + threadIdx.x, GTH = (uint64_t)P * PB;
+        for (uint32_t h = 0; h < nh; ++h) {
+            const uint32_t u = __ldcg(p.q.heavy + h);
+            const int32_t du = din[u];
+            const uint32_t a = __ldg(p.q.prp + u), b = __ldg(p.q.prp + u + 1);
+            for (uint64_t e = a + gt; e < b; e += GTH) push_relax(p, (uint32_t)e, du);
+        }
+    }
+    if (!grid_barrier(lc, p.q.pctl)) return;
+    if (pb == 0 && threadIdx.x == 0) p.q.pctl[0] = 0u;   // every CTA has read the heavy count
+    // 3. my vertices in blocks of 1024 (4 KiB, inside one chunk: chunks are multiples of 4 KiB
+    //    and slices chunk-aligned), 4 per thread with 16-byte loads: d' = min(d, minima),
+    //    instrumented stores, chunk state, vote, commit (a2, a3); the minima are reset to
+    //    INT32_MAX for the next push round
+    unsigned long long cs = 0;
+    const uint32_t nblk = (p.g.nv + 1023) / 1024;
+    for (uint32_t t = pb; t < nblk; t += P) {
+        const uint32_t lo = p.g.v0 + t * 1024, nvt = min(lo + 1024, p.g.v0 + p.g.nv) - lo;
+        const uint32_t i = 4 * threadIdx.x;
+        bool changed = false;
+        if (i + 4 <= nvt) {
+            const int4 old = *reinterpret_cast<const int4 *>(din + lo + i);
+            int4 *mp = reinterpret_cast<int4 *>(p.q.ptmp + (lo - p.g.v0) + i);
+            int4 m;
+            asm volatile("ld.global.cg.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(m.x), "=r"(m.y), "=r"(m.z), "=r"(m.w) : "l"(mp));
+            if (m.x != INT32_MAX || m.y != INT32_MAX || m.z != INT32_MAX || m.w != INT32_MAX)
+                *mp = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX);
+            const int4 best = make_int4(min(old.x, m.x), min(old.y, m.y), min(old.z, m.z), min(old.w, m.w));
+            proact::put(lc, p.region_out, (uint64_t)(lo + i) * 4, best);
+            const int32_t ob[4] = {old.x, old.y, old.z, old.w}, bb[4] = {best.x, best.y, best.z, best.w};
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (bb[q] != ob[q]) {
+                    changed = true;
+                    cs += __ldg(p.g.outdeg + lo + i + q);
+                }
+        } else {
+            for (uint32_t j = i; j < nvt && j < i + 4; ++j) {
+                const uint32_t v = lo + j;
+                const int32_t old = din[v];
+                const int32_t m = ld_cg_i(p.q.ptmp + (v - p.g.v0));
+                if (m != INT32_MAX) p.q.ptmp[v - p.g.v0] = INT32_MAX;
+                const int32_t best = min(old, m);
+                proact::put(lc, p.region_out, (uint64_t)v * 4, best);
+                if (best != old) {
+                    changed = true;
+                    cs += __ldg(p.g.outdeg + v);
+                }
+            }
+        }
+        const int any = __syncthreads_or(changed);   // orders the block's puts before the commit
+        if (threadIdx.x == 0) {
+            const uint64_t off = (uint64_t)lo * 4;
+            const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
+            if (any) {
+                proact::mark_changed(lc, p.region_out, off);
+                proact::vote(lc);
+            }
+            if (any || prev) proact::mark_push(lc, p.region_out, off);
+            proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
+        }
+    }
+    count_changed(p, cs);
+}
+
+__global__ void push_count_kernel(const uint32_t *rowidx, uint64_t E, uint32_t *cnt)
+{
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E; e += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&cnt[rowidx[e]], 1u);
+}
+__global__ void push_scatter_kernel(const uint32_t *colptr, const uint32_t *rowidx, const int32_t *w, uint32_t nv,
+                                    uint32_t *cursor, uint32_t *pcol, int32_t *pwt)
+{
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < nv; v += gridDim.x * blockDim.x)
+        for (uint32_t e = colptr[v]; e < colptr[v + 1]; ++e) {
+            const uint32_t pos = atomicAdd(&cursor[rowidx[e]], 1u);
+            pcol[pos] = v;
+            pwt[pos] = w[e];
+        }
+}
+__global__ void push_heavy_count_kernel(const uint32_t *prp, uint32_t V, uint32_t *n)
+{
+    uint32_t c = 0;
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x)
+        c += prp[u + 1] - prp[u] > PUSH_HEAVY;
+    if (c) atomicAdd(n, c);
 }
 
 __global__ void pr_init_kernel(float *contrib, const uint32_t *outdeg, uint32_t V, float r0)
@@ -1450,6 +1787,45 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
             GCK(cudaFree(slot));
         }
     }
+    // SSSP push rounds (reading R24): my in-edges grouped by source, dprev, minima, heavy list
+    G.E_all = E;
+    if (d_w) {
+        GCK(cudaMalloc((void **)&G.prp, 4 * ((size_t)V + 1)));
+        GCK(cudaMalloc((void **)&G.pcol, 4 * std::max<uint64_t>(1, G.E_own)));
+        GCK(cudaMalloc((void **)&G.pwt, 4 * std::max<uint64_t>(1, G.E_own)));
+        GCK(cudaMalloc((void **)&G.dprev, 4 * (size_t)V));
+        GCK(cudaMalloc((void **)&G.ptmp, 4 * std::max<size_t>(1, G.nv)));
+        GCK(cudaMalloc((void **)&G.pctl, 16));
+        GCK(cudaMalloc((void **)&G.dcnt, 16));
+        GCK(cudaMallocHost((void **)&G.hcnt, 8));
+        *G.hcnt = 0ull;
+        GCK(cudaMemsetAsync(G.pctl, 0, 16, s));
+        GCK(cudaMemsetAsync(G.dcnt, 0, 16, s));
+        GCK(cudaMemsetAsync(G.dprev, 0x7F, 4 * (size_t)V, s));   // any value: round 0 rewrites it
+        uint32_t *cnt = nullptr, *nh = nullptr;
+        GCK(cudaMalloc((void **)&cnt, 4 * ((size_t)V + 1)));
+        GCK(cudaMalloc((void **)&nh, 4));
+        GCK(cudaMemsetAsync(cnt, 0, 4 * ((size_t)V + 1), s));
+        GCK(cudaMemsetAsync(nh, 0, 4, s));
+        if (G.E_own) push_count_kernel<<<1184, 256, 0, s>>>(G.rowidx, G.E_own, cnt);
+        GCK(cudaGetLastError());
+        rc = exclusive_scan(cnt, G.prp, (uint64_t)V + 1, s);
+        if (rc) return rc;
+        GCK(cudaMemcpyAsync(cnt, G.prp, 4 * ((size_t)V + 1), cudaMemcpyDeviceToDevice, s));   // cursors
+        if (G.nv) push_scatter_kernel<<<1184, 256, 0, s>>>(G.colptr, G.rowidx, G.w, G.nv, cnt, G.pcol, G.pwt);
+        push_heavy_count_kernel<<<1184, 256, 0, s>>>(G.prp, V, nh);
+        GCK(cudaGetLastError());
+        GCK(cudaMemcpyAsync(&G.nheavy_max, nh, 4, cudaMemcpyDeviceToHost, s));
+        GCK(cudaStreamSynchronize(s));
+        GCK(cudaMalloc((void **)&G.heavy, 4 * std::max<uint32_t>(1, G.nheavy_max)));
+        GCK(cudaFree(cnt));
+        GCK(cudaFree(nh));
+        // ptmp must read INT32_MAX (0xFF.. is -1): set it properly
+        {
+            std::vector<int32_t> inf(std::max<size_t>(1, G.nv), INT32_MAX);
+            GCK(cudaMemcpy(G.ptmp, inf.data(), 4 * inf.size(), cudaMemcpyHostToDevice));
+        }
+    }
     GCK(cudaStreamSynchronize(s));
     {
         // the opt-in stays at the round-1 value (a 45056-entry table): besides allowing the launch,
@@ -1494,6 +1870,17 @@ int proact_graph_free(int id)
     cudaFree(G.runv_ph);
     if (G.rowidx_h) cudaFree(G.rowidx_h);
     if (G.hot_ids) cudaFree(G.hot_ids);
+    if (G.prp) {
+        cudaFree(G.prp);
+        cudaFree(G.pcol);
+        cudaFree(G.pwt);
+        cudaFree(G.dprev);
+        cudaFree(G.ptmp);
+        cudaFree(G.heavy);
+        cudaFree(G.pctl);
+        cudaFree(G.dcnt);
+        cudaFreeHost(G.hcnt);
+    }
     G = Graph();
     return PROACT_OK;
 }
@@ -1593,23 +1980,78 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     p.region_out = region_out;
     p.first = first ? 1 : 0;
     p.pad = 0;
+    // pull or push this round (reading R24).  PROACT_SSSP_PUSH: 0 = always pull, 1 = always push,
+    // unset = by the frontier: the out-degree sum of my vertices that changed last round, scaled
+    // to the whole graph (V / nv), below PROACT_SSSP_PUSH_PCT % (default 8) of the edges -> push.
+    // The counter is the previous round's (copied after its kernel; stale only if the caller did
+    // not synchronise -- either choice computes the same distances)
+    Graph &Gr = graphs[graph];
+    cudaStream_t s = (cudaStream_t)stream;
+    const char *pe = getenv("PROACT_SSSP_PUSH");
+    const int pmode = pe ? atoi(pe) : -1;
+    if (first) Gr.round = 0;
+    memset(&p.q, 0, sizeof(p.q));
+    // A push round needs dprev = the previous round's input: push rounds keep it, pull rounds
+    // only when asked (track) -- the copy costs a pass over V per round, so pull rounds track only
+    // once the frontier is below 4x the push threshold, and a round may push only if the round
+    // before it tracked.
+    bool push = false, track = false;
+    if (Gr.prp && pmode != 0) {
+        if (first) {
+            GCK(cudaMemsetAsync(Gr.dcnt, 0, 16, s));
+            push = true;   // the frontier is the source alone
+        } else if (pmode == 1) {
+            push = true;
+        } else {
+            const char *pp = getenv("PROACT_SSSP_PUSH_PCT");
+            const double pct = pp ? atof(pp) : 8.0;
+            const double est = 100.0 * (double)*Gr.hcnt * (double)Gr.V / (double)std::max(1u, Gr.nv);
+            push = Gr.tracked && est < pct * (double)Gr.E_all;
+            track = est < 4.0 * pct * (double)Gr.E_all;
+        }
+        p.q = PushDev{Gr.prp, Gr.pcol, Gr.pwt, Gr.dprev, Gr.ptmp, Gr.heavy, Gr.pctl, Gr.dcnt,
+                      track ? 1u : 0u, Gr.round & 1u};
+    }
+    Gr.tracked = push || track;
+    Gr.last_mode = push ? 1 : 0;
     launch_ctx lc;
     void *args[2] = {&lc, &p};
     int regs[1] = {region_out};
+    if (push) {
+        rc = proact_launch(regs, 1, (const void *)sssp_push_kernel, 0, PB, args, 0, stream);
+        if (rc) return rc;
+        GCK(cudaMemcpyAsync(Gr.hcnt, Gr.dcnt + p.q.par, 8, cudaMemcpyDeviceToHost, s));
+        Gr.round++;
+        return PROACT_OK;
+    }
     if (l2_window_on()) {
         proact_region_info ri;
         if (proact_region_info_get(region_in, &ri) == PROACT_OK)
             proact_internal_l2_window(ri.replica_base, ri.total_bytes);
     }
+    auto after = [&](int rc2) {
+        if (rc2 == PROACT_OK && p.q.dcnt) {
+            if (cudaMemcpyAsync(Gr.hcnt, Gr.dcnt + p.q.par, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+                return (int)PROACT_ERR_CUDA;
+            Gr.round++;
+        }
+        return rc2;
+    };
     const int cl = hot_cluster(p.g.nhot);
     if (cl > 0) {
         const void *k = cl == 1 ? (const void *)sssp_hot_kernel<1>
                       : cl == 2 ? (const void *)sssp_hot_kernel<2>
                       : cl == 4 ? (const void *)sssp_hot_kernel<4> : (const void *)sssp_hot_kernel<8>;
-        return proact_launch_ex(regs, 1, k, 0, GB * PG, args, 4 * ((size_t)PG * CPS + (cl == 1 ? p.g.nhot : HOT_SLICE)),
-                                stream, cl > 1 ? (unsigned)cl << PROACT_LAUNCH_CLUSTER_SHIFT : 0u);
+        return after(proact_launch_ex(regs, 1, k, 0, GB * PG, args, 4 * ((size_t)PG * CPS + (cl == 1 ? p.g.nhot : HOT_SLICE)),
+                                      stream, cl > 1 ? (unsigned)cl << PROACT_LAUNCH_CLUSTER_SHIFT : 0u));
     }
-    return proact_launch(regs, 1, (const void *)sssp_kernel, 0, GB, args, 0, stream);
+    return after(proact_launch(regs, 1, (const void *)sssp_kernel, 0, GB, args, 0, stream));
+}
+
+int proact_sssp_last_mode(int graph)
+{
+    if (graph < 0 || graph >= MAXGRAPH || !graphs[graph].used) return PROACT_ERR_INVALID;
+    return graphs[graph].last_mode;
 }
 
 // Force-load this translation unit's kernels (see proact_internal_preload_workloads).
@@ -1623,7 +2065,9 @@ __attribute__((visibility("hidden"))) int proact_internal_preload_graph(void)
                        (const void *)pagerank_hot_kernel<4>, (const void *)pagerank_hot_kernel<8>,
                        (const void *)hot_slot_kernel, (const void *)hot_encode_kernel,
                        (const void *)sssp_hot_kernel<1>, (const void *)sssp_hot_kernel<2>,
-                       (const void *)sssp_hot_kernel<4>, (const void *)sssp_hot_kernel<8>};
+                       (const void *)sssp_hot_kernel<4>, (const void *)sssp_hot_kernel<8>,
+                       (const void *)sssp_push_kernel, (const void *)push_count_kernel,
+                       (const void *)push_scatter_kernel, (const void *)push_heavy_count_kernel};
     for (const void *f : k)
         if (cudaFuncGetAttributes(&a, f) != cudaSuccess) return PROACT_ERR_CUDA;
     return PROACT_OK;

@@ -360,5 +360,10 @@ class SSSP(_Graph):
         return cap
 
     @property
+    def last_mode(self) -> int:
+        """0 if the last round pulled over every in-edge, 1 if it pushed from the frontier (R24)."""
+        return rt.lib().proact_sssp_last_mode(self.gid)
+
+    @property
     def current(self) -> torch.Tensor:
         return self.bufs[self.k & 1]

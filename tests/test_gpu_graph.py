@@ -5,6 +5,8 @@ fp64-accumulating oracle (reading R12); both sides round r to fp32 once per iter
 SSSP: int32 distances bit-exact and the same number of rounds (reading R13).
 Graphs: synthetic RMAT (stand-in for Wikipedia / HV15R).
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -239,6 +241,71 @@ def test_sssp_reset_reruns_identically():
     for runs in run_ranks(2, _sssp_rerun_body, V, src, dst, w, s0, 4096):
         for rounds, d in runs:
             assert rounds == want_rounds and np.array_equal(d, want)
+
+
+def _sssp_modes_body(r, G, V, src, dst, w, s0, chunk, mech, hot, reruns=1):
+    rt.set_config(mech=mech)
+    st = torch.cuda.Stream()
+    S = wl.SSSP(V, src, dst, w, s0, chunk, stream=st, hot=hot)
+    out = []
+    for _ in range(reruns):
+        S.reset()
+        rt.host_barrier()
+        modes = []
+        while True:
+            more = S.step(st)
+            modes.append(S.last_mode)
+            if not more:
+                break
+        out.append((len(modes), modes, S.current.cpu().numpy().copy()))
+    rt.check_device()
+    S.free()
+    return out
+
+
+@pytest.mark.parametrize("push", ["1", "auto"])
+@pytest.mark.parametrize("G,scale,chunk,mech,hot", [(1, 12, 4096, _lib.MECH_FUSED, -1),
+                                                    (2, 13, 4096, _lib.MECH_FUSED, 0),
+                                                    (3, 12, 8192, _lib.MECH_FUSED, 97),
+                                                    (2, 12, 4096, _lib.MECH_INLINE, -1),
+                                                    (2, 12, 4096, _lib.MECH_BULK, -1),
+                                                    (2, 12, 4096, _lib.MECH_DMA, -1),
+                                                    (4, 14, 16384, _lib.MECH_FUSED, 1000)])
+def test_sssp_push_rounds_match_oracle(G, scale, chunk, mech, hot, push):
+    """Push rounds (reading R24: only the sources whose distance changed in the previous round
+    relax their edges into my vertices) give the oracle's distances and round count bit-exactly,
+    always-push and auto (pull while the frontier is large), on every rank's full replica; a
+    rerun after reset() (dprev then holds the previous run's last input) is identical."""
+    src, dst = synth.rmat(scale, 16)
+    V = 1 << scale
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
+    os.environ["PROACT_SSSP_PUSH"] = push if push != "auto" else "-1"
+    try:
+        outs = run_ranks(G, _sssp_modes_body, V, src, dst, w, s0, chunk, mech, hot, 2)
+    finally:
+        os.environ.pop("PROACT_SSSP_PUSH", None)
+    for runs in outs:
+        for rounds, modes, d in runs:
+            assert rounds == want_rounds
+            assert np.array_equal(d, want)
+            assert modes[0] == 1                       # round 0: the frontier is the source
+            if push == "1":
+                assert all(m == 1 for m in modes)
+
+
+def test_sssp_auto_switches_pull_and_push():
+    """Auto mode on RMAT-14: the large middle rounds pull, the first and the late rounds push."""
+    src, dst = synth.rmat(14, 16)
+    V = 1 << 14
+    w = synth.weights(src.size)
+    s0 = int(np.bincount(src, minlength=V).argmax())
+    want, want_rounds, _ = oracle.sssp(V, src, dst, w, s0)
+    (runs,) = run_ranks(1, _sssp_modes_body, V, src, dst, w, s0, 4096, _lib.MECH_FUSED, -1)
+    rounds, modes, d = runs[0]
+    assert rounds == want_rounds and np.array_equal(d, want)
+    assert 0 in modes and modes[0] == 1 and modes[-1] == 1, modes
 
 
 def test_votes_are_epoch_tagged():

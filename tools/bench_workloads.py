@@ -166,8 +166,9 @@ def sssp(args, src, dst, V):
         cv = args.chunk // 4
         nch = (V + cv - 1) // cv
         prev = S.current.clone()
-        kern, algs, k = [], [], 0
+        kern, algs, modes, k = [], [], [], 0
         dirty = None
+        front = None   # vertices whose distance changed in the previous round (push frontier)
         while True:
             a, b = ev(), ev()
             i = S.k & 1
@@ -178,17 +179,25 @@ def sssp(args, src, dst, V):
             S.k += 1
             st.synchronize()
             kern.append(a.elapsed_time(b))
-            de = S.e_own if dirty is None else int(epc[dirty].sum())
-            algs.append(4.0 * S.e_own + 8.0 * de + 12.0 * (S.v1 - S.v0))
+            mode = S.last_mode
+            modes.append(mode)
+            if mode == 0:   # pull (reading R13)
+                de = S.e_own if dirty is None else int(epc[dirty].sum())
+                algs.append(4.0 * S.e_own + 8.0 * de + 12.0 * (S.v1 - S.v0))
+            else:           # push (reading R24): scan input + dprev, frontier out-edges, my vertices
+                fe = int(outdeg[s0]) if front is None else int(outdeg[front].sum())
+                algs.append(8.0 * V + 12.0 * fe + 12.0 * (S.v1 - S.v0))
             cur = S.current
             pad = nch * cv - V
-            diff = torch.nn.functional.pad((cur != prev).to(torch.int32), (0, pad))
+            chg = cur != prev
+            diff = torch.nn.functional.pad(chg.to(torch.int32), (0, pad))
             dirty = (diff.view(nch, cv).sum(1) > 0).cpu().numpy()
+            front = chg.cpu().numpy()
             prev = cur.clone()
             k += 1
             if rt.last_vote() == 0 or k >= V:
                 break
-        out = {"rounds": rounds, "t": sum(times[args.warmup:]), "kern_ms": kern, "alg": algs,
+        out = {"rounds": rounds, "t": sum(times[args.warmup:]), "kern_ms": kern, "alg": algs, "modes": modes,
                "nhot": S.nhot, "e_own": S.e_own}
         if G == 1:   # tracking overhead: a whole run under ELIDE vs LOCAL
             oh = {}
@@ -206,6 +215,7 @@ def sssp(args, src, dst, V):
         S.free()
         return out
     epc = np.bincount(src // (args.chunk // 4), minlength=(V + args.chunk // 4 - 1) // (args.chunk // 4))
+    outdeg = np.bincount(src, minlength=V)   # G = 1 roofline: every out-edge lands on this rank
     res = run_ranks(args.ranks, body)
     t = max(r["t"] for r in res)
     rounds = res[0]["rounds"]
@@ -223,12 +233,14 @@ def sssp(args, src, dst, V):
     if args.ranks == 1:
         r0 = res[0]
         kms, alg = sum(r0["kern_ms"]), sum(r0["alg"])
-        line["roofline"] = {"bound": "hbm", "kernel": "sssp_hot_kernel" if r0["nhot"] else "sssp_kernel",
+        line["roofline"] = {"bound": "hbm", "kernel": ("sssp_hot_kernel" if r0["nhot"] else "sssp_kernel") + " / sssp_push_kernel",
                             "kernel_ms_per_round": [round(x, 4) for x in r0["kern_ms"]],
+                            "mode_per_round": ["push" if m else "pull" for m in r0["modes"]],
                             "alg_bytes_per_run": alg, "achieved": alg / kms / 1e6, "peak": peak_hbm(),
                             "unit": "GB/s", "frac": alg / kms / 1e6 / peak_hbm(),
-                            "note": "4 B/in-edge scanned + 8 B/in-edge of a changed source chunk + 12 B/vertex "
-                                    "per round, summed over the run / summed kernel time"}
+                            "note": "pull round: 4 B/in-edge scanned + 8 B/in-edge of a changed source chunk + 12 B/vertex; "
+                                    "push round (R24): 8 B/vertex of the graph (input + previous input) + 12 B per "
+                                    "frontier out-edge + 12 B/vertex of mine; summed over the run / summed kernel time"}
     if not args.no_cpu:
         import oracle
         tm = {}
