@@ -571,19 +571,27 @@ def main():
     # P2P stores): iterations/s of the same step with each mechanism, N > 1 only (at N = 1
     # there is nothing to move and every mechanism is the plain kernel)
     baselines = None
-    if world > 1 and not args.no_baselines:
-        baselines = {}
-        kk = max(2, args.steps // 2)
-        legs = [("bulk_cudaMemcpyPeer", _lib.MECH_BULK, False), ("naive_p2p_inline", _lib.MECH_INLINE, False)]
-        if dist.get_backend() == "nccl":
-            legs.append(("nccl_allgather", _lib.MECH_LOCAL, True))
-        for name, m, use_nccl in legs:
-            rt.set_config(mech=m)
-            mode["nccl"] = use_nccl
-            step()
-            baselines[name] = kk * I / (timed(step, kk) / 1000.0)
+    try:   # an optional leg: a failure is reported in the line, not fatal to it
+        if world > 1 and not args.no_baselines:
+            baselines = {}
+            kk = max(2, args.steps // 2)
+            legs = [("bulk_cudaMemcpyPeer", _lib.MECH_BULK, False), ("naive_p2p_inline", _lib.MECH_INLINE, False)]
+            if dist.get_backend() == "nccl":
+                legs.append(("nccl_allgather", _lib.MECH_LOCAL, True))
+            for name, m, use_nccl in legs:
+                rt.set_config(mech=m)
+                mode["nccl"] = use_nccl
+                step()
+                baselines[name] = kk * I / (timed(step, kk) / 1000.0)
+            mode["nccl"] = nccl_base
+            rt.set_config(mech=mech)
+    except Exception as ex:   # noqa: BLE001
+        baselines = {"error": f"{type(ex).__name__}: {ex}"[:300]}
         mode["nccl"] = nccl_base
-        rt.set_config(mech=mech)
+        try:
+            rt.set_config(mech=mech)
+        except Exception:   # noqa: BLE001
+            pass
 
     # ---- NEXT-1, the paper's decomposition (Sec. V-C; Fig. 8/9) on the same
     # ranks: LOCAL = no transfer at all and no waits (the infinite-bandwidth bound; replicas go
@@ -591,87 +599,103 @@ def main():
     # = transfers after the kernel.  opportunity = T_bulk - T_local; captured = (T_bulk - T_proact)
     # / opportunity; overlap = captured with the tracking overhead added back
     decomposition = None
-    if world > 1 and not args.no_baselines and baselines and mech in (_lib.MECH_FUSED, _lib.MECH_ELIDE):
-        kk = max(2, args.steps // 2)
-        dv = {}
-        for name, m in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE)):
-            rt.set_config(mech=m)
-            step()
-            dv[name] = timed(step, kk) / (kk * I)   # ms per phase
-        rt.set_config(mech=mech)
-        t_p = ms / (args.steps * I)
-        t_b = 1000.0 / baselines["bulk_cudaMemcpyPeer"]
-        opp = t_b - dv["local"]
-        decomposition = {"ms_per_phase": {"proact": t_p, "bulk": t_b, "local_no_transfer": dv["local"],
-                                          "elide_tracking_only": dv["elide"]},
-                         "tracking_overhead_frac": dv["elide"] / dv["local"] - 1.0,
-                         "opportunity_ms": opp,
-                         "opportunity_captured": (t_b - t_p) / opp if opp > 0 else None,
-                         "overlap_frac": (t_b - t_p + dv["elide"] - dv["local"]) / opp if opp > 0 else None,
-                         "note": "paper Sec. V-C: infinite-BW bound = LOCAL, tracking overhead = ELIDE vs LOCAL"}
+    try:   # an optional leg: a failure is reported in the line, not fatal to it
+        if world > 1 and not args.no_baselines and baselines and mech in (_lib.MECH_FUSED, _lib.MECH_ELIDE):
+            kk = max(2, args.steps // 2)
+            dv = {}
+            for name, m in (("local", _lib.MECH_LOCAL), ("elide", _lib.MECH_ELIDE)):
+                rt.set_config(mech=m)
+                step()
+                dv[name] = timed(step, kk) / (kk * I)   # ms per phase
+            rt.set_config(mech=mech)
+            t_p = ms / (args.steps * I)
+            t_b = 1000.0 / baselines["bulk_cudaMemcpyPeer"]
+            opp = t_b - dv["local"]
+            decomposition = {"ms_per_phase": {"proact": t_p, "bulk": t_b, "local_no_transfer": dv["local"],
+                                              "elide_tracking_only": dv["elide"]},
+                             "tracking_overhead_frac": dv["elide"] / dv["local"] - 1.0,
+                             "opportunity_ms": opp,
+                             "opportunity_captured": (t_b - t_p) / opp if opp > 0 else None,
+                             "overlap_frac": (t_b - t_p + dv["elide"] - dv["local"]) / opp if opp > 0 else None,
+                             "note": "paper Sec. V-C: infinite-BW bound = LOCAL, tracking overhead = ELIDE vs LOCAL"}
+    except Exception as ex:   # noqa: BLE001
+        decomposition = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+        mode["nccl"] = nccl_base
+        try:
+            rt.set_config(mech=mech)
+        except Exception:   # noqa: BLE001
+            pass
 
     # ---- halo-only variant (reading R8: the one config-2 variant whose roofline allows
     # >= 6x at G = 8): per-chunk destinations = the neighbours; PROACT (tuned) and the baselines
     halo = None
-    if world > 1 and not args.no_halo:
-        J.set_halo_only()
-        kk = max(2, args.steps // 2)
-        # the halo exchange moves two rows per rank: the profiler picks again, over few agent warps
-        # (chunks bound nowhere never reach the agent) and the producer-CTA placement
-        full_cfg = rt.get_config()
-        halo_tuned = None
-        if tuned is not None:
-            def run_halo(c):
-                if c["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
-                    for rid in J.rid:
-                        rt.rechunk(rid, c["chunk_bytes"])
-                    J.set_halo_only()   # rechunk drops per-chunk destinations
-                for _ in range(3):
-                    J.step(s)
-                ts = []
-                for _ in range(5):
-                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    a.record(s)
-                    J.step(s, barrier=True)
-                    b.record(s)
-                    s.synchronize()
-                    ts.append(a.elapsed_time(b))
-                return statistics.median(ts)
+    try:   # an optional leg: a failure is reported in the line, not fatal to it
+        if world > 1 and not args.no_halo:
+            J.set_halo_only()
+            kk = max(2, args.steps // 2)
+            # the halo exchange moves two rows per rank: the profiler picks again, over few agent warps
+            # (chunks bound nowhere never reach the agent) and the producer-CTA placement
+            full_cfg = rt.get_config()
+            halo_tuned = None
+            if tuned is not None:
+                def run_halo(c):
+                    if c["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+                        for rid in J.rid:
+                            rt.rechunk(rid, c["chunk_bytes"])
+                        J.set_halo_only()   # rechunk drops per-chunk destinations
+                    for _ in range(3):
+                        J.step(s)
+                    ts = []
+                    for _ in range(5):
+                        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        a.record(s)
+                        J.step(s, barrier=True)
+                        b.record(s)
+                        s.synchronize()
+                        ts.append(a.elapsed_time(b))
+                    return statistics.median(ts)
 
-            hspace = "mech=0;chunk=131072,1048576;warps=1,2,4;push=0,1;akern=0,1,2"
-            hb = rt.autotune(f"bench_jacobi_halo_N{N}_G{world}", run_halo, hspace)
-            if hb["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
-                for rid in J.rid:
-                    rt.rechunk(rid, hb["chunk_bytes"])
-                J.set_halo_only()
-            rt.set_config(agent_warps=hb["agent_warps"], push=hb["push"], agent_kernel=hb["agent_kernel"])
-            halo_tuned = {"space": hspace, "best": {k: hb[k] for k in ("chunk_bytes", "agent_warps", "push",
-                                                                     "agent_kernel")}}
-        legs = [("proact", mech), ("bulk_cudaMemcpyPeer", _lib.MECH_BULK), ("naive_p2p_inline", _lib.MECH_INLINE)]
-        hv = {}
-        for name, m in legs:
-            rt.set_config(mech=m)
-            mode["nccl"] = False
-            step()
-            hv[name] = kk * I / (timed(step, kk) / 1000.0)
+                hspace = "mech=0;chunk=131072,1048576;warps=1,2,4;push=0,1;akern=0,1,2"
+                hb = rt.autotune(f"bench_jacobi_halo_N{N}_G{world}", run_halo, hspace)
+                if hb["chunk_bytes"] != rt.region_info(J.rid[0]).chunk_bytes:
+                    for rid in J.rid:
+                        rt.rechunk(rid, hb["chunk_bytes"])
+                    J.set_halo_only()
+                rt.set_config(agent_warps=hb["agent_warps"], push=hb["push"], agent_kernel=hb["agent_kernel"])
+                halo_tuned = {"space": hspace, "best": {k: hb[k] for k in ("chunk_bytes", "agent_warps", "push",
+                                                                         "agent_kernel")}}
+            legs = [("proact", mech), ("bulk_cudaMemcpyPeer", _lib.MECH_BULK), ("naive_p2p_inline", _lib.MECH_INLINE)]
+            hv = {}
+            for name, m in legs:
+                rt.set_config(mech=m)
+                mode["nccl"] = False
+                step()
+                hv[name] = kk * I / (timed(step, kk) / 1000.0)
+            mode["nccl"] = nccl_base
+            rt.set_config(mech=mech, agent_warps=full_cfg["agent_warps"], push=full_cfg["push"],
+                          agent_kernel=full_cfg["agent_kernel"])
+            h_rows = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
+            h_ingress = 4.0 * N * max(1, h_rows) if world > 1 else 0.0
+            ht = 1000.0 / hv["proact"] * 1000.0   # us per phase
+            h_nvl = h_ingress / (NVL * 1e9) * 1e6
+            halo = {"value": hv["proact"], "unit": "iters/s", "tuned": halo_tuned,
+                    "baselines_iters_per_s": {k: v for k, v in hv.items() if k != "proact"},
+                    "speedup_vs_n1": None,
+                    "step_roofline": {"t_hbm_us": t_hbm_us, "t_nvl_us": h_nvl, "t_phase_us": ht,
+                                      "frac": max(t_hbm_us, h_nvl) / ht,
+                                      "nvlink_ingress_GBps_per_gpu": h_ingress / (ht * 1e-6) / 1e9},
+                    "note": "per-chunk destinations = neighbours (boundary rows only); rows other ranks own "
+                            "are not replicated"}
+    except Exception as ex:   # noqa: BLE001
+        halo = {"error": f"{type(ex).__name__}: {ex}"[:300]}
         mode["nccl"] = nccl_base
-        rt.set_config(mech=mech, agent_warps=full_cfg["agent_warps"], push=full_cfg["push"],
-                      agent_kernel=full_cfg["agent_kernel"])
-        h_rows = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
-        h_ingress = 4.0 * N * max(1, h_rows) if world > 1 else 0.0
-        ht = 1000.0 / hv["proact"] * 1000.0   # us per phase
-        h_nvl = h_ingress / (NVL * 1e9) * 1e6
-        halo = {"value": hv["proact"], "unit": "iters/s", "tuned": halo_tuned,
-                "baselines_iters_per_s": {k: v for k, v in hv.items() if k != "proact"},
-                "speedup_vs_n1": None,
-                "step_roofline": {"t_hbm_us": t_hbm_us, "t_nvl_us": h_nvl, "t_phase_us": ht,
-                                  "frac": max(t_hbm_us, h_nvl) / ht,
-                                  "nvlink_ingress_GBps_per_gpu": h_ingress / (ht * 1e-6) / 1e9},
-                "note": "per-chunk destinations = neighbours (boundary rows only); rows other ranks own "
-                        "are not replicated"}
+        try:
+            rt.set_config(mech=mech)
+        except Exception:   # noqa: BLE001
+            pass
 
     n1_value = (2 * I / (n1_ms / 1000.0)) if n1_ms else (value if world == 1 else None)
-    if halo is not None and n1_value:
+    if halo is not None and n1_value and "value" in halo:
         halo["speedup_vs_n1"] = halo["value"] / n1_value
     # transfer-agent cost: SMs dedicated to the agent x phase time per GB pushed
     egress_gb = 4.0 * N * nrows * (world - 1) / 1e9
@@ -686,38 +710,46 @@ def main():
 
     # ---- e2e through the C-ABI host-buffer entry point
     e2e = None
-    if not args.no_e2e:
-        xh = torch.from_numpy(synth.jacobi_init(N)).pin_memory()
-        out = torch.empty((N, N), dtype=torch.float32).pin_memory()
-        nb = [0, 0]
+    try:   # an optional leg: a failure is reported in the line, not fatal to it
+        if not args.no_e2e:
+            xh = torch.from_numpy(synth.jacobi_init(N)).pin_memory()
+            out = torch.empty((N, N), dtype=torch.float32).pin_memory()
+            nb = [0, 0]
 
-        def e2e_step():
-            h, d = wl.jacobi_solve_host(xh, out, N, I, chunk, args.rpt, s)
-            nb[0], nb[1] = h, d
+            def e2e_step():
+                h, d = wl.jacobi_solve_host(xh, out, N, I, chunk, args.rpt, s)
+                nb[0], nb[1] = h, d
 
-        e2e_step()
-        torch.cuda.synchronize()
-        ems = timed(e2e_step, max(2, min(args.steps, 3)))
-        seq = max(2, min(args.steps, 3)) * I / (ems / 1000.0)
-        # the pipelined entry point: K solves (steps), each with its own H2D of the input and D2H
-        # of its result inside the timed region, solve k's phases overlapping the copies of k +- 1
-        outs = [out, torch.empty((N, N), dtype=torch.float32).pin_memory()]
-        # a stream of K solves: the first H2D and the last D2H (each ~19 ms over PCIe, measured
-        # full duplex by tools/probes/pcie_duplex.py) cannot overlap compute; K amortises them
-        K = max(4, min(2 * args.steps, 20))
+            e2e_step()
+            torch.cuda.synchronize()
+            ems = timed(e2e_step, max(2, min(args.steps, 3)))
+            seq = max(2, min(args.steps, 3)) * I / (ems / 1000.0)
+            # the pipelined entry point: K solves (steps), each with its own H2D of the input and D2H
+            # of its result inside the timed region, solve k's phases overlapping the copies of k +- 1
+            outs = [out, torch.empty((N, N), dtype=torch.float32).pin_memory()]
+            # a stream of K solves: the first H2D and the last D2H (each ~19 ms over PCIe, measured
+            # full duplex by tools/probes/pcie_duplex.py) cannot overlap compute; K amortises them
+            K = max(4, min(2 * args.steps, 20))
 
-        def e2e_pipe(k):
-            h, d = wl.jacobi_solve_host_pipelined(xh, [outs[j & 1] for j in range(k)], N, I, chunk, args.rpt, s)
-            nb[0], nb[1] = h, d
+            def e2e_pipe(k):
+                h, d = wl.jacobi_solve_host_pipelined(xh, [outs[j & 1] for j in range(k)], N, I, chunk, args.rpt, s)
+                nb[0], nb[1] = h, d
 
-        e2e_pipe(2)
-        torch.cuda.synchronize()
-        pms = timed(lambda: e2e_pipe(K), 1)
-        e2e = {"value": K * I / (pms / 1000.0), "unit": "iters/s",
-               "h2d_bytes_per_step": nb[0], "d2h_bytes_per_step": nb[1],
-               "api": "proact_jacobi_solve_host_pipelined", "steps": K,
-               "sequential_value": seq, "sequential_api": "proact_jacobi_solve_host"}
-        del xh, out, outs   # 3 GiB of pinned host memory: release before the secondary legs
+            e2e_pipe(2)
+            torch.cuda.synchronize()
+            pms = timed(lambda: e2e_pipe(K), 1)
+            e2e = {"value": K * I / (pms / 1000.0), "unit": "iters/s",
+                   "h2d_bytes_per_step": nb[0], "d2h_bytes_per_step": nb[1],
+                   "api": "proact_jacobi_solve_host_pipelined", "steps": K,
+                   "sequential_value": seq, "sequential_api": "proact_jacobi_solve_host"}
+            del xh, out, outs   # 3 GiB of pinned host memory: release before the secondary legs
+    except Exception as ex:   # noqa: BLE001
+        e2e = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+        mode["nccl"] = nccl_base
+        try:
+            rt.set_config(mech=mech)
+        except Exception:   # noqa: BLE001
+            pass
 
     line = None
     if rank == 0:
