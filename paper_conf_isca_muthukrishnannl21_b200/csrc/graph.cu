@@ -113,9 +113,9 @@ struct Graph {
     int32_t *pwt = nullptr;                // [E_own] weight
     int32_t *dprev = nullptr;              // [V] previous round's input distances
     int32_t *ptmp = nullptr;               // [nv] minima of the round, INT32_MAX between rounds
-    uint32_t *heavy = nullptr;             // [nheavy_max] frontier sources with > PUSH_HEAVY edges here
+    uint2 *heavy = nullptr;                // [nheavy_max] pieces (source, first edge) of heavy frontier sources
     uint32_t nheavy_max = 0;
-    uint32_t *pctl = nullptr;              // [4]: heavy count, barrier arrivals, barrier generation
+    uint32_t *pctl = nullptr;              // [4]: heavy pieces, barrier arrivals, barrier generation, claims
     unsigned long long *dcnt = nullptr;    // [2] per round parity: out-degree sum of my changed vertices
     unsigned long long *hcnt = nullptr;    // pinned: the last round's sum (read for the next decision)
     uint32_t round = 0;
@@ -337,7 +337,8 @@ struct PushDev {
     const uint32_t *prp, *pcol;
     const int32_t *pwt;
     int32_t *dprev, *ptmp;
-    uint32_t *heavy, *pctl;
+    uint2 *heavy;
+    uint32_t *pctl;
     unsigned long long *dcnt;
     uint32_t track, par;   // track: pull kernels keep dprev current this round
 };
@@ -868,7 +869,8 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
 }
 
 // Helpers of the SSSP push rounds (reading R24; see sssp_push_kernel) shared with the pull kernels.
-constexpr uint32_t PUSH_HEAVY = 1024;   // frontier sources with more edges here: spread over the grid
+constexpr uint32_t PUSH_HEAVY = 1024;   // frontier sources with more edges here: queued as pieces
+constexpr uint32_t PUSH_PIECE = 4096;   // edges per heavy piece (one CTA claims a piece)
 constexpr uint32_t PB = 256;            // threads per push-round CTA (x 4 vertices = one 4 KiB block)
 
 __device__ __forceinline__ int32_t ld_cg_i(const int32_t *p)
@@ -1335,7 +1337,10 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
 // frontier is found by comparing the arrived input with a PRIVATE copy of the previous input
 // (dprev, kept current in every round): the output replica itself cannot serve, peers' agents
 // already write this round's chunks into it.
-__global__ void __launch_bounds__(PB, 4) sssp_push_kernel(launch_ctx lc, SsspParams p)
+#ifndef PROACT_PUSH_MINB
+#define PROACT_PUSH_MINB 6   // push-round CTAs per SM (r02s sweep: 6 > 4 > 8, latency-bound loops)
+#endif
+__global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_ctx lc, SsspParams p)
 {
     if (proact::agent_dispatch(lc)) return;
     const region_dev &Ri = lc.ctx->region[p.region_in];
@@ -1361,8 +1366,10 @@ __global__ void __launch_bounds__(PB, 4) sssp_push_kernel(launch_ctx lc, SsspPar
             if ((p.first || du != dp) && du != INT32_MAX) {
                 e0 = __ldg(p.q.prp + u);
                 e1 = __ldg(p.q.prp + u + 1);
-                if (e1 - e0 > PUSH_HEAVY) {
-                    p.q.heavy[atomicAdd(&p.q.pctl[0], 1u)] = (uint32_t)u;
+                if (e1 - e0 > PUSH_HEAVY) {   // pieces of PUSH_PIECE edges, claimed by CTAs in step 2
+                    const uint32_t np = (e1 - e0 + PUSH_PIECE - 1) / PUSH_PIECE;
+                    const uint32_t k0 = atomicAdd(&p.q.pctl[0], np);
+                    for (uint32_t k = 0; k < np; ++k) p.q.heavy[k0 + k] = make_uint2((uint32_t)u, e0 + k * PUSH_PIECE);
                     e1 = e0;
                 }
             }
@@ -1455,19 +1462,28 @@ __global__ void __launch_bounds__(PB, 4) sssp_push_kernel(launch_ctx lc, SsspPar
             }
     }
     if (!grid_barrier(lc, p.q.pctl)) return;
-    // 2. heavy frontier sources: their edges spread over every producer thread
+    // 2. heavy frontier sources, in pieces of PUSH_PIECE edges claimed dynamically by CTAs (a
+    //    piece's edges: one per thread, independent loads)
     {
+        __shared__ uint32_t hk;
         const uint32_t nh = __ldcg(p.q.pctl);
-        const uint64_t gt = (uint64_t)pb * PB + threadIdx.x, GTH = (uint64_t)P * PB;
-        for (uint32_t h = 0; h < nh; ++h) {
-            const uint32_t u = __ldcg(p.q.heavy + h);
-            const int32_t du = din[u];
-            const uint32_t a = __ldg(p.q.prp + u), b = __ldg(p.q.prp + u + 1);
-            for (uint64_t e = a + gt; e < b; e += GTH) push_relax(p, (uint32_t)e, du);
+        for (;;) {
+            if (threadIdx.x == 0) hk = atomicAdd(&p.q.pctl[3], 1u);
+            __syncthreads();
+            const uint32_t k = hk;
+            __syncthreads();
+            if (k >= nh) break;
+            const uint2 pc = __ldcg(p.q.heavy + k);
+            const int32_t du = din[pc.x];
+            const uint32_t b = min(pc.y + PUSH_PIECE, __ldg(p.q.prp + pc.x + 1));
+            for (uint32_t e = pc.y + threadIdx.x; e < b; e += PB) push_relax(p, e, du);
         }
     }
     if (!grid_barrier(lc, p.q.pctl)) return;
-    if (pb == 0 && threadIdx.x == 0) p.q.pctl[0] = 0u;   // every CTA has read the heavy count
+    if (pb == 0 && threadIdx.x == 0) {   // every CTA has read the piece count and left its claims
+        p.q.pctl[0] = 0u;
+        p.q.pctl[3] = 0u;
+    }
     // 3. my vertices in blocks of 1024 (4 KiB, inside one chunk: chunks are multiples of 4 KiB
     //    and slices chunk-aligned), 4 per thread with 16-byte loads: d' = min(d, minima),
     //    instrumented stores, chunk state, vote, commit (a2, a3); the minima are reset to
@@ -1540,9 +1556,11 @@ __global__ void push_scatter_kernel(const uint32_t *colptr, const uint32_t *rowi
 }
 __global__ void push_heavy_count_kernel(const uint32_t *prp, uint32_t V, uint32_t *n)
 {
-    uint32_t c = 0;
-    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x)
-        c += prp[u + 1] - prp[u] > PUSH_HEAVY;
+    uint32_t c = 0;   // pieces of all sources that can be heavy
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < V; u += gridDim.x * blockDim.x) {
+        const uint32_t d = prp[u + 1] - prp[u];
+        if (d > PUSH_HEAVY) c += (d + PUSH_PIECE - 1) / PUSH_PIECE;
+    }
     if (c) atomicAdd(n, c);
 }
 
@@ -1817,7 +1835,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
         GCK(cudaGetLastError());
         GCK(cudaMemcpyAsync(&G.nheavy_max, nh, 4, cudaMemcpyDeviceToHost, s));
         GCK(cudaStreamSynchronize(s));
-        GCK(cudaMalloc((void **)&G.heavy, 4 * std::max<uint32_t>(1, G.nheavy_max)));
+        GCK(cudaMalloc((void **)&G.heavy, sizeof(uint2) * std::max<uint32_t>(1, G.nheavy_max)));
         GCK(cudaFree(cnt));
         GCK(cudaFree(nh));
         // ptmp must read INT32_MAX (0xFF.. is -1): set it properly
