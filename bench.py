@@ -18,7 +18,8 @@ same step with the uninstrumented LOCAL mechanism: the paper's tracking-overhead
 decomposition, Sec. V-C).  N = 1 also adds `secondary` (outside the timed
 region): config 2 on two loopback ranks of this GPU with every transfer mechanism (the
 PROACT path itself; at G = 1 nothing is replicated) and BASELINE.json configs 3-4
-(PageRank / SSSP, RMAT-24) with their rooflines and oracle baselines.
+(PageRank / SSSP, RMAT-24) with their rooflines and oracle baselines, and a config-5
+chunk sweep (transfer microbenchmark, the paper's Fig. 6 shape) on two loopback ranks.
 
 --impl reference: the CPU oracle (oracle/) timed as it stands on the host cores, on
 the same config/metric; rank 0 only under torchrun.
@@ -287,6 +288,27 @@ def secondary_legs(N: int, peak: float) -> dict:
         if "local_no_transfer" in ms and "bulk_cudaMemcpyPeer" in ms and best:
             opp = ms["bulk_cudaMemcpyPeer"] - ms["local_no_transfer"]
             out[leg]["opportunity_captured"] = ((ms["bulk_cudaMemcpyPeer"] - proact[best]) / opp) if opp > 0 else None
+            out[leg]["opportunity_note"] = ("(T_bulk - T_proact) / (T_bulk - T_local); above 1 = the PROACT phase ran "
+                                            "faster than the no-transfer LOCAL phase on these ranks (run-to-run noise "
+                                            "of a few us when the opportunity itself is a few us)")
+    # config 5 (transfer microbenchmark, the paper's Fig. 6 shape): chunk sweep, PROACT (producer
+    # placement) vs the baselines, two loopback ranks, R = 256 MiB, pure mode (K = 1)
+    e = dict(env, G="2", RBYTES=str(256 << 20), K="1", CHUNKS="4096,65536,1048576,4194304",
+             MECHS="fused,inline,bulk,dma", AKERNS="2", PUSHES="1", WARPS="8", PHASES="8")
+    pts = _json_lines([py, os.path.join(ROOT, "tools", "sweep_micro.py")], e, 600)
+    fig6 = {}
+    for p in pts:
+        if "error" in p:
+            fig6.setdefault("errors", []).append(p["error"])
+            continue
+        name = {"fused": "proact_producer_tile_push", "inline": "naive_p2p_inline", "bulk": "bulk_cudaMemcpyPeer",
+                "dma": "dma_copy_engine_program"}.get(p["mech"], p["mech"])
+        fig6.setdefault(str(p["chunk"]), {})[name] = p["ms"]
+    for ch, row in fig6.items():
+        if ch != "errors" and "proact_producer_tile_push" in row and "bulk_cudaMemcpyPeer" in row:
+            row["speedup_vs_bulk"] = row["bulk_cudaMemcpyPeer"] / row["proact_producer_tile_push"]
+    out["micro_fig6"] = {"ms_per_phase_by_chunk": fig6, "R_bytes": 256 << 20, "G": 2,
+                         "note": "BASELINE.json config 5 shape (all-gather of R, pure mode), loopback"}
     for wk in ("pagerank", "sssp"):
         pts = _json_lines([py, os.path.join(ROOT, "tools", "bench_workloads.py"), "--workload", wk,
                            "--steps", "3", "--warmup", "1"], env, 900)
