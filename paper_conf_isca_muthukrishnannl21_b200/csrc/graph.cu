@@ -69,6 +69,7 @@ struct Item {
     uint32_t run_pr;         // first entry of this item in runv_pr (PageRank runs of PR_RUN edges)
     uint32_t run_ss;         // first entry of this item in runv_ss (SSSP runs of SSSP_RUN edges)
     uint32_t run_ph;         // first entry of this item in runv_ph (hot-kernel runs of PRH_RUN edges)
+    uint32_t run_p8;         // first entry of this item in runv_p8 (PageRank hot runs of PRH_RUN_PR edges)
 };
 
 struct GraphDev {
@@ -84,6 +85,7 @@ struct GraphDev {
     const uint16_t *runv_pr;  // per PageRank run (RUN consecutive in-edges of an item): tile-local
     const uint16_t *runv_ss;  //   vertex of its first edge (the merge-path search, done once at build)
     const uint16_t *runv_ph;
+    const uint16_t *runv_p8;
     const uint32_t *rowidx_h; // [E_own] rowidx with hot sources encoded as HOT_BIT | slot (nhot > 0)
     const uint32_t *hot_ids;  // [nhot] the hot sources (highest out-degree), ascending ids
     uint32_t V, v0, nv, nitems, nhot;
@@ -101,7 +103,7 @@ struct Graph {
     unsigned long long *acc_f = nullptr;
     int32_t *acc_i = nullptr;
     uint32_t *acc_cnt = nullptr;
-    uint16_t *runv_pr = nullptr, *runv_ss = nullptr, *runv_ph = nullptr;
+    uint16_t *runv_pr = nullptr, *runv_ss = nullptr, *runv_ph = nullptr, *runv_p8 = nullptr;
     uint32_t *rowidx_h = nullptr, *hot_ids = nullptr;
     uint32_t nhot = 0;
     uint64_t e_hot = 0;   // my in-edges whose source is hot
@@ -174,6 +176,9 @@ __device__ __forceinline__ T hot_lookup(const T *hot, uint32_t hot_s, uint32_t m
 }
 #ifndef PROACT_PRH_PG
 #define PROACT_PRH_PG 4
+#endif
+#ifndef PROACT_PRH_RUN_PR   // pagerank_hot_kernel: consecutive in-edges per thread and run (4 or 8;
+#define PROACT_PRH_RUN_PR 4  // 16-byte index loads from a 4-edge-aligned base, RUN/4 of them)
 #endif
 #ifndef PROACT_PRH_RUN
 #define PROACT_PRH_RUN 4
@@ -463,9 +468,9 @@ __global__ void runv_kernel(const Item *items, const uint32_t *colptr, uint32_t 
     const Item it = items[blockIdx.x];
     const uint32_t lo = it.tile * GT, nvt = min(lo + GT, nv) - lo;
     // hot-kernel runs (which == 2, PRH_VEC) start at the 4-edge-aligned base below e0
-    const uint32_t b0 = which == 2 && PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0;
+    const uint32_t b0 = which >= 2 && PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0;
     const uint32_t nrun = (it.e1 - b0 + RUN - 1) / RUN;
-    const uint32_t off = which == 2 ? it.run_ph : which ? it.run_ss : it.run_pr;
+    const uint32_t off = which == 3 ? it.run_p8 : which == 2 ? it.run_ph : which ? it.run_ss : it.run_pr;
     for (uint32_t j = threadIdx.x; j < nrun; j += blockDim.x)
         runv[off + j] = (uint16_t)vertex_of(colptr + lo, nvt, max(it.e0, b0 + j * RUN));
 }
@@ -502,6 +507,29 @@ __device__ __forceinline__ bool split_arrive(const GraphDev &g, const Item &it, 
 // bit-reproducible for any schedule; r' = (float)((1-d)/V + d * sum) as in the oracle (R12).
 constexpr double FIX = 4611686018427387904.0;          // 2^62
 constexpr double UNFIX = 1.0 / 4611686018427387904.0;  // 2^-62
+#ifndef PROACT_PR_FIX_INT
+#define PROACT_PR_FIX_INT 0   // 1: integer rounding (bit-identical; measured no faster: 1.053 vs 1.044 ms)
+#endif
+// round(g * 2^62) to nearest, ties to even, for an fp32 contribution 0 <= g < 1 -- the value
+// __double2ll_rn((double)g * 2^62) computes, from the float's bits with integer ALU operations only
+// (no fp32 -> fp64 -> s64 conversions, which share the slower conversion pipe, per edge)
+__device__ __forceinline__ unsigned long long fix62(float g)
+{
+#if PROACT_PR_FIX_INT
+    const uint32_t b = __float_as_uint(g);
+    const int ex = (int)(b >> 23);                      // biased exponent (sign bit 0: g >= 0)
+    if (ex == 0) return 0ull;                           // 0 and denormals: below 2^-126 * 2^62 < 1/2
+    const unsigned long long m = (b & 0x7FFFFFu) | 0x800000u;
+    const int sh = ex - 127 - 23 + 62;                  // g * 2^62 = m * 2^sh
+    if (sh >= 0) return m << sh;
+    const int r = -sh;
+    if (r > 24) return 0ull;                            // m * 2^-r < 2^24 * 2^-25 = 1/2
+    const unsigned long long q = m >> r, rem = m & ((1ull << r) - 1ull), half = 1ull << (r - 1);
+    return q + ((rem > half || (rem == half && (q & 1ull))) ? 1ull : 0ull);
+#else
+    return (unsigned long long)__double2ll_rn((double)g * FIX);
+#endif
+}
 
 __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx lc, PrParams p)
 {
@@ -566,7 +594,7 @@ __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx
                         sum = 0ull;
                         nxt = cp[++i + 1];
                     }
-                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
+                    sum += fix62(g[q]);
                 }
             }
             // hub fast path: every lane active, single-vertex runs, the same vertex
@@ -636,7 +664,7 @@ __device__ __forceinline__ uint32_t claim_group(const launch_ctx &lc, uint32_t n
 template <int CL>
 __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(launch_ctx lc, PrParams p)
 {
-    constexpr int RUN = PROACT_PRH_RUN;
+    constexpr int RUN = PROACT_PRH_RUN_PR;
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
     __shared__ uint32_t acc_lo_a[PG][GT], acc_hi_a[PG][GT];
@@ -688,22 +716,25 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         // trip instead of two
         uint32_t xn[RUN], in_ = 0;
 #if PROACT_PRH_VEC
-        static_assert(PROACT_PRH_RUN == 4, "PRH_VEC loads one run of 4 edges as 16 bytes");
+        static_assert(RUN % 4 == 0, "PRH_VEC loads a run as RUN / 4 16-byte vectors");
         const uint32_t abase = it.e0 & ~3u;   // runs start 16-byte aligned; edges < e0 are masked
         auto load_idx = [&](uint32_t base) {
             const uint32_t r0 = base + lrun * RUN;
             if (r0 < it.e1) {
-                uint32_t v0, v1, v2, v3;
-                asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-                             : "=r"(v0), "=r"(v1), "=r"(v2), "=r"(v3) : "l"(p.g.rowidx_h + r0), "l"(pf));
-                xn[0] = v0;
-                xn[1] = v1;
-                xn[2] = v2;
-                xn[3] = v3;
+#pragma unroll
+                for (int v = 0; v < RUN / 4; ++v) {
+                    uint32_t v0, v1, v2, v3;
+                    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                                 : "=r"(v0), "=r"(v1), "=r"(v2), "=r"(v3) : "l"(p.g.rowidx_h + r0 + 4 * v), "l"(pf));
+                    xn[4 * v] = v0;
+                    xn[4 * v + 1] = v1;
+                    xn[4 * v + 2] = v2;
+                    xn[4 * v + 3] = v3;
+                }
 #pragma unroll
                 for (int q = 0; q < RUN; ++q)
                     if (r0 + q >= it.e1 || r0 + q < it.e0) xn[q] = HOT_BIT;   // not this item's edge
-                in_ = ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - abase) / RUN, pf);
+                in_ = ld_stream_u16(p.g.runv_p8 + it.run_p8 + (r0 - abase) / RUN, pf);
             } else {
 #pragma unroll
                 for (int q = 0; q < RUN; ++q) xn[q] = HOT_BIT;
@@ -716,7 +747,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
             const uint32_t r0 = base + lrun * RUN;
 #pragma unroll
             for (int q = 0; q < RUN; ++q) xn[q] = r0 + q < it.e1 ? ld_stream_u(p.g.rowidx_h + r0 + q, pf) : HOT_BIT;
-            in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_ph + it.run_ph + (r0 - it.e0) / RUN, pf) : 0u;
+            in_ = r0 < it.e1 ? ld_stream_u16(p.g.runv_p8 + it.run_p8 + (r0 - it.e0) / RUN, pf) : 0u;
         };
 #endif
         if (PROACT_PRH_PIPE) load_idx(abase);
@@ -763,7 +794,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
                         sum = 0ull;
                         nxt = cp[++i + 1];
                     }
-                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
+                    sum += fix62(g[q]);
                 }
                 if (!multi) {
                     kin = i;
@@ -819,7 +850,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
                         sum = 0ull;
                         nxt = cp[++i + 1];
                     }
-                    sum += (unsigned long long)__double2ll_rn((double)g[q] * FIX);
+                    sum += fix62(g[q]);
                 }
             }
             const uint32_t i0 = __shfl_sync(0xFFFFFFFFu, i, 0);
@@ -1617,6 +1648,7 @@ int graph_dev(int id, GraphDev *g)
     g->runv_pr = G.runv_pr;
     g->runv_ss = G.runv_ss;
     g->runv_ph = G.runv_ph;
+    g->runv_p8 = G.runv_p8;
     g->rowidx_h = G.rowidx_h ? G.rowidx_h : G.rowidx;   // no table: plain ids (all < HOT_BIT)
     g->hot_ids = G.hot_ids;
     g->nhot = G.nhot;
@@ -1707,7 +1739,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
     GCK(cudaMemcpyAsync(&e_own, G.colptr + G.nv, 4, cudaMemcpyDeviceToHost, s));
     GCK(cudaStreamSynchronize(s));
     G.E_own = e_own;
-    GCK(cudaMalloc((void **)&G.rowidx, 4 * ((size_t)e_own + 4)));   // +4: 16-byte index loads
+    GCK(cudaMalloc((void **)&G.rowidx, 4 * ((size_t)e_own + 8)));   // +8: 16-byte index loads, runs of 8
     if (d_w) GCK(cudaMalloc((void **)&G.w, 4 * ((size_t)e_own + 4)));   // +4: 16-byte loads
     GCK(cudaMemcpyAsync(indeg, G.colptr, 4 * ((size_t)G.nv + 1), cudaMemcpyDeviceToDevice, s));   // cursors
     if (E) scatter_kernel<<<1184, 256, 0, s>>>(d_src, d_dst, d_w, E, v0, v1, indeg, G.rowidx, G.w);
@@ -1736,25 +1768,29 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
         }
         split.insert(split.end(), whole.begin(), whole.end());   // big (hub) work first
         G.nitems = (uint32_t)split.size();
-        uint64_t npr = 0, nss = 0, nph = 0;
+        uint64_t npr = 0, nss = 0, nph = 0, np8 = 0;
         for (Item &it : split) {
             it.run_pr = (uint32_t)npr;
             it.run_ss = (uint32_t)nss;
             it.run_ph = (uint32_t)nph;
+            it.run_p8 = (uint32_t)np8;
             npr += (it.e1 - it.e0 + PROACT_PR_RUN - 1) / PROACT_PR_RUN;
             nss += (it.e1 - it.e0 + PROACT_SSSP_RUN - 1) / PROACT_SSSP_RUN;
             nph += (it.e1 - (PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0) + PROACT_PRH_RUN - 1) / PROACT_PRH_RUN;
+            np8 += (it.e1 - (PROACT_PRH_VEC ? (it.e0 & ~3u) : it.e0) + PROACT_PRH_RUN_PR - 1) / PROACT_PRH_RUN_PR;
         }
-        if (npr >= (1ull << 32) || nss >= (1ull << 32) || nph >= (1ull << 32)) return PROACT_ERR_NOMEM;
+        if (npr >= (1ull << 32) || nss >= (1ull << 32) || nph >= (1ull << 32) || np8 >= (1ull << 32)) return PROACT_ERR_NOMEM;
         GCK(cudaMalloc((void **)&G.items, sizeof(Item) * std::max<size_t>(1, split.size())));
         GCK(cudaMemcpy(G.items, split.data(), sizeof(Item) * split.size(), cudaMemcpyHostToDevice));
         GCK(cudaMalloc((void **)&G.runv_pr, 2 * std::max<uint64_t>(1, npr)));
         GCK(cudaMalloc((void **)&G.runv_ss, 2 * std::max<uint64_t>(1, nss)));
         GCK(cudaMalloc((void **)&G.runv_ph, 2 * std::max<uint64_t>(1, nph)));
+        GCK(cudaMalloc((void **)&G.runv_p8, 2 * std::max<uint64_t>(1, np8)));
         if (G.nitems) {
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PR_RUN, 0, G.runv_pr);
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_SSSP_RUN, 1, G.runv_ss);
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN, 2, G.runv_ph);
+            runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN_PR, 3, G.runv_p8);
             GCK(cudaGetLastError());
         }
         const size_t ns = std::max<uint32_t>(1, G.nslot);
@@ -1791,7 +1827,7 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
             GCK(cudaMalloc((void **)&slot, 4 * (size_t)V));
             GCK(cudaMemsetAsync(slot, 0xFF, 4 * (size_t)V, s));
             hot_slot_kernel<<<(unsigned)((H + 255) / 256), 256, 0, s>>>(G.hot_ids, (uint32_t)H, slot);
-            GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 4)));
+            GCK(cudaMalloc((void **)&G.rowidx_h, 4 * (G.E_own + 8)));
             unsigned long long *neh = nullptr;
             GCK(cudaMalloc((void **)&neh, 8));
             GCK(cudaMemsetAsync(neh, 0, 8, s));
@@ -1886,6 +1922,7 @@ int proact_graph_free(int id)
     cudaFree(G.runv_pr);
     cudaFree(G.runv_ss);
     cudaFree(G.runv_ph);
+    cudaFree(G.runv_p8);
     if (G.rowidx_h) cudaFree(G.rowidx_h);
     if (G.hot_ids) cudaFree(G.hot_ids);
     if (G.prp) {

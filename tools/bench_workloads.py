@@ -123,6 +123,16 @@ def pagerank(args, src, dst, V):
     line["roofline_l1_gather"] = {"bound": "l1tex_wavefronts", "gathers_per_launch": e_max,
                                   "peak_gathers_per_s": rate, "t_min_ms": t_l1, "frac": t_l1 / kms,
                                   "note": "global gathers (in-edges of non-hot sources); 1 wavefront/clk/SM x SMs x 1965 MHz"}
+    # the same bound MEASURED: tools/probes/gather_peak.cu (an index stream + random 4-byte gathers
+    # from a 64 MiB L2-resident vector and nothing else, the best CTA shape), on a B200 of this pool
+    try:
+        gp = max(json.loads(l)["gathers_per_s"] for l in open(os.path.join(ROOT, "profiles", "r02p_gather_peak.jsonl"))
+                 if l.startswith("{"))
+        line["roofline_gather_measured"] = {"bound": "random 4-byte gathers (measured)", "peak_gathers_per_s": gp,
+                                            "t_min_ms": e_max / gp * 1e3, "frac": e_max / gp * 1e3 / kms,
+                                            "source": "profiles/r02p_gather_peak.jsonl (tools/probes/gather_peak.cu)"}
+    except (OSError, ValueError):
+        pass
     if "overhead" in res[0]:
         o = res[0]["overhead"]
         line["overhead"] = {"local_ms_per_phase": o["local_ms"], "elide_ms_per_phase": o["elide_ms"],
