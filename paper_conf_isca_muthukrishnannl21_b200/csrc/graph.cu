@@ -1785,12 +1785,14 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
         GCK(cudaMalloc((void **)&G.runv_pr, 2 * std::max<uint64_t>(1, npr)));
         GCK(cudaMalloc((void **)&G.runv_ss, 2 * std::max<uint64_t>(1, nss)));
         GCK(cudaMalloc((void **)&G.runv_ph, 2 * std::max<uint64_t>(1, nph)));
-        GCK(cudaMalloc((void **)&G.runv_p8, 2 * std::max<uint64_t>(1, np8)));
+        if (PROACT_PRH_RUN_PR != PROACT_PRH_RUN) GCK(cudaMalloc((void **)&G.runv_p8, 2 * std::max<uint64_t>(1, np8)));
+        else G.runv_p8 = G.runv_ph;   // same runs: one array
         if (G.nitems) {
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PR_RUN, 0, G.runv_pr);
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_SSSP_RUN, 1, G.runv_ss);
             runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN, 2, G.runv_ph);
-            runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN_PR, 3, G.runv_p8);
+            if (PROACT_PRH_RUN_PR != PROACT_PRH_RUN)
+                runv_kernel<<<G.nitems, 256, 0, s>>>(G.items, G.colptr, G.nv, PROACT_PRH_RUN_PR, 3, G.runv_p8);
             GCK(cudaGetLastError());
         }
         const size_t ns = std::max<uint32_t>(1, G.nslot);
@@ -1921,8 +1923,8 @@ int proact_graph_free(int id)
     cudaFree(G.acc_cnt);
     cudaFree(G.runv_pr);
     cudaFree(G.runv_ss);
+    if (G.runv_p8 != G.runv_ph) cudaFree(G.runv_p8);
     cudaFree(G.runv_ph);
-    cudaFree(G.runv_p8);
     if (G.rowidx_h) cudaFree(G.rowidx_h);
     if (G.hot_ids) cudaFree(G.hot_ids);
     if (G.prp) {

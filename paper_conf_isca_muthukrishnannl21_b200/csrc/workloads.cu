@@ -120,14 +120,24 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *b)
 {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
+#ifndef PROACT_JACOBI_WAIT_NS   // > 0: waits suspend in hardware up to this long per try (a waiting
+#define PROACT_JACOBI_WAIT_NS 0   // warp then takes no issue slots; the phase completion wakes it)
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
 {
     uint32_t done;
     do {
+#if PROACT_JACOBI_WAIT_NS > 0
+        asm volatile("{\n\t.reg .pred p;\n\t"
+                     "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+                     "selp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(done) : "r"(smem_u32(b)), "r"(parity), "n"(PROACT_JACOBI_WAIT_NS) : "memory");
+#else
         asm volatile("{\n\t.reg .pred p;\n\t"
                      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
                      "selp.u32 %0, 1, 0, p;\n\t}"
                      : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+#endif
     } while (!done);
 }
 __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes, uint64_t *bar)
