@@ -115,6 +115,7 @@ struct Graph {
     int32_t *pwt = nullptr;                // [E_own] weight
     int32_t *dprev = nullptr;              // [V] previous round's input distances
     int32_t *ptmp = nullptr;               // [nv] minima of the round, INT32_MAX between rounds
+    uint32_t *ptouch = nullptr;            // [nv / 1024] a frontier edge reached the 4 KiB block
     uint2 *heavy = nullptr;                // [nheavy_max] pieces (source, first edge) of heavy frontier sources
     uint32_t nheavy_max = 0;
     uint32_t *pctl = nullptr;              // [4]: heavy pieces, barrier arrivals, barrier generation, claims
@@ -342,6 +343,7 @@ struct PushDev {
     const uint32_t *prp, *pcol;
     const int32_t *pwt;
     int32_t *dprev, *ptmp;
+    uint32_t *ptouch;
     uint2 *heavy;
     uint32_t *pctl;
     unsigned long long *dcnt;
@@ -971,6 +973,7 @@ __device__ __forceinline__ void push_relax(const SsspParams &p, uint32_t e, int3
     const int64_t c = (int64_t)du + (int64_t)__ldg(p.q.pwt + e);
     const int32_t cand = c < (int64_t)INT32_MAX ? (int32_t)c : INT32_MAX;
     atomicMin(p.q.ptmp + v, cand);
+    p.q.ptouch[v >> 10] = 1u;   // the block's minima need a look in step 3
 }
 
 constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
@@ -1519,11 +1522,29 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
     //    and slices chunk-aligned), 4 per thread with 16-byte loads: d' = min(d, minima),
     //    instrumented stores, chunk state, vote, commit (a2, a3); the minima are reset to
     //    INT32_MAX for the next push round
+    //    A block no frontier edge reached, in a chunk that did not change last round, already
+    //    holds d' in the output replica (it holds d^{k-1} = d^k = d^{k+1} there, and so do the
+    //    peers' copies): it is committed without loads or stores.
     unsigned long long cs = 0;
     const uint32_t nblk = (p.g.nv + 1023) / 1024;
+    __shared__ uint32_t blk_work;
     for (uint32_t t = pb; t < nblk; t += P) {
         const uint32_t lo = p.g.v0 + t * 1024, nvt = min(lo + 1024, p.g.v0 + p.g.nv) - lo;
         const uint32_t i = 4 * threadIdx.x;
+        const uint64_t off = (uint64_t)lo * 4;
+        if (threadIdx.x == 0) {
+            const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
+            const bool touched = __ldcg(p.q.ptouch + t) != 0u;
+            if (touched) p.q.ptouch[t] = 0u;
+            blk_work = (prev ? 2u : 0u) | (touched ? 1u : 0u);
+        }
+        __syncthreads();
+        const uint32_t work = blk_work;
+        if (work == 0u) {   // untouched, unchanged: commit only (a3)
+            if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
+            __syncthreads();   // blk_work is rewritten by the next block
+            continue;
+        }
         bool changed = false;
         if (i + 4 <= nvt) {
             const int4 old = *reinterpret_cast<const int4 *>(din + lo + i);
@@ -1557,13 +1578,11 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
         }
         const int any = __syncthreads_or(changed);   // orders the block's puts before the commit
         if (threadIdx.x == 0) {
-            const uint64_t off = (uint64_t)lo * 4;
-            const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
             if (any) {
                 proact::mark_changed(lc, p.region_out, off);
                 proact::vote(lc);
             }
-            if (any || prev) proact::mark_push(lc, p.region_out, off);
+            if (any || (work & 2u)) proact::mark_push(lc, p.region_out, off);
             proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
         }
     }
@@ -1851,6 +1870,8 @@ int proact_graph_build_ex(const uint32_t *d_src, const uint32_t *d_dst, const in
         GCK(cudaMalloc((void **)&G.pwt, 4 * std::max<uint64_t>(1, G.E_own)));
         GCK(cudaMalloc((void **)&G.dprev, 4 * (size_t)V));
         GCK(cudaMalloc((void **)&G.ptmp, 4 * std::max<size_t>(1, G.nv)));
+        GCK(cudaMalloc((void **)&G.ptouch, 4 * std::max<size_t>(1, (G.nv + 1023) / 1024)));
+        GCK(cudaMemsetAsync(G.ptouch, 0, 4 * std::max<size_t>(1, (G.nv + 1023) / 1024), s));
         GCK(cudaMalloc((void **)&G.pctl, 16));
         GCK(cudaMalloc((void **)&G.dcnt, 16));
         GCK(cudaMallocHost((void **)&G.hcnt, 8));
@@ -1933,6 +1954,7 @@ int proact_graph_free(int id)
         cudaFree(G.pwt);
         cudaFree(G.dprev);
         cudaFree(G.ptmp);
+        cudaFree(G.ptouch);
         cudaFree(G.heavy);
         cudaFree(G.pctl);
         cudaFree(G.dcnt);
@@ -2066,7 +2088,7 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
             push = Gr.tracked && est < pct * (double)Gr.E_all;
             track = est < 4.0 * pct * (double)Gr.E_all;
         }
-        p.q = PushDev{Gr.prp, Gr.pcol, Gr.pwt, Gr.dprev, Gr.ptmp, Gr.heavy, Gr.pctl, Gr.dcnt,
+        p.q = PushDev{Gr.prp, Gr.pcol, Gr.pwt, Gr.dprev, Gr.ptmp, Gr.ptouch, Gr.heavy, Gr.pctl, Gr.dcnt,
                       track ? 1u : 0u, Gr.round & 1u};
     }
     Gr.tracked = push || track;

@@ -1387,6 +1387,17 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         unsigned total = grid ? grid : cap;
         const unsigned reserve = std::min(cap - 1, agent_ctas * lost);
         if (total + reserve > cap) total = cap - reserve;
+        // loopback with three or more ranks per device: a producer that keeps the default carve-out
+        // (graph kernels, keeps_l1) leaves too little shared memory on any SM it occupies for
+        // another rank's agent CTA, and the CTA scheduler spreads producers over every SM first --
+        // one rank's agent could then never start while the other ranks' producers wait for its
+        // data (observed: PageRank G = 3 / 4 loopback, wait-all timeouts).  Keep whole SMs free:
+        // the ranks' producer CTAs together stay below the SMs not needed by their agents.
+        if (keeps_l1(kernel) && c->ranks_on_device >= 3) {
+            const long rod3 = c->ranks_on_device;
+            const long free_sms = (long)c->nsm - rod3 * (long)agent_ctas;
+            total = std::min(total, (unsigned)std::max(1L, free_sms / rod3));
+        }
         if (cluster > 1) total = std::max(cluster, total / cluster * cluster);
         *(launch_ctx *)args[0] = lc;
         CK(launch_producer(kernel, total, block, args, smem, s, c->device, l2b, l2n, true, cluster));
