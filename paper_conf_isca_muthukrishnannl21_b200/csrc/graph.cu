@@ -348,6 +348,7 @@ struct PushDev {
     uint32_t *pctl;
     unsigned long long *dcnt;
     uint32_t track, par;   // track: pull kernels keep dprev current this round
+    uint32_t skip, pad;    // push round: mark the blocks frontier edges reach, skip the others
 };
 struct SsspParams {
     GraphDev g;
@@ -973,7 +974,7 @@ __device__ __forceinline__ void push_relax(const SsspParams &p, uint32_t e, int3
     const int64_t c = (int64_t)du + (int64_t)__ldg(p.q.pwt + e);
     const int32_t cand = c < (int64_t)INT32_MAX ? (int32_t)c : INT32_MAX;
     atomicMin(p.q.ptmp + v, cand);
-    p.q.ptouch[v >> 10] = 1u;   // the block's minima need a look in step 3
+    if (p.q.skip) p.q.ptouch[v >> 10] = 1u;   // the block's minima need a look in step 3
 }
 
 constexpr uint32_t CHG_WORDS = 4096;   // changed-chunk bitmap in shared memory (<= 131072 chunks)
@@ -1534,8 +1535,8 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
         const uint64_t off = (uint64_t)lo * 4;
         if (threadIdx.x == 0) {
             const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
-            const bool touched = __ldcg(p.q.ptouch + t) != 0u;
-            if (touched) p.q.ptouch[t] = 0u;
+            const bool touched = !p.q.skip || __ldcg(p.q.ptouch + t) != 0u;
+            if (touched && p.q.skip) p.q.ptouch[t] = 0u;
             blk_work = (prev ? 2u : 0u) | (touched ? 1u : 0u);
         }
         __syncthreads();
@@ -2074,7 +2075,7 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
     // only when asked (track) -- the copy costs a pass over V per round, so pull rounds track only
     // once the frontier is below 4x the push threshold, and a round may push only if the round
     // before it tracked.
-    bool push = false, track = false;
+    bool push = false, track = false, skip = true;   // skip: tiny frontiers (first round: the source)
     if (Gr.prp && pmode != 0) {
         if (first) {
             GCK(cudaMemsetAsync(Gr.dcnt, 0, 16, s));
@@ -2087,9 +2088,11 @@ int proact_sssp_phase(int graph, int region_in, int region_out, int first, void 
             const double est = 100.0 * (double)*Gr.hcnt * (double)Gr.V / (double)std::max(1u, Gr.nv);
             push = Gr.tracked && est < pct * (double)Gr.E_all;
             track = est < 4.0 * pct * (double)Gr.E_all;
+            const char *sp = getenv("PROACT_SSSP_SKIP_PCT");
+            skip = est < (sp ? atof(sp) : 1.0) * (double)Gr.E_all;
         }
         p.q = PushDev{Gr.prp, Gr.pcol, Gr.pwt, Gr.dprev, Gr.ptmp, Gr.ptouch, Gr.heavy, Gr.pctl, Gr.dcnt,
-                      track ? 1u : 0u, Gr.round & 1u};
+                      track ? 1u : 0u, Gr.round & 1u, skip ? 1u : 0u, 0u};
     }
     Gr.tracked = push || track;
     Gr.last_mode = push ? 1 : 0;
