@@ -1528,64 +1528,75 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
     //    peers' copies): it is committed without loads or stores.
     unsigned long long cs = 0;
     const uint32_t nblk = (p.g.nv + 1023) / 1024;
-    __shared__ uint32_t blk_work;
-    for (uint32_t t = pb; t < nblk; t += P) {
-        const uint32_t lo = p.g.v0 + t * 1024, nvt = min(lo + 1024, p.g.v0 + p.g.nv) - lo;
-        const uint32_t i = 4 * threadIdx.x;
-        const uint64_t off = (uint64_t)lo * 4;
-        if (threadIdx.x == 0) {
-            const bool prev = !p.first && proact::local_changed(lc, p.region_in, off);
-            const bool touched = !p.q.skip || __ldcg(p.q.ptouch + t) != 0u;
-            if (touched && p.q.skip) p.q.ptouch[t] = 0u;
-            blk_work = (prev ? 2u : 0u) | (touched ? 1u : 0u);
+    __shared__ uint32_t blk_work[PB];
+    // the CTA's blocks pb, pb + P, ... in passes of PB: thread j reads block j's flags (one round
+    // trip for the pass instead of one per block)
+    for (uint32_t b0 = 0; pb + b0 * P < nblk; b0 += PB) {
+        {
+            const uint32_t tj = pb + (b0 + threadIdx.x) * P;
+            uint32_t w = 0u;
+            if (tj < nblk) {
+                const bool prev = !p.first && proact::local_changed(lc, p.region_in, (uint64_t)(p.g.v0 + tj * 1024) * 4);
+                const bool touched = !p.q.skip || __ldcg(p.q.ptouch + tj) != 0u;
+                if (touched && p.q.skip) p.q.ptouch[tj] = 0u;
+                w = (prev ? 2u : 0u) | (touched ? 1u : 0u);
+            }
+            blk_work[threadIdx.x] = w;
+            __syncthreads();
         }
-        __syncthreads();
-        const uint32_t work = blk_work;
-        if (work == 0u) {   // untouched, unchanged: commit only (a3)
-            if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
-            __syncthreads();   // blk_work is rewritten by the next block
-            continue;
-        }
-        bool changed = false;
-        if (i + 4 <= nvt) {
-            const int4 old = *reinterpret_cast<const int4 *>(din + lo + i);
-            int4 *mp = reinterpret_cast<int4 *>(p.q.ptmp + (lo - p.g.v0) + i);
-            int4 m;
-            asm volatile("ld.global.cg.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(m.x), "=r"(m.y), "=r"(m.z), "=r"(m.w) : "l"(mp));
-            if (m.x != INT32_MAX || m.y != INT32_MAX || m.z != INT32_MAX || m.w != INT32_MAX)
-                *mp = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX);
-            const int4 best = make_int4(min(old.x, m.x), min(old.y, m.y), min(old.z, m.z), min(old.w, m.w));
-            proact::put(lc, p.region_out, (uint64_t)(lo + i) * 4, best);
-            const int32_t ob[4] = {old.x, old.y, old.z, old.w}, bb[4] = {best.x, best.y, best.z, best.w};
-#pragma unroll
-            for (int q = 0; q < 4; ++q)
-                if (bb[q] != ob[q]) {
-                    changed = true;
-                    cs += __ldg(p.g.outdeg + lo + i + q);
-                }
-        } else {
-            for (uint32_t j = i; j < nvt && j < i + 4; ++j) {
-                const uint32_t v = lo + j;
-                const int32_t old = din[v];
-                const int32_t m = ld_cg_i(p.q.ptmp + (v - p.g.v0));
-                if (m != INT32_MAX) p.q.ptmp[v - p.g.v0] = INT32_MAX;
-                const int32_t best = min(old, m);
-                proact::put(lc, p.region_out, (uint64_t)v * 4, best);
-                if (best != old) {
-                    changed = true;
-                    cs += __ldg(p.g.outdeg + v);
+        for (uint32_t jb = 0; jb < PB; ++jb) {
+            const uint32_t t = pb + (b0 + jb) * P;
+            if (t >= nblk) break;
+            const uint32_t lo = p.g.v0 + t * 1024, nvt = min(lo + 1024, p.g.v0 + p.g.nv) - lo;
+            const uint32_t i = 4 * threadIdx.x;
+            const uint64_t off = (uint64_t)lo * 4;
+            const uint32_t work = blk_work[jb];
+            if (work == 0u) {   // untouched, unchanged: commit only (a3)
+                if (threadIdx.x == 0) proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
+                continue;
+            }
+            bool changed = false;
+            if (i + 4 <= nvt) {
+                const int4 old = *reinterpret_cast<const int4 *>(din + lo + i);
+                int4 *mp = reinterpret_cast<int4 *>(p.q.ptmp + (lo - p.g.v0) + i);
+                int4 m;
+                asm volatile("ld.global.cg.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(m.x), "=r"(m.y), "=r"(m.z), "=r"(m.w) : "l"(mp));
+                if (m.x != INT32_MAX || m.y != INT32_MAX || m.z != INT32_MAX || m.w != INT32_MAX)
+                    *mp = make_int4(INT32_MAX, INT32_MAX, INT32_MAX, INT32_MAX);
+                const int4 best = make_int4(min(old.x, m.x), min(old.y, m.y), min(old.z, m.z), min(old.w, m.w));
+                proact::put(lc, p.region_out, (uint64_t)(lo + i) * 4, best);
+                const int32_t ob[4] = {old.x, old.y, old.z, old.w}, bb[4] = {best.x, best.y, best.z, best.w};
+    #pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (bb[q] != ob[q]) {
+                        changed = true;
+                        cs += __ldg(p.g.outdeg + lo + i + q);
+                    }
+            } else {
+                for (uint32_t j = i; j < nvt && j < i + 4; ++j) {
+                    const uint32_t v = lo + j;
+                    const int32_t old = din[v];
+                    const int32_t m = ld_cg_i(p.q.ptmp + (v - p.g.v0));
+                    if (m != INT32_MAX) p.q.ptmp[v - p.g.v0] = INT32_MAX;
+                    const int32_t best = min(old, m);
+                    proact::put(lc, p.region_out, (uint64_t)v * 4, best);
+                    if (best != old) {
+                        changed = true;
+                        cs += __ldg(p.g.outdeg + v);
+                    }
                 }
             }
-        }
-        const int any = __syncthreads_or(changed);   // orders the block's puts before the commit
-        if (threadIdx.x == 0) {
-            if (any) {
-                proact::mark_changed(lc, p.region_out, off);
-                proact::vote(lc);
+            const int any = __syncthreads_or(changed);   // orders the block's puts before the commit
+            if (threadIdx.x == 0) {
+                if (any) {
+                    proact::mark_changed(lc, p.region_out, off);
+                    proact::vote(lc);
+                }
+                if (any || (work & 2u)) proact::mark_push(lc, p.region_out, off);
+                proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
             }
-            if (any || (work & 2u)) proact::mark_push(lc, p.region_out, off);
-            proact::commit_span(lc, p.region_out, off, (uint64_t)nvt * 4);
         }
+        __syncthreads();   // blk_work is rewritten by the next pass
     }
     count_changed(p, cs);
 }
