@@ -21,7 +21,7 @@ from paper_conf_isca_muthukrishnannl21_b200 import _lib, run_ranks  # noqa: E402
 from paper_conf_isca_muthukrishnannl21_b200 import runtime as rt  # noqa: E402
 from paper_conf_isca_muthukrishnannl21_b200 import workloads as wl  # noqa: E402
 
-SPACE = "mech=0,1,2,5;chunk=131072,1048576,16777216;warps=8,32;piece=65536;push=1;disc=0;akern=1"
+SPACE = "mech=0,1,2,5;chunk=131072,1048576,16777216;warps=8,32;piece=65536;push=0,1;disc=0;akern=0,1,2"
 NAMES = {v: k for k, v in _lib.MECH_NAMES.items()}
 
 
@@ -77,12 +77,16 @@ def main():
         rows.append((work, best))
     import json
     cache = json.load(open(os.environ["PROACT_TUNE_CACHE"]))
-    lines = ["| workload (G loopback) | mechanism | chunk | agent warps | piece | phase ms |", "|---|---|---|---|---|---|"]
+    lines = ["| workload (G loopback) | mechanism | placement | push | chunk | agent warps | phase ms |",
+             "|---|---|---|---|---|---|---|"]
+    place = {0: "agent CTAs in the grid", 1: "separate agent kernel", 2: "producer-CTA transfer warps"}
     for work, b in rows:
         ms = cache.get(f"{work}_G{args.ranks}_loopback", {}).get("ms")
         agent = b["mech"] in (_lib.MECH_FUSED, _lib.MECH_ELIDE)
-        lines.append(f"| {work} (G={args.ranks}) | {_lib.MECH_NAMES[b['mech']]} | {b['chunk_bytes']} | "
-                     f"{b['agent_warps'] if agent else '-'} | {b['piece_bytes'] if agent else '-'} | {ms:.3f} |")
+        lines.append(f"| {work} (G={args.ranks}) | {_lib.MECH_NAMES[b['mech']]} | "
+                     f"{place.get(b['agent_kernel'], '?') if agent else '-'} | "
+                     f"{('TMA (tile push)' if b['agent_kernel'] == 2 else 'TMA' if b['push'] == 1 else 'VEC16') if agent else '-'} | {b['chunk_bytes']} | "
+                     f"{b['agent_warps'] if agent and b['agent_kernel'] != 2 else '-'} | {ms:.3f} |")
     txt = "\n".join(lines) + f"\n\nspace: `{SPACE}`\n"
     print(txt)
     if args.out:
