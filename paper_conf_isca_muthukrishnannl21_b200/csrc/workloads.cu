@@ -90,6 +90,9 @@ constexpr int JV = PROACT_JACOBI_JV;    // float4 column groups per compute thre
 constexpr uint32_t JOS = PROACT_JACOBI_OUT_RING;   // MODE 2: output slots of JSR row strips (4 KiB each)
 constexpr int JSR = PROACT_JACOBI_SPAN_ROWS;       // rows per pushed span
 constexpr int JW = JC * 32 * 4 * JV;    // strip width in columns = 4 KiB of a row
+#ifndef PROACT_JACOBI_OUT_STORE   // output stores: 0 plain, 1 evict-first hint, 2 .cs in MODE 0
+#define PROACT_JACOBI_OUT_STORE 2
+#endif
 #ifndef PROACT_JACOBI_OUT_EVICT_LAST   // G > 1: output rows evict-last until the agent has read them
 #define PROACT_JACOBI_OUT_EVICT_LAST 0
 #endif
@@ -311,6 +314,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     char *outb = lc.ctx->region[p.region_out].base;
     uint64_t pol_out = 0;
     if (PROACT_JACOBI_OUT_EVICT_LAST) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_out));
+    if (PROACT_JACOBI_OUT_STORE == 1) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_out));
     uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
     uint32_t kt = 0;   // tiles handed to the committer
     uint32_t oq = 0;   // MODE 2: next output span of this CTA
@@ -421,7 +425,18 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                         asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
                                      ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
                     } else {
+#if PROACT_JACOBI_OUT_STORE == 1   // evict-first hint (experiment)
+                        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                                     ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
+#elif PROACT_JACOBI_OUT_STORE == 2
+                        // no agent reads this output back (MODE 0): streaming stores (st.cs), ~1 %
+                        // faster under the power cap (profiles/r02k_jacobi_store_policy.log); an
+                        // agent's read-back (MODE 1) wants the lines kept in L2
+                        if (MODE == 0) __stcs(reinterpret_cast<float4 *>(outb + off), o);
+                        else *reinterpret_cast<float4 *>(outb + off) = o;
+#else
                         *reinterpret_cast<float4 *>(outb + off) = o;
+#endif
                     }
                 }
                 }
