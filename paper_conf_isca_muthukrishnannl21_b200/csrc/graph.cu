@@ -960,12 +960,20 @@ __device__ __forceinline__ void track_input(const launch_ctx &lc, const SsspPara
     if (proact::producer_block(lc) == 0)
         for (uint64_t u = n4 * 4 + threadIdx.x; u < p.g.V; u += blockDim.x) p.q.dprev[u] = din[u];
 }
-// out-degree sum of my changed vertices, for the next round's pull / push decision (host)
-__device__ __forceinline__ void count_changed(const SsspParams &p, unsigned long long cs)
+// out-degree sum of my changed vertices, for the next round's pull / push decision (host): warp
+// sums meet in the CTA's shared accumulator (one global atomic per CTA, count_flush at the end --
+// a global atomic per warp and tile serialises on one address)
+__device__ __forceinline__ void count_changed(const SsspParams &p, unsigned long long cs, unsigned long long *cta)
 {
     if (!p.q.dcnt) return;   // (callers accumulate in 32 bits: a thread's vertices' out-degrees)
     for (int o = 16; o > 0; o >>= 1) cs += __shfl_xor_sync(0xFFFFFFFFu, cs, o);
-    if ((threadIdx.x & 31u) == 0u && cs) atomicAdd(&p.q.dcnt[p.q.par], cs);
+    if ((threadIdx.x & 31u) == 0u && cs) atomicAdd(cta, cs);
+}
+__device__ __forceinline__ void count_flush(const SsspParams &p, const unsigned long long *cta)
+{
+    if (!p.q.dcnt) return;
+    __syncthreads();
+    if (threadIdx.x == 0 && *cta) atomicAdd(&p.q.dcnt[p.q.par], *cta);
 }
 // relax edge e (source distance du) into my vertex pcol[e]: a fire-and-forget atomicMin (RED)
 __device__ __forceinline__ void push_relax(const SsspParams &p, uint32_t e, int32_t du)
@@ -996,9 +1004,11 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
     const uint32_t cv = Ri.chunk_bytes / 4;
     const uint32_t cshift = __popc(cv) == 1 ? (uint32_t)(__ffs(cv) - 1) : 0u, cdiv = __popc(cv) == 1 ? 0u : cv;
     __shared__ uint32_t kclaim;
+    __shared__ unsigned long long cs_cta;
     bool ready = false;
     if (p.q.dcnt) {   // every CTA keeps its share of dprev current (if asked), items or not
         if (threadIdx.x == 0) {
+            cs_cta = 0ull;
             proact::wait_all(lc, p.region_in);
             if (proact::producer_block(lc) == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;
         }
@@ -1111,7 +1121,7 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
                 changed |= best != old;
                 if (best != old) cs += __ldg(p.g.outdeg + v);
             }
-            count_changed(p, cs);
+            count_changed(p, cs, &cs_cta);
             // per-tile chunk state (SPARSE region): changed now -> flag bit + vote; push if
             // changed now or in the previous round (the peers' ping-pong copy holds d^{k-1})
             const int any = __syncthreads_or(changed);
@@ -1128,6 +1138,7 @@ __global__ void __launch_bounds__(GB, PROACT_SSSP_MINB) sssp_kernel(launch_ctx l
         }
         __syncthreads();
     }
+    count_flush(p, &cs_cta);
 }
 
 // ---- SSSP with the hot-source table and the pipelined index stream (as pagerank_hot_kernel).
@@ -1161,9 +1172,11 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         return p.first || (chg[g >> 5] >> (g & 31) & 1u);
     };
     // (a7) wait for the previous generation, snapshot its changed bits, stage the hot table
+    __shared__ unsigned long long cs_cta;
     if (threadIdx.x == 0) {
         proact::wait_all(lc, p.region_in);
         nout = 0u;
+        cs_cta = 0ull;
         if (p.q.dcnt && proact::producer_block(lc) == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;
     }
     __syncthreads();
@@ -1342,7 +1355,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
                 changed |= best != old;
                 if (best != old) cs += __ldg(p.g.outdeg + v);
             }
-            count_changed(p, cs);
+            count_changed(p, cs, &cs_cta);
             if (__any_sync(0xFFFFFFFFu, changed) && lane == 0) any_a[grp] = 1u;
             grp_bar(grp);   // orders the group's puts before the commit (a3)
             if (t == 0) {   // chunk state as in sssp_kernel
@@ -1359,6 +1372,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_SSH_MINB) sssp_hot_kernel(laun
         }
         grp_bar(grp);
     }
+    count_flush(p, &cs_cta);
     if (CL > 1) cluster_sync_all();   // my slice stays readable until every peer is done
 }
 
@@ -1382,8 +1396,10 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
     const int32_t *din = reinterpret_cast<const int32_t *>(Ri.base);
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t P = proact::producer_grid(lc), pb = proact::producer_block(lc);
+    __shared__ unsigned long long cs_cta;
     if (threadIdx.x == 0) {
         proact::wait_all(lc, p.region_in);   // (a7) the previous generation is here
+        cs_cta = 0ull;
         if (pb == 0) p.q.dcnt[p.q.par ^ 1u] = 0ull;   // the next round's accumulator
     }
     __syncthreads();
@@ -1598,7 +1614,8 @@ __global__ void __launch_bounds__(PB, PROACT_PUSH_MINB) sssp_push_kernel(launch_
         }
         __syncthreads();   // blk_work is rewritten by the next pass
     }
-    count_changed(p, cs);
+    count_changed(p, cs, &cs_cta);
+    count_flush(p, &cs_cta);
 }
 
 __global__ void push_count_kernel(const uint32_t *rowidx, uint64_t E, uint32_t *cnt)
