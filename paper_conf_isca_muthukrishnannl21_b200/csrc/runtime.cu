@@ -1235,7 +1235,10 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     lc.ctx = c->d;
     lc.epoch = c->epoch;
     lc.mech = (uint16_t)cfg.mech;
-    lc.push = (uint16_t)cfg.push;
+    // ELIDE moves no data: its agent (tallies, discovery, flags) needs no TMA staging ring, which
+    // would otherwise take a whole SM's shared memory per agent CTA from the producer
+    const int push = cfg.mech == PROACT_MECH_ELIDE ? PROACT_PUSH_VEC16 : cfg.push;
+    lc.push = (uint16_t)push;
     lc.piece_bytes = cfg.piece_bytes;
     lc.discovery = (uint16_t)cfg.discovery;
     uint32_t armed = 0;
@@ -1275,8 +1278,8 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     // TMA (BULK) agents: issuing warps per agent CTA, each with its slice of the CTA's staging
     // memory (PROACT_AGENT_BULK_WARPS, default 1; separate agent kernel only)
     static const unsigned bulk_w = (unsigned)std::min(8, std::max(1, env_int("PROACT_AGENT_BULK_WARPS", 1)));
-    const unsigned bw = separate && cfg.push == PROACT_PUSH_BULK ? bulk_w : 1u;
-    unsigned wpc = cfg.push == PROACT_PUSH_BULK ? bw : agent_block / 32;
+    const unsigned bw = separate && push == PROACT_PUSH_BULK ? bulk_w : 1u;
+    unsigned wpc = push == PROACT_PUSH_BULK ? bw : agent_block / 32;
     unsigned agent_ctas = agent ? (cfg.agent_warps + wpc - 1) / wpc : 0;
     // at most half of this rank's share of the SMs hosts agent CTAs: beyond that the producer
     // starves (loopback G = 2, 96 agent warps: 7.8 ms per microbenchmark phase instead of 0.76,
@@ -1286,7 +1289,7 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
     const unsigned agent_cap = std::max(1u, (unsigned)c->nsm / ((c->ranks_on_device > 2 ? 4u : 2u) *
                                                                 (unsigned)std::max(1, c->ranks_on_device)));
     agent_ctas = std::min(agent_ctas, agent_cap);
-    if (agent && !separate && cfg.push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
+    if (agent && !separate && push == PROACT_PUSH_BULK && smem < PROACT_BULK_SMEM) smem = PROACT_BULK_SMEM;
     lc.agent_warps = (uint16_t)(agent ? std::min<unsigned>(cfg.agent_warps, agent_ctas * wpc) : 0);
     int nb = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, (int)block, smem));
@@ -1329,7 +1332,7 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         launch_ctx la = lc;
         la.agent_ctas = (uint16_t)agent_ctas;
         la.flags |= (uint16_t)(bw << proact::LCF_BULK_WARPS_SHIFT);
-        const size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
+        const size_t asmem = push != PROACT_PUSH_BULK ? 0 : (agent_ctas > 32 ? AGENT_SMEM_SMALL : AGENT_SMEM);
         agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
         CK(cudaGetLastError());
         c->resident_total += agent_ctas;   // its CTAs count themselves resident too
@@ -1355,9 +1358,9 @@ int proact_launch_ex(const int *regions, int nregions, const void *kernel, unsig
         // three or more ranks sharing a device (loopback) use the small ring: an agent CTA that needs a whole SM's
         // shared memory can find no SM once several ranks' persistent grids are spread over the
         // device (observed with 4 ranks x 16 agent CTAs: the agent never becomes resident)
-        size_t asmem = cfg.push != PROACT_PUSH_BULK ? 0
+        size_t asmem = push != PROACT_PUSH_BULK ? 0
                        : (agent_ctas > 32 || c->ranks_on_device > 2 ? AGENT_SMEM_SMALL : AGENT_SMEM);
-        if (cfg.push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
+        if (push == PROACT_PUSH_BULK && env_int("PROACT_AGENT_SMEM_KB", 0) > 0)
             asmem = std::min(AGENT_SMEM_MAX, (size_t)env_int("PROACT_AGENT_SMEM_KB", 0) * 1024 + 1024);
         agent_kernel<<<agent_ctas, agent_block, asmem, s>>>(la);
         CK(cudaGetLastError());
