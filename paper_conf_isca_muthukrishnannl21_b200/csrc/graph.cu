@@ -510,6 +510,9 @@ __device__ __forceinline__ bool split_arrive(const GraphDev &g, const Item &it, 
 // bit-reproducible for any schedule; r' = (float)((1-d)/V + d * sum) as in the oracle (R12).
 constexpr double FIX = 4611686018427387904.0;          // 2^62
 constexpr double UNFIX = 1.0 / 4611686018427387904.0;  // 2^-62
+#ifndef PROACT_PR_LIMBS   // pagerank_hot_kernel sums: 0 = two 32-bit halves (atomic + dependent carry
+#define PROACT_PR_LIMBS 0    // atomic), 1 = three limbs of fire-and-forget adds (measured 1.060 vs 1.043 ms)
+#endif
 #ifndef PROACT_PR_FIX_INT
 #define PROACT_PR_FIX_INT 0   // 1: integer rounding (bit-identical; measured no faster: 1.053 vs 1.044 ms)
 #endif
@@ -670,13 +673,38 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
     constexpr int RUN = PROACT_PRH_RUN_PR;
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
+#if PROACT_PR_LIMBS
+    // the 62-bit fixed-point sums as three 20/20/24-bit limbs, each a fire-and-forget 32-bit shared
+    // RED (no returned value, no carry chain): a limb accumulator takes < 4096 adds per item (a
+    // vertex gets at most one add per warp iteration on the hub path, <= 64 at its two ends), and
+    // the top limb's total is bounded by the sum itself (< 2^64 >> 40)
+    __shared__ uint32_t acc_l0_a[PG][GT], acc_lo_a[PG][GT], acc_hi_a[PG][GT];
+    uint32_t *acc_l0 = acc_l0_a[threadIdx.x / GB];
+#else
     __shared__ uint32_t acc_lo_a[PG][GT], acc_hi_a[PG][GT];
+#endif
     __shared__ uint32_t kclaim_a[PG], last_a[PG], nout;
     const uint32_t grp = threadIdx.x / GB, t = threadIdx.x % GB;
     uint32_t *acc_lo = acc_lo_a[grp], *acc_hi = acc_hi_a[grp], *cp = dyn + grp * CPS;
     float *hot = reinterpret_cast<float *>(dyn + PG * CPS);
     const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
     const uint64_t pl = pol_last(), pf = pol_first();
+#if PROACT_PR_LIMBS
+    auto acc_add = [&](uint32_t i, unsigned long long x) {
+        const uint32_t a = (uint32_t)x & 0xFFFFFu, b = (uint32_t)(x >> 20) & 0xFFFFFu, c = (uint32_t)(x >> 40);
+        if (a) atomicAdd(&acc_l0[i], a);
+        if (b) atomicAdd(&acc_lo[i], b);
+        if (c) atomicAdd(&acc_hi[i], c);
+    };
+    auto acc_get = [&](uint32_t i) {
+        return (unsigned long long)acc_l0[i] + ((unsigned long long)acc_lo[i] << 20) + ((unsigned long long)acc_hi[i] << 40);
+    };
+    auto acc_set = [&](uint32_t i, unsigned long long v) {
+        acc_l0[i] = (uint32_t)v & 0xFFFFFu;
+        acc_lo[i] = (uint32_t)(v >> 20) & 0xFFFFFu;
+        acc_hi[i] = (uint32_t)(v >> 40);
+    };
+#else
     auto acc_add = [&](uint32_t i, unsigned long long x) {
         const uint32_t xl = (uint32_t)x, old = atomicAdd(&acc_lo[i], xl);
         const uint32_t carry = old + xl < old ? 1u : 0u;
@@ -684,6 +712,11 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         if (xh) atomicAdd(&acc_hi[i], xh);
     };
     auto acc_get = [&](uint32_t i) { return ((unsigned long long)acc_hi[i] << 32) | acc_lo[i]; };
+    auto acc_set = [&](uint32_t i, unsigned long long v) {
+        acc_lo[i] = (uint32_t)v;
+        acc_hi[i] = (uint32_t)(v >> 32);
+    };
+#endif
     if (threadIdx.x == 0) {
         proact::wait_all(lc, p.region_in);   // (a7) previous generation is here
         nout = 0u;
@@ -712,7 +745,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         const Item it = p.g.items[k];
         const uint32_t lo = p.g.v0 + it.tile * GT, nvt = min(lo + GT, p.g.v0 + p.g.nv) - lo;
         for (uint32_t i = t; i <= nvt; i += GB) cp[i] = ld_stream_u(p.g.colptr + (lo - p.g.v0 + i), pf);
-        for (uint32_t i = t; i < nvt; i += GB) acc_lo[i] = acc_hi[i] = 0u;
+        for (uint32_t i = t; i < nvt; i += GB) acc_set(i, 0ull);
         grp_bar(grp);
         // index stream software-pipelined one round ahead (PRH_PIPE): the next round's rowidx /
         // run entries are in flight while this round's gathers are, so a round costs one L2 round
@@ -883,9 +916,7 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
             fin = last_a[grp] != 0;
             if (fin) {
                 for (uint32_t i = t; i < nvt; i += GB) {
-                    const unsigned long long v = __ldcg(&ga[i]);
-                    acc_lo[i] = (uint32_t)v;
-                    acc_hi[i] = (uint32_t)(v >> 32);
+                    acc_set(i, __ldcg(&ga[i]));
                     ga[i] = 0ull;   // ready for the next launch
                 }
                 if (t == 0) p.g.acc_cnt[it.slot] = 0;
