@@ -510,31 +510,11 @@ __device__ __forceinline__ bool split_arrive(const GraphDev &g, const Item &it, 
 // bit-reproducible for any schedule; r' = (float)((1-d)/V + d * sum) as in the oracle (R12).
 constexpr double FIX = 4611686018427387904.0;          // 2^62
 constexpr double UNFIX = 1.0 / 4611686018427387904.0;  // 2^-62
-#ifndef PROACT_PR_LIMBS   // pagerank_hot_kernel sums: 0 = two 32-bit halves (atomic + dependent carry
-#define PROACT_PR_LIMBS 0    // atomic), 1 = three limbs of fire-and-forget adds (measured 1.060 vs 1.043 ms)
-#endif
-#ifndef PROACT_PR_FIX_INT
-#define PROACT_PR_FIX_INT 0   // 1: integer rounding (bit-identical; measured no faster: 1.053 vs 1.044 ms)
-#endif
-// round(g * 2^62) to nearest, ties to even, for an fp32 contribution 0 <= g < 1 -- the value
-// __double2ll_rn((double)g * 2^62) computes, from the float's bits with integer ALU operations only
-// (no fp32 -> fp64 -> s64 conversions, which share the slower conversion pipe, per edge)
+// the fixed-point value of one fp32 contribution: round(g * 2^62), ties to even (an integer-only
+// variant from the float's bits measured no faster, profiles/r02p_pagerank_fix62_int.log)
 __device__ __forceinline__ unsigned long long fix62(float g)
 {
-#if PROACT_PR_FIX_INT
-    const uint32_t b = __float_as_uint(g);
-    const int ex = (int)(b >> 23);                      // biased exponent (sign bit 0: g >= 0)
-    if (ex == 0) return 0ull;                           // 0 and denormals: below 2^-126 * 2^62 < 1/2
-    const unsigned long long m = (b & 0x7FFFFFu) | 0x800000u;
-    const int sh = ex - 127 - 23 + 62;                  // g * 2^62 = m * 2^sh
-    if (sh >= 0) return m << sh;
-    const int r = -sh;
-    if (r > 24) return 0ull;                            // m * 2^-r < 2^24 * 2^-25 = 1/2
-    const unsigned long long q = m >> r, rem = m & ((1ull << r) - 1ull), half = 1ull << (r - 1);
-    return q + ((rem > half || (rem == half && (q & 1ull))) ? 1ull : 0ull);
-#else
     return (unsigned long long)__double2ll_rn((double)g * FIX);
-#endif
 }
 
 __global__ void __launch_bounds__(GB, PROACT_PR_MINB) pagerank_kernel(launch_ctx lc, PrParams p)
@@ -673,38 +653,13 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
     constexpr int RUN = PROACT_PRH_RUN_PR;
     if (proact::agent_dispatch(lc)) return;
     extern __shared__ uint32_t dyn[];   // [PG][CPS] colptr windows, then the hot table
-#if PROACT_PR_LIMBS
-    // the 62-bit fixed-point sums as three 20/20/24-bit limbs, each a fire-and-forget 32-bit shared
-    // RED (no returned value, no carry chain): a limb accumulator takes < 4096 adds per item (a
-    // vertex gets at most one add per warp iteration on the hub path, <= 64 at its two ends), and
-    // the top limb's total is bounded by the sum itself (< 2^64 >> 40)
-    __shared__ uint32_t acc_l0_a[PG][GT], acc_lo_a[PG][GT], acc_hi_a[PG][GT];
-    uint32_t *acc_l0 = acc_l0_a[threadIdx.x / GB];
-#else
     __shared__ uint32_t acc_lo_a[PG][GT], acc_hi_a[PG][GT];
-#endif
     __shared__ uint32_t kclaim_a[PG], last_a[PG], nout;
     const uint32_t grp = threadIdx.x / GB, t = threadIdx.x % GB;
     uint32_t *acc_lo = acc_lo_a[grp], *acc_hi = acc_hi_a[grp], *cp = dyn + grp * CPS;
     float *hot = reinterpret_cast<float *>(dyn + PG * CPS);
     const float *cin = reinterpret_cast<const float *>(lc.ctx->region[p.region_in].base);
     const uint64_t pl = pol_last(), pf = pol_first();
-#if PROACT_PR_LIMBS
-    auto acc_add = [&](uint32_t i, unsigned long long x) {
-        const uint32_t a = (uint32_t)x & 0xFFFFFu, b = (uint32_t)(x >> 20) & 0xFFFFFu, c = (uint32_t)(x >> 40);
-        if (a) atomicAdd(&acc_l0[i], a);
-        if (b) atomicAdd(&acc_lo[i], b);
-        if (c) atomicAdd(&acc_hi[i], c);
-    };
-    auto acc_get = [&](uint32_t i) {
-        return (unsigned long long)acc_l0[i] + ((unsigned long long)acc_lo[i] << 20) + ((unsigned long long)acc_hi[i] << 40);
-    };
-    auto acc_set = [&](uint32_t i, unsigned long long v) {
-        acc_l0[i] = (uint32_t)v & 0xFFFFFu;
-        acc_lo[i] = (uint32_t)(v >> 20) & 0xFFFFFu;
-        acc_hi[i] = (uint32_t)(v >> 40);
-    };
-#else
     auto acc_add = [&](uint32_t i, unsigned long long x) {
         const uint32_t xl = (uint32_t)x, old = atomicAdd(&acc_lo[i], xl);
         const uint32_t carry = old + xl < old ? 1u : 0u;
@@ -716,7 +671,6 @@ __global__ void __launch_bounds__(GB * PG, PROACT_PRH_MINB) pagerank_hot_kernel(
         acc_lo[i] = (uint32_t)v;
         acc_hi[i] = (uint32_t)(v >> 32);
     };
-#endif
     if (threadIdx.x == 0) {
         proact::wait_all(lc, p.region_in);   // (a7) previous generation is here
         nout = 0u;

@@ -90,8 +90,8 @@ constexpr int JV = PROACT_JACOBI_JV;    // float4 column groups per compute thre
 constexpr uint32_t JOS = PROACT_JACOBI_OUT_RING;   // MODE 2: output slots of JSR row strips (4 KiB each)
 constexpr int JSR = PROACT_JACOBI_SPAN_ROWS;       // rows per pushed span
 constexpr int JW = JC * 32 * 4 * JV;    // strip width in columns = 4 KiB of a row
-#ifndef PROACT_JACOBI_OUT_STORE   // output stores: 0 plain, 1 evict-first hint, 2 .cs in MODE 0
-#define PROACT_JACOBI_OUT_STORE 2
+#ifndef PROACT_JACOBI_OUT_STORE   // output stores: 0 plain, 1 st.cs in MODE 0 (an evict-first hint
+#define PROACT_JACOBI_OUT_STORE 1   // measured between the two, profiles/r02k_jacobi_store_policy.log)
 #endif
 #ifndef PROACT_JACOBI_OUT_EVICT_LAST   // G > 1: output rows evict-last until the agent has read them
 #define PROACT_JACOBI_OUT_EVICT_LAST 0
@@ -123,24 +123,15 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *b)
 {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
-#ifndef PROACT_JACOBI_WAIT_NS   // > 0: waits suspend in hardware up to this long per try (a waiting
-#define PROACT_JACOBI_WAIT_NS 0   // warp then takes no issue slots; the phase completion wakes it)
-#endif
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
 {
+    // (a suspend-time hint on this try_wait measured no different: profiles/r02k_jacobi_wait_hint.log)
     uint32_t done;
     do {
-#if PROACT_JACOBI_WAIT_NS > 0
-        asm volatile("{\n\t.reg .pred p;\n\t"
-                     "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
-                     "selp.u32 %0, 1, 0, p;\n\t}"
-                     : "=r"(done) : "r"(smem_u32(b)), "r"(parity), "n"(PROACT_JACOBI_WAIT_NS) : "memory");
-#else
         asm volatile("{\n\t.reg .pred p;\n\t"
                      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
                      "selp.u32 %0, 1, 0, p;\n\t}"
                      : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
-#endif
     } while (!done);
 }
 __device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes, uint64_t *bar)
@@ -314,7 +305,6 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
     char *outb = lc.ctx->region[p.region_out].base;
     uint64_t pol_out = 0;
     if (PROACT_JACOBI_OUT_EVICT_LAST) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_out));
-    if (PROACT_JACOBI_OUT_STORE == 1) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_out));
     uint32_t q = 0;    // next stream item (same sequence as the producer warp's)
     uint32_t kt = 0;   // tiles handed to the committer
     uint32_t oq = 0;   // MODE 2: next output span of this CTA
@@ -372,9 +362,6 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
             tpush = false;
             for (uint64_t c = a0 / Ro.chunk_bytes; c * Ro.chunk_bytes < a1 && !tpush; ++c)
                 tpush = proact::transfers(lc, Ro, (uint32_t)c);
-#if defined(PROACT_TP_EXP) && PROACT_TP_EXP == 2   // timing experiment: no staging at all
-            tpush = false;
-#endif
         }
         auto rows = [&](auto fast_tag) {
             constexpr bool FAST = decltype(fast_tag)::value;
@@ -414,9 +401,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                     }
                     const uint64_t off = ((uint64_t)i * N + j) * 4;
                     if (MODE == 2) {   // the local copy now, the span for the transfer warp
-#if !defined(PROACT_TP_EXP) || PROACT_TP_EXP != 1   // (1: timing experiment, no staging stores)
                         if (tpush) *reinterpret_cast<float4 *>(ostrip + 4 * tid + g * GW) = o;
-#endif
                         *reinterpret_cast<float4 *>(outb + off) = o;
                     } else if (!FAST && lc.mech == PROACT_MECH_INLINE) {
                         proact::put(lc, p.region_out, off, o);
@@ -425,10 +410,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                         asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
                                      ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
                     } else {
-#if PROACT_JACOBI_OUT_STORE == 1   // evict-first hint (experiment)
-                        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
-                                     ::"l"(outb + off), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w), "l"(pol_out) : "memory");
-#elif PROACT_JACOBI_OUT_STORE == 2
+#if PROACT_JACOBI_OUT_STORE == 1
                         // no agent reads this output back (MODE 0): streaming stores (st.cs), ~1 %
                         // faster under the power cap (profiles/r02k_jacobi_store_policy.log); an
                         // agent's read-back (MODE 1) wants the lines kept in L2
