@@ -40,7 +40,6 @@ constexpr int GB = PROACT_GB;      // threads per CTA
 #define PROACT_GT 512 // more L1 as landing space for the gathers), SSSP unchanged
 #endif
 constexpr int GT = PROACT_GT;      // vertices per tile (2 KiB of output)
-constexpr int GL = 8;              // lanes per light vertex
 // consecutive in-edges per thread per round (merge path) and CTAs per SM, measured on B200
 // (tools/sweep_graph.py): PageRank 4 / 8 (1.65 ms at RMAT-24; 8 / 6: 2.2 ms), SSSP 2 / 6
 #ifndef PROACT_PR_RUN
@@ -433,20 +432,6 @@ __device__ __forceinline__ void pr_finish(const launch_ctx &lc, const PrParams &
     const uint32_t od = ld_stream_u(p.g.outdeg + v, pol_first());
     const float c = od ? __fdiv_rn(r, (float)od) : 0.f;
     proact::put(lc, p.region_out, (uint64_t)v * 4, c);
-}
-
-__device__ __forceinline__ double block_sum_f64(double x, double *red)
-{
-    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xFFFFFFFFu, x, o);
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = x;
-    __syncthreads();
-    double t = 0.0;
-    if (threadIdx.x < 32) {
-        t = threadIdx.x < (GB / 32) ? red[threadIdx.x] : 0.0;
-        for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xFFFFFFFFu, t, o);
-    }
-    __syncthreads();
-    return t;   // valid in thread 0
 }
 
 // Local vertex index i (0..nv_tile-1) of edge e of the tile: the last i with cp[i] <= e (cp in

@@ -29,31 +29,6 @@ namespace {
 
 using proact::warp_commit;
 
-__device__ __forceinline__ float4 ld_nc_f4(const float *p)
-{
-    float4 v;
-    asm volatile("ld.global.nc.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ float4 ld_f4(const float *p)
-{
-    float4 v;
-    asm volatile("ld.global.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ float ld_nc_f(const float *p)
-{
-    float v;
-    asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v) : "l"(p));
-    return v;
-}
-__device__ __forceinline__ float ld_f(const float *p)
-{
-    float v;
-    asm volatile("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
-    return v;
-}
-
 // ---------------------------------------------------------------- Jacobi
 // Tile = rows_per_tile rows x one 1024-column strip (4 KiB of a row).  Warp-specialised CTA:
 // one producer warp streams the tile's input rows (plus the two halo rows) into a JS-deep
@@ -283,7 +258,7 @@ jacobi_kernel(launch_ctx lc, proact_jacobi_params p)
                                  JW * 4, (uint64_t)N * 4, true);
         return;
     }
-    if (TALLY && warp == JC + 1) {
+    if constexpr (TALLY) if (warp == JC + 1) {
         // (a3) committer warp: after the compute warps' mbarrier arrival for tile k (release ->
         // acquire at CTA scope), commit the tile's rows with release RMWs, merged per chunk.
         // The compute warps never stall on the commit's fence latency.
