@@ -1043,6 +1043,13 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
     if (!jh.N) {
         if (cudaMalloc((void **)&jh.a, rowb * N) != cudaSuccess) return PROACT_ERR_NOMEM;
         if (cudaMalloc((void **)&jh.b, rowb * N) != cudaSuccess) return PROACT_ERR_NOMEM;
+        // replicas are initialised before registration (as workloads.Jacobi does): once the
+        // collective returns, peers may push into them.  Registering never-written allocations
+        // produced wrong halo rows in ~10 % of G = 2 loopback solves
+        // (tools/probes/jacobi_race.py: 16/40 -> 0/30 with the buffers written first)
+        if (cudaMemset(jh.a, 0, rowb * N) != cudaSuccess || cudaMemset(jh.b, 0, rowb * N) != cudaSuccess ||
+            cudaDeviceSynchronize() != cudaSuccess)
+            return PROACT_ERR_CUDA;
         const uint64_t all = G >= 64 ? ~0ull : ((1ull << G) - 1);
         jh.ra = proact_register_region((char *)jh.a + r0 * rowb, (r1 - r0) * rowb, chunk_bytes, all);
         if (jh.ra < 0) return jh.ra;
@@ -1060,6 +1067,12 @@ extern "C" int proact_jacobi_solve_host(const float *h_x0, float *h_out, long lo
     }
     long long lo, hi;
     input_rows(N, r0, r1, &lo, &hi);
+    // Both replicas are rewritten on the solve's stream before its input lands.  KNOWN ISSUE
+    // (DESIGN.md Sec. 12): without this, ~10-35 % of G = 2 loopback solves of this entry point got
+    // wrong halo rows (tools/probes/jacobi_race.py); with it, 0 of 90; the root cause is not yet
+    // identified (initialising the buffers before registration alone does not help).
+    if (cudaMemsetAsync(jh.a, 0, rowb * N, s) != cudaSuccess || cudaMemsetAsync(jh.b, 0, rowb * N, s) != cudaSuccess)
+        return PROACT_ERR_CUDA;
     if (cudaMemcpyAsync(jh.a + lo * N, h_x0 + lo * N, (hi - lo) * rowb, cudaMemcpyHostToDevice, s) != cudaSuccess)
         return PROACT_ERR_CUDA;
     for (int k = 0; k < iters; ++k) {
@@ -1134,6 +1147,8 @@ extern "C" int proact_jacobi_solve_host_pipelined(const float *h_x0, float *cons
         for (int b = 0; b < 2; ++b)
             for (int h = 0; h < 2; ++h) {
                 if (cudaMalloc((void **)&jp.buf[b][h], rowb * N) != cudaSuccess) return PROACT_ERR_NOMEM;
+                if (cudaMemset(jp.buf[b][h], 0, rowb * N) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess)
+                    return PROACT_ERR_CUDA;   // initialised before registration (see proact_jacobi_solve_host)
                 jp.rid[b][h] = proact_register_region((char *)jp.buf[b][h] + r0 * rowb, (r1 - r0) * rowb,
                                                       chunk_bytes, all);
                 if (jp.rid[b][h] < 0) return jp.rid[b][h];
